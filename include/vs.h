@@ -1,0 +1,140 @@
+/*
+ * vs.h — C ABI of libvs: column-vector-sparse fp16 SpMM / SDDMM for B200 (sm_100a).
+ *
+ * Method: Chen, Qu, Liu, Ding, Xie, "Efficient Tensor Core-Based GPU Kernels for
+ * Structured Sparsity under Reduced Precision", SC'21.  "P:n" below = line n of the
+ * paper text (reference PAPER.md).
+ *
+ * Column-vector sparse encoding (§4.2, Fig. 8):
+ *   A matrix of M rows and K columns is cut into W = ceil(M/V) row windows of V rows.
+ *   Inside window w, column k is a "column vector" A[wV .. wV+V-1][k].  Only nonzero
+ *   column vectors are stored, CSR-style:
+ *     row_ptr[W+1]   int32, row_ptr[0] = 0, non-decreasing; window w owns vectors
+ *                    p in [row_ptr[w], row_ptr[w+1]).
+ *     col_idx[nnz_v] int32, the column k of vector p (the encoder emits ascending k).
+ *     vals[nnz_v*V]  fp16, vector-major: vals[p*V + r] = A[wV + r][col_idx[p]]
+ *                    ("elements within each nonzero column vector are stored in
+ *                    consecutive addresses, and the consecutive vectors in the same
+ *                    row are also consecutive").  Rows wV+r >= M of the last
+ *                    window are padding and hold +0.0.
+ *   V is 1, 2, 4 or 8 (V=1 is plain scalar CSR).
+ *
+ * General conventions (apply to every entry point):
+ *   - All matrix / index pointers are DEVICE pointers (unless a name ends in _host).
+ *     fp16 buffers are IEEE binary16 passed as void*.
+ *   - Every call is stream-ordered on `stream` (a cudaStream_t; NULL = legacy default
+ *     stream) and asynchronous, except where a phase below says it synchronises.
+ *   - Ownership: the caller allocates and frees every buffer.  The library allocates no
+ *     device memory and keeps no global mutable state except a once-initialised cache of
+ *     device attributes, so calls are thread-safe.
+ *   - Errors: argument checks run on the host before anything is enqueued.  Bad V,
+ *     negative sizes, a NULL required pointer -> VS_ERROR_INVALID_VALUE; device is not
+ *     sm_100 -> VS_ERROR_NOT_SUPPORTED; an fp16 pointer not 2-byte aligned, vals not
+ *     2-byte aligned or an int32 pointer not 4-byte aligned -> VS_ERROR_MISALIGNED;
+ *     a failed launch -> VS_ERROR_CUDA.  Faults inside kernels surface asynchronously
+ *     as in CUDA.  No C++ exception ever crosses this ABI.
+ *   - Preconditions not checked (undefined behaviour if violated): row_ptr[0] == 0 and
+ *     non-decreasing; 0 <= col_idx < K (SpMM) / < N (SDDMM); output buffers do not
+ *     alias inputs.  Kernels do not rely on col_idx order (duplicates sum in SpMM).
+ *   - Sizes are int64; indices int32 (so nnz_v < 2^31); all address arithmetic is 64-bit.
+ *   - Any M, N, K >= 0 is accepted: the fast path wants 16-byte aligned dense operands
+ *     and N % 8 == 0 (SpMM) / K % 8 == 0 (SDDMM); everything else takes a guarded path
+ *     that gives the same results.
+ *   - Arithmetic: fp16 x fp16 products accumulated in fp32 (HMMA.884.F32.F32),
+ *     results rounded to fp16 round-to-nearest-even (output precision is a reading,
+ *     DESIGN.md R1).  Results are deterministic (no atomics on outputs).
+ */
+#ifndef VS_H_
+#define VS_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* Same type as cudaStream_t (struct CUstream_st*); declared here so this header does
+   not need the CUDA headers. */
+typedef struct CUstream_st* vs_stream_t;
+
+typedef enum {
+  VS_SUCCESS = 0,
+  VS_ERROR_INVALID_VALUE = 1,
+  VS_ERROR_NOT_SUPPORTED = 2,
+  VS_ERROR_CUDA = 3,
+  VS_ERROR_MISALIGNED = 4
+} vs_status_t;
+
+/* Human-readable name of a status code (static storage, never NULL). */
+const char* vs_status_string(vs_status_t s);
+
+/* Library version as MAJOR*10000 + MINOR*100 + PATCH. */
+int vs_version(void);
+
+/*
+ * vs_encode_colvec — dense matrix or mask [M x K] -> column-vector CSR with grain V.
+ * Defined by §4.2 P:622-633 and the worked example of Fig. 8.
+ *
+ *   dense : fp16 [M x K] row-major (leading dimension K), or NULL.
+ *   mask  : uint8 [M x K] row-major, or NULL.  At least one of dense / mask is required.
+ *   Keep predicate for window w, column k:
+ *     mask != NULL : any_{r<V, wV+r<M} mask[wV+r][k] != 0
+ *     mask == NULL : any_{r<V, wV+r<M} bits(dense[wV+r][k]) != 0   (so -0.0 is kept;
+ *                    a kept vector may contain zeros, as (0,1) in Fig. 8)
+ *   row_ptr : int32 [W+1] output, W = ceil(M/V).  Always written.
+ *
+ *   Count mode (col_idx == NULL): writes row_ptr only.  If nnz_vec_host != NULL, the call
+ *     synchronises `stream` and stores nnz_v = row_ptr[W] into *nnz_vec_host.
+ *   Full mode (col_idx != NULL): writes row_ptr, col_idx[nnz_v] (ascending k inside each
+ *     window) and, if vals != NULL, vals[nnz_v*V] (requires dense != NULL; rows >= M
+ *     padded with +0.0; vals must be 2-byte aligned).  Capacity precondition: col_idx
+ *     holds >= nnz_v entries and vals >= nnz_v*V (e.g. from a previous count-mode call,
+ *     or the bound W*K).  Asynchronous unless nnz_vec_host != NULL (then it synchronises
+ *     and stores nnz_v).
+ *   M == 0 or K == 0 gives row_ptr = 0 everywhere and nnz_v = 0.
+ */
+vs_status_t vs_encode_colvec(int64_t M, int64_t K, int V,
+                             const void* dense, const uint8_t* mask,
+                             int32_t* row_ptr, int32_t* col_idx, void* vals,
+                             int64_t* nnz_vec_host, vs_stream_t stream);
+
+/*
+ * vs_spmm — C[M x N] = A[M x K] * B[K x N], A sparse in column-vector CSR.
+ * Problem statement §4.1 P:571-588 (B, C row-major; A in CSR); kernel §5.3-5.4
+ * P:846-921 (each output tile V x TileN).
+ *
+ *   row_ptr[W+1], col_idx[nnz_v], vals[nnz_v*V] : A as above, W = ceil(M/V).
+ *   B : fp16 [K x N] row-major.   C : fp16 [M x N] row-major, fully overwritten
+ *   (beta = 0; windows without vectors produce zeros).
+ *   C[i][j] = fp16_rn( sum_{p in window i/V} vals[p*V + i%V] * B[col_idx[p]][j] ),
+ *   summed in fp32.
+ *   M == 0 or N == 0: no-op.  K == 0 or nnz_v == 0: C is zero-filled.
+ */
+vs_status_t vs_spmm(int64_t M, int64_t K, int64_t N, int V,
+                    const int32_t* row_ptr, const int32_t* col_idx, const void* vals,
+                    const void* B, void* C, vs_stream_t stream);
+
+/*
+ * vs_sddmm — out = (A * B) sampled at a column-vector mask D [M x N].
+ * Problem statement §4.1 P:589-593 (C in CSR, A row-major, B column-major "to replace
+ * the transpose"); kernel §6.3-6.4; D a binary mask stored in the
+ * column-vector encoding.
+ *
+ *   row_ptr[W+1], col_idx[nnz_v] : the mask pattern over [M x N], W = ceil(M/V).
+ *   A  : fp16 [M x K] row-major.
+ *   Bt : fp16 [N x K] row-major (= the paper's column-major B [K x N]).
+ *   out_vals : fp16 [nnz_v * V], aligned with col_idx:
+ *     out_vals[p*V + r] = fp16_rn( sum_{k<K} A[wV+r][k] * Bt[col_idx[p]][k] ) for
+ *     p in window w and wV+r < M; padded rows (wV+r >= M) get +0.0.
+ *   The mask only selects positions: no scaling and no multiplication by mask values.
+ *   M == 0, N == 0 or nnz_v == 0: no-op.  K == 0: out_vals zero-filled.
+ */
+vs_status_t vs_sddmm(int64_t M, int64_t N, int64_t K, int V,
+                     const int32_t* row_ptr, const int32_t* col_idx,
+                     const void* A, const void* Bt, void* out_vals, vs_stream_t stream);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* VS_H_ */
