@@ -1,0 +1,177 @@
+"""paper_conf_sc_chenqldx21_b200 — column-vector-sparse fp16 SpMM / SDDMM for B200 (sm_100a).
+
+Thin Python binding of the C ABI in include/vs.h (libvs.so, built in-tree by _build.py).
+Argument marshalling only: torch supplies device memory and the current stream; every
+step of the path runs in the library's CUDA kernels.  There is no CPU fallback — if
+libvs.so is missing or the device is not sm_100 the calls raise.
+
+Method: Chen et al., "Efficient Tensor Core-Based GPU Kernels for Structured Sparsity
+under Reduced Precision", SC'21 (column-vector sparse encoding §4.2; SpMM §5
+P:635-921; SDDMM §6).
+
+Entry points (same names as the C ABI):
+  vs_encode_colvec(M, K, V, dense=None, mask=None, row_ptr, col_idx=None, vals=None, ...)
+  vs_spmm(M, K, N, V, row_ptr, col_idx, vals, B, C)
+  vs_sddmm(M, N, K, V, row_ptr, col_idx, A, Bt, out_vals)
+Conveniences that allocate outputs: encode(), spmm(), sddmm().
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import threading
+
+__all__ = ["VSError", "lib_path", "load", "vs_encode_colvec", "vs_spmm", "vs_sddmm",
+           "encode", "spmm", "sddmm", "num_windows"]
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+lib_path = os.path.join(_PKG, "libvs.so")
+_lib = None
+_lock = threading.Lock()
+
+_P = ctypes.c_void_p
+_I64 = ctypes.c_int64
+
+STATUS = {0: "VS_SUCCESS", 1: "VS_ERROR_INVALID_VALUE", 2: "VS_ERROR_NOT_SUPPORTED",
+          3: "VS_ERROR_CUDA", 4: "VS_ERROR_MISALIGNED"}
+
+
+class VSError(RuntimeError):
+    def __init__(self, status: int, where: str):
+        self.status = status
+        super().__init__(f"{where}: {STATUS.get(status, status)}")
+
+
+def load():
+    """Loads libvs.so (raises if it has not been built)."""
+    global _lib
+    with _lock:
+        if _lib is None:
+            if not os.path.exists(lib_path):
+                raise ImportError(f"{lib_path} is missing: run __graft_entry__.build() "
+                                  "(nvcc -gencode arch=compute_100a,code=sm_100a)")
+            L = ctypes.CDLL(lib_path)
+            L.vs_status_string.restype = ctypes.c_char_p
+            L.vs_status_string.argtypes = [ctypes.c_int]
+            L.vs_version.restype = ctypes.c_int
+            L.vs_version.argtypes = []
+            L.vs_encode_colvec.restype = ctypes.c_int
+            L.vs_encode_colvec.argtypes = [_I64, _I64, ctypes.c_int, _P, _P, _P, _P, _P,
+                                           ctypes.POINTER(ctypes.c_int64), _P]
+            L.vs_spmm.restype = ctypes.c_int
+            L.vs_spmm.argtypes = [_I64, _I64, _I64, ctypes.c_int, _P, _P, _P, _P, _P, _P]
+            L.vs_sddmm.restype = ctypes.c_int
+            L.vs_sddmm.argtypes = [_I64, _I64, _I64, ctypes.c_int, _P, _P, _P, _P, _P, _P]
+            _lib = L
+    return _lib
+
+
+def _check(st: int, where: str):
+    if st != 0:
+        raise VSError(st, where)
+
+
+def _stream(stream):
+    import torch
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return ctypes.c_void_p(stream.cuda_stream)
+
+
+def _ptr(t, dtype=None, name="tensor"):
+    """Device pointer of a contiguous CUDA tensor (None -> NULL)."""
+    if t is None:
+        return None
+    import torch
+    if not isinstance(t, torch.Tensor) or not t.is_cuda:
+        raise TypeError(f"{name} must be a CUDA tensor")
+    if dtype is not None and t.dtype != dtype:
+        raise TypeError(f"{name} must be {dtype}, got {t.dtype}")
+    if not t.is_contiguous():
+        raise ValueError(f"{name} must be contiguous")
+    return ctypes.c_void_p(t.data_ptr()) if t.numel() > 0 else None
+
+
+def num_windows(M: int, V: int) -> int:
+    return -(-int(M) // int(V)) if M > 0 else 0
+
+
+# ------------------------------------------------------------------ C-ABI mirrors
+
+def vs_encode_colvec(M, K, V, dense=None, mask=None, row_ptr=None, col_idx=None, vals=None,
+                     want_nnz=False, stream=None):
+    """Mirror of vs_encode_colvec.  Count mode when col_idx is None.  Returns nnz_v when
+    ``want_nnz`` (the call then synchronises the stream), else None."""
+    import torch
+    nnz = ctypes.c_int64(-1)
+    st = load().vs_encode_colvec(
+        int(M), int(K), int(V), _ptr(dense, torch.float16, "dense"),
+        _ptr(mask, torch.uint8, "mask"), _ptr(row_ptr, torch.int32, "row_ptr"),
+        _ptr(col_idx, torch.int32, "col_idx"), _ptr(vals, torch.float16, "vals"),
+        ctypes.byref(nnz) if want_nnz else None, _stream(stream))
+    _check(st, "vs_encode_colvec")
+    return int(nnz.value) if want_nnz else None
+
+
+def vs_spmm(M, K, N, V, row_ptr, col_idx, vals, B, C, stream=None):
+    import torch
+    st = load().vs_spmm(int(M), int(K), int(N), int(V), _ptr(row_ptr, torch.int32, "row_ptr"),
+                        _ptr(col_idx, torch.int32, "col_idx"), _ptr(vals, torch.float16, "vals"),
+                        _ptr(B, torch.float16, "B"), _ptr(C, torch.float16, "C"), _stream(stream))
+    _check(st, "vs_spmm")
+
+
+def vs_sddmm(M, N, K, V, row_ptr, col_idx, A, Bt, out_vals, stream=None):
+    import torch
+    st = load().vs_sddmm(int(M), int(N), int(K), int(V), _ptr(row_ptr, torch.int32, "row_ptr"),
+                         _ptr(col_idx, torch.int32, "col_idx"), _ptr(A, torch.float16, "A"),
+                         _ptr(Bt, torch.float16, "Bt"), _ptr(out_vals, torch.float16, "out_vals"),
+                         _stream(stream))
+    _check(st, "vs_sddmm")
+
+
+# ------------------------------------------------------------------ conveniences
+
+def encode(V, dense=None, mask=None, capacity=None, stream=None):
+    """Encodes ``dense`` (fp16 [M,K]) and/or ``mask`` (uint8 [M,K]) with grain V.
+    Returns (row_ptr, col_idx, vals) (vals None for a mask-only call).
+
+    Without ``capacity`` a count-mode call sizes the outputs (one stream sync).  With a
+    capacity (>= nnz_v, e.g. W*K) the encode is a single asynchronous call and the outputs
+    are returned at full capacity length; row_ptr[-1] holds nnz_v."""
+    import torch
+    src = dense if dense is not None else mask
+    M, K = src.shape
+    W = num_windows(M, V)
+    dev = src.device
+    row_ptr = torch.empty(W + 1, dtype=torch.int32, device=dev)
+    if capacity is None:
+        capacity = vs_encode_colvec(M, K, V, dense, mask, row_ptr, want_nnz=True, stream=stream)
+    col_idx = torch.empty(int(capacity), dtype=torch.int32, device=dev)
+    vals = torch.empty(int(capacity) * V, dtype=torch.float16, device=dev) if dense is not None else None
+    # with capacity 0 there is nothing to write: still produce row_ptr
+    vs_encode_colvec(M, K, V, dense, mask, row_ptr,
+                     col_idx if capacity > 0 else None, vals if capacity > 0 else None,
+                     stream=stream)
+    return row_ptr, col_idx, vals
+
+
+def spmm(row_ptr, col_idx, vals, B, M, V, out=None, stream=None):
+    """C[M,N] = A * B for A = (row_ptr, col_idx, vals) with grain V."""
+    import torch
+    K, N = B.shape
+    C = out if out is not None else torch.empty((M, N), dtype=torch.float16, device=B.device)
+    vs_spmm(M, K, N, V, row_ptr, col_idx, vals, B, C, stream=stream)
+    return C
+
+
+def sddmm(row_ptr, col_idx, A, Bt, V, nnz=None, out=None, stream=None):
+    """out_vals = (A Bt^T) sampled at the mask (row_ptr, col_idx); A [M,K], Bt [N,K]."""
+    import torch
+    M, K = A.shape
+    N = Bt.shape[0]
+    if out is None:
+        n = int(row_ptr[-1].item()) if nnz is None else int(nnz)
+        out = torch.empty(n * V, dtype=torch.float16, device=A.device)
+    vs_sddmm(M, N, K, V, row_ptr, col_idx, A, Bt, out, stream=stream)
+    return out

@@ -1,0 +1,138 @@
+// vs_api.cu — the C ABI of include/vs.h: argument checks, dispatch, launch status.
+// No exception crosses this boundary; every entry point returns a vs_status_t.
+#include <mutex>
+
+#include "../../include/vs.h"
+#include "common.cuh"
+
+namespace vs {
+cudaError_t launch_encode(int64_t M, int64_t K, int V, const void* dense, const uint8_t* mask,
+                          int32_t* row_ptr, int32_t* col_idx, void* vals, cudaStream_t s);
+cudaError_t launch_spmm(int64_t M, int64_t K, int64_t N, int V, const int32_t* row_ptr,
+                        const int32_t* col_idx, const void* vals, const void* B, void* C,
+                        cudaStream_t s);
+cudaError_t launch_sddmm(int64_t M, int64_t N, int64_t K, int V, const int32_t* row_ptr,
+                         const int32_t* col_idx, const void* A, const void* Bt, void* out,
+                         int num_sms, cudaStream_t s);
+}  // namespace vs
+
+namespace {
+
+constexpr int kMaxDevices = 64;
+struct DevInfo {
+  int ok;  // 1 = sm_100, 0 = other
+  int num_sms;
+};
+DevInfo g_dev[kMaxDevices];
+std::once_flag g_dev_once[kMaxDevices];
+
+// Device attributes of the current device, queried once per device.
+bool device_info(DevInfo* out) {
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= kMaxDevices) return false;
+  std::call_once(g_dev_once[dev], [dev] {
+    int major = 0, minor = 0, sms = 0;
+    cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev);
+    cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    g_dev[dev].ok = (major == 10 && minor == 0) ? 1 : 0;
+    g_dev[dev].num_sms = sms > 0 ? sms : 148;
+  });
+  *out = g_dev[dev];
+  return true;
+}
+
+bool valid_v(int V) { return V == 1 || V == 2 || V == 4 || V == 8; }
+bool al(const void* p, uintptr_t a) { return (reinterpret_cast<uintptr_t>(p) & (a - 1)) == 0; }
+
+vs_status_t from_cuda(cudaError_t e) { return e == cudaSuccess ? VS_SUCCESS : VS_ERROR_CUDA; }
+
+vs_status_t check_device(DevInfo* info) {
+  if (!device_info(info)) return VS_ERROR_CUDA;
+  return info->ok ? VS_SUCCESS : VS_ERROR_NOT_SUPPORTED;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* vs_status_string(vs_status_t s) {
+  switch (s) {
+    case VS_SUCCESS: return "VS_SUCCESS";
+    case VS_ERROR_INVALID_VALUE: return "VS_ERROR_INVALID_VALUE";
+    case VS_ERROR_NOT_SUPPORTED: return "VS_ERROR_NOT_SUPPORTED";
+    case VS_ERROR_CUDA: return "VS_ERROR_CUDA";
+    case VS_ERROR_MISALIGNED: return "VS_ERROR_MISALIGNED";
+  }
+  return "VS_ERROR_UNKNOWN";
+}
+
+int vs_version(void) { return 100; /* 0.1.0 */ }
+
+vs_status_t vs_encode_colvec(int64_t M, int64_t K, int V, const void* dense, const uint8_t* mask,
+                             int32_t* row_ptr, int32_t* col_idx, void* vals,
+                             int64_t* nnz_vec_host, vs_stream_t stream) {
+  if (!valid_v(V) || M < 0 || K < 0) return VS_ERROR_INVALID_VALUE;
+  if (dense == nullptr && mask == nullptr) return VS_ERROR_INVALID_VALUE;
+  if (row_ptr == nullptr) return VS_ERROR_INVALID_VALUE;
+  if (vals != nullptr && dense == nullptr) return VS_ERROR_INVALID_VALUE;
+  if (!al(row_ptr, 4) || (col_idx && !al(col_idx, 4))) return VS_ERROR_MISALIGNED;
+  if ((dense && !al(dense, 2)) || (vals && !al(vals, 2))) return VS_ERROR_MISALIGNED;
+  DevInfo info;
+  vs_status_t st = check_device(&info);
+  if (st != VS_SUCCESS) return st;
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  const int64_t W = vs::ceil_div64(M, V);
+  if (W == 0) {
+    // row_ptr = [0]
+    if (cudaMemsetAsync(row_ptr, 0, sizeof(int32_t), s) != cudaSuccess) return VS_ERROR_CUDA;
+  } else {
+    cudaError_t e = vs::launch_encode(M, K, V, dense, mask, row_ptr, col_idx, vals, s);
+    if (e != cudaSuccess) return VS_ERROR_CUDA;
+  }
+  if (nnz_vec_host != nullptr) {
+    int32_t nnz = 0;
+    if (cudaMemcpyAsync(&nnz, row_ptr + W, sizeof(int32_t), cudaMemcpyDeviceToHost, s) !=
+        cudaSuccess)
+      return VS_ERROR_CUDA;
+    if (cudaStreamSynchronize(s) != cudaSuccess) return VS_ERROR_CUDA;
+    *nnz_vec_host = nnz;
+  }
+  return VS_SUCCESS;
+}
+
+vs_status_t vs_spmm(int64_t M, int64_t K, int64_t N, int V, const int32_t* row_ptr,
+                    const int32_t* col_idx, const void* vals, const void* B, void* C,
+                    vs_stream_t stream) {
+  if (!valid_v(V) || M < 0 || K < 0 || N < 0) return VS_ERROR_INVALID_VALUE;
+  if (M == 0 || N == 0) return VS_SUCCESS;
+  // col_idx / vals / B may be NULL only when they are never read (nnz_v == 0 or K == 0)
+  if (row_ptr == nullptr || C == nullptr) return VS_ERROR_INVALID_VALUE;
+  if (!al(row_ptr, 4) || (col_idx && !al(col_idx, 4))) return VS_ERROR_MISALIGNED;
+  if ((vals && !al(vals, 2)) || (B && !al(B, 2)) || !al(C, 2)) return VS_ERROR_MISALIGNED;
+  DevInfo info;
+  vs_status_t st = check_device(&info);
+  if (st != VS_SUCCESS) return st;
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  if (K == 0) return from_cuda(cudaMemsetAsync(C, 0, (size_t)(M * N) * 2, s));
+  return from_cuda(vs::launch_spmm(M, K, N, V, row_ptr, col_idx, vals, B, C, s));
+}
+
+vs_status_t vs_sddmm(int64_t M, int64_t N, int64_t K, int V, const int32_t* row_ptr,
+                     const int32_t* col_idx, const void* A, const void* Bt, void* out_vals,
+                     vs_stream_t stream) {
+  if (!valid_v(V) || M < 0 || K < 0 || N < 0) return VS_ERROR_INVALID_VALUE;
+  if (M == 0 || N == 0) return VS_SUCCESS;
+  // col_idx / A / Bt / out_vals may be NULL only when never touched (nnz_v == 0)
+  if (row_ptr == nullptr) return VS_ERROR_INVALID_VALUE;
+  if (!al(row_ptr, 4) || (col_idx && !al(col_idx, 4))) return VS_ERROR_MISALIGNED;
+  if ((A && !al(A, 2)) || (Bt && !al(Bt, 2)) || (out_vals && !al(out_vals, 2)))
+    return VS_ERROR_MISALIGNED;
+  DevInfo info;
+  vs_status_t st = check_device(&info);
+  if (st != VS_SUCCESS) return st;
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  return from_cuda(vs::launch_sddmm(M, N, K, V, row_ptr, col_idx, A, Bt, out_vals, info.num_sms, s));
+}
+
+}  // extern "C"
