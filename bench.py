@@ -1,0 +1,682 @@
+#!/usr/bin/env python
+"""bench.py — throughput of the column-vector-sparse hot path on B200.
+
+One STEP = one pass of the whole hot path (encode -> SpMM -> SDDMM) over the
+workload's batch of synthetic layer problems (synth/workloads.py).  Per problem:
+  vs_encode_colvec(W dense)                         -> (row_ptr, col_idx, vals)   [a1]
+  vs_spmm(W, X)            Y  [M x N] = W X          (§5)            [a2-a6]
+  vs_sddmm(pattern W; G, X) dW = (G X^T) o pattern   (§6)           [a7-a10]
+(the forward / weight-gradient pair of P:1625-1633; SDDMM inner dimension = N).
+
+metric = effective TFLOP/s = (2*nnz*N [SpMM] + 2*nnz*N [SDDMM]) / step time, nnz = stored
+scalars (nnz_v * V), summed over all problems and all ranks, divided by the max over ranks
+of the step time (device time, CUDA events).  The step is replayed as one CUDA graph; the
+L2 is flushed (512 MiB write) between timed steps and the flush is not timed.
+
+Also reported: per-kernel-class device time (events inside an instrumented graph), the
+roofline of the dominant kernel, end-to-end throughput with host buffers (H2D + D2H inside
+the timed region), the fp64 oracle on the host cores (cpu_baseline), same-box cuBLAS Hgemm /
+GemmEx and cuSPARSE speedups per cell, and SM clocks sampled during the timed region.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                  [--workload dlmc_layer|rn50_layer|c1] [--no-baselines] [--no-cpu]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+METRIC = "SpMM/SDDMM effective TFLOP/s & speedup vs cuBLAS Hgemm, V=2/4/8, 50–98% sparse"
+UNIT = "TFLOP/s"
+DEFAULT_WORKLOAD = "dlmc_layer"
+
+
+def parse_args(argv=None):
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--workload", default=DEFAULT_WORKLOAD)
+    ap.add_argument("--no-baselines", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--reps", type=int, default=20, help="launches per per-cell micro timing")
+    ap.add_argument("--detail", default=os.path.join(ROOT, "gpurun_out", "bench_detail.json"))
+    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--streams", type=int, default=8,
+                    help="concurrent graph branches across independent problems")
+    return ap.parse_args(argv)
+
+
+# ----------------------------------------------------------------------- helpers
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return {"hbm_gbs": d["hbm_gbs"], "bf16_tflops": d["bf16_tflops"],
+                "bf16_tflops_sustained": d.get("bf16_tflops_sustained", d["bf16_tflops"]),
+                "source": "measured (MEASURED_PEAKS.json)"}
+    return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0,
+            "source": "fallback (B200_PROFILING.md)"}
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons every 200 ms while the timed region runs."""
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+    NAMES = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+
+    def __init__(self, device_index: int):
+        self.dev = device_index
+        self.rows = []
+        self.proc = None
+        self.thread = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                 "-lms", "200", "-i", str(self.dev)],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except (OSError, FileNotFoundError):
+            self.proc = None
+            return self
+        self.thread = threading.Thread(target=self._read, daemon=True)
+        self.thread.start()
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) >= 9:
+                self.rows.append(parts)
+
+    def stop(self):
+        if self.proc is not None:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+        if self.thread is not None:
+            self.thread.join(timeout=2)
+        sm = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in self.rows if r[2].replace(".", "").isdigit()]
+        reasons = set()
+        for r in self.rows:
+            for name, v in zip(self.NAMES, r[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(name)
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def dist_env():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def problem_flops(nnz_v, p):
+    nnz = nnz_v * p.V
+    return 2.0 * nnz * p.N, 2.0 * nnz * p.N  # SpMM, SDDMM (inner dimension N)
+
+
+def alg_bytes(p, nnz_v, k_ref):
+    """Algorithmic HBM bytes per launch."""
+    W = -(-p.M // p.V)
+    spmm = 4 * (W + 1) + nnz_v * (4 + 2 * p.V) + 2 * k_ref * p.N + 2 * p.M * p.N
+    sddmm = 4 * (W + 1) + 4 * nnz_v + 2 * p.M * p.N + 2 * k_ref * p.N + 2 * nnz_v * p.V
+    encode = 2 * p.M * p.K + 4 * (W + 1) + nnz_v * (4 + 2 * p.V)
+    return {"encode": encode, "spmm": spmm, "sddmm": sddmm}
+
+
+# --------------------------------------------------------------- reference (oracle) arm
+
+_INPUT_CACHE = {}
+
+
+def layer_inputs(p):
+    """Seeded host inputs of one layer problem (W dense, X, G), memoised."""
+    from synth import gen
+    if p.id not in _INPUT_CACHE:
+        rng = gen.make_rng(p.id)
+        Wd = gen.colvec_dense(rng, p.M, p.K, p.V, 1.0 - p.S, kind=p.kind)
+        X = gen.dense_operand(rng, p.K, p.N)
+        G = gen.dense_operand(rng, p.M, p.N)
+        _INPUT_CACHE[p.id] = (Wd, X, G)
+    return _INPUT_CACHE[p.id]
+
+
+def oracle_sample_run(problems, seconds):
+    """Runs the fp64 oracle (encode + SpMM + SDDMM) over problems in order until ~seconds of
+    CPU work; returns (flops, elapsed, n_problems)."""
+    import oracle
+    flops, t_used, n = 0.0, 0.0, 0
+    for p in problems:
+        Wd, X, G = layer_inputs(p)
+        t0 = time.perf_counter()
+        rp, ci, va = oracle.encode(p.M, p.K, p.V, dense=Wd)
+        oracle.spmm(p.M, p.K, p.N, p.V, rp, ci, va, X)
+        oracle.sddmm(p.M, p.K, p.N, p.V, rp, ci, G, X)
+        t_used += time.perf_counter() - t0
+        f1, f2 = problem_flops(int(rp[-1]), p)
+        flops += f1 + f2
+        n += 1
+        if t_used >= seconds:
+            break
+    return flops, t_used, n
+
+
+def sample_order(problems):
+    """Deterministic interleaving so a bounded sample spans shapes, V and S."""
+    return problems[::7] + [p for i, p in enumerate(problems) if i % 7]
+
+
+def run_reference(args):
+    ws, rank, _ = dist_env()
+    if rank != 0:
+        return 0
+    import oracle
+    from synth.workloads import WORKLOADS
+    problems = sample_order(WORKLOADS[args.workload]())
+    per_step = max(2.0, min(20.0, 150.0 / max(1, args.steps + args.warmup)))
+    for _ in range(args.warmup):
+        oracle_sample_run(problems, per_step)
+    vals, tot_t, tot_f, nprob = [], 0.0, 0.0, 0
+    for _ in range(args.steps):
+        f, t, n = oracle_sample_run(problems, per_step)
+        vals.append(f / t / 1e12)
+        tot_t += t
+        tot_f += f
+        nprob = n
+    value = tot_f / tot_t / 1e12
+    cores = oracle.num_threads()
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT,
+        "n_gpus": ws, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": 1e3 * tot_t / max(1, args.steps), "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": args.workload, "sample": f"first {nprob} problems of the "
+                   "interleaved workload order per step"},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
+                         "sample": f"{nprob} problems (~{per_step:.0f} s of fp64 oracle work) per step"},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------------ our arm
+
+class LayerBuffers:
+    """Device (and pinned host) buffers of one layer problem."""
+
+    def __init__(self, p, torch, dev, with_host: bool):
+        self.p = p
+        Wd, X, G = layer_inputs(p)
+        self.W = -(-p.M // p.V)
+        self.cap = self.W * p.K
+        self.Wd = torch.from_numpy(Wd).to(dev)
+        self.X = torch.from_numpy(X).to(dev)
+        self.G = torch.from_numpy(G).to(dev)
+        self.row_ptr = torch.zeros(self.W + 1, dtype=torch.int32, device=dev)
+        self.col_idx = torch.zeros(self.cap, dtype=torch.int32, device=dev)
+        self.vals = torch.zeros(self.cap * p.V, dtype=torch.float16, device=dev)
+        self.Y = torch.zeros((p.M, p.N), dtype=torch.float16, device=dev)
+        self.dW = torch.zeros(self.cap * p.V, dtype=torch.float16, device=dev)
+        if with_host:
+            self.h_Wd = torch.from_numpy(Wd).pin_memory()
+            self.h_X = torch.from_numpy(X).pin_memory()
+            self.h_G = torch.from_numpy(G).pin_memory()
+            self.h_Y = torch.empty((p.M, p.N), dtype=torch.float16).pin_memory()
+            self.h_dW = None  # sized after the first encode
+        self.nnz_v = None
+        self.k_ref = None
+
+    # the three ABI calls of one problem
+    def encode(self, vs):
+        p = self.p
+        vs.vs_encode_colvec(p.M, p.K, p.V, self.Wd, None, self.row_ptr, self.col_idx, self.vals)
+
+    def spmm(self, vs):
+        p = self.p
+        vs.vs_spmm(p.M, p.K, p.N, p.V, self.row_ptr, self.col_idx, self.vals, self.X, self.Y)
+
+    def sddmm(self, vs):
+        p = self.p
+        vs.vs_sddmm(p.M, p.K, p.N, p.V, self.row_ptr, self.col_idx, self.G, self.X, self.dW)
+
+
+def capture(torch, fn, stream):
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=stream):
+        fn()
+    return g
+
+
+def time_graph(torch, g, stream, reps=1):
+    s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with torch.cuda.stream(stream):
+        s.record()
+        for _ in range(reps):
+            g.replay()
+        e.record()
+    e.synchronize()
+    return s.elapsed_time(e) / reps
+
+
+def run_ours(args):
+    import numpy as np
+    import torch
+    import paper_conf_sc_chenqldx21_b200 as vs
+    from synth.workloads import WORKLOADS
+
+    ws, rank, local = dist_env()
+    assert ws == args.gpus or ws == 1, f"--gpus {args.gpus} but WORLD_SIZE={ws}"
+    if ws > 1:
+        import torch.distributed as dist
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    else:
+        torch.cuda.set_device(0)
+    dev = torch.device("cuda", torch.cuda.current_device())
+    vs.load()
+    peaks = load_peaks()
+    problems = WORKLOADS[args.workload]()
+    stream = torch.cuda.Stream()
+    bufs = [LayerBuffers(p, torch, dev, with_host=not args.no_e2e) for p in problems]
+
+    # eager pass: sizes (nnz_v, referenced columns) and a sanity check of the launch path
+    with torch.cuda.stream(stream):
+        for b in bufs:
+            b.encode(vs)
+            b.spmm(vs)
+            b.sddmm(vs)
+    stream.synchronize()
+    for b in bufs:
+        b.nnz_v = int(b.row_ptr[-1].item())
+        ci = b.col_idx[:b.nnz_v].cpu().numpy()
+        b.k_ref = int(np.unique(ci).size)
+        if not args.no_e2e:
+            b.h_dW = torch.empty(b.nnz_v * b.p.V, dtype=torch.float16).pin_memory()
+
+    flops_spmm = sum(problem_flops(b.nnz_v, b.p)[0] for b in bufs)
+    flops_sddmm = sum(problem_flops(b.nnz_v, b.p)[1] for b in bufs)
+    flops_step = flops_spmm + flops_sddmm
+    launches_per_step = len(bufs) * 3  # encode_fused (+ one memset node), spmm, sddmm
+
+    def step_serial():
+        for b in bufs:
+            b.encode(vs)
+            b.spmm(vs)
+            b.sddmm(vs)
+
+    branches = [torch.cuda.Stream() for _ in range(max(1, args.streams))]
+
+    def forked(body):
+        """Runs body(b) for every problem, problem i on branch i % S (independent problems
+        become parallel branches of the captured graph)."""
+        def run():
+            cur = torch.cuda.current_stream()
+            for st in branches:
+                st.wait_stream(cur)
+            for i, b in enumerate(bufs):
+                with torch.cuda.stream(branches[i % len(branches)]):
+                    body(b)
+            for st in branches:
+                cur.wait_stream(st)
+        return run
+
+    def body(b):
+        b.encode(vs)
+        b.spmm(vs)
+        b.sddmm(vs)
+
+    step = forked(body)
+
+    # instrumented copy of the step: external events around every ABI call
+    ev = []
+
+    def step_instr():
+        for b in bufs:
+            row = []
+            for name, fn in (("encode", b.encode), ("spmm", b.spmm), ("sddmm", b.sddmm)):
+                s = torch.cuda.Event(enable_timing=True, external=True)
+                e = torch.cuda.Event(enable_timing=True, external=True)
+                s.record()
+                fn(vs)
+                e.record()
+                row.append((name, s, e))
+            ev.append(row)
+
+    g_step = capture(torch, step, stream)
+    g_serial = capture(torch, step_serial, stream)
+    g_instr = capture(torch, step_instr, stream)
+    flush = torch.empty(512 * 1024 * 1024 // 4, dtype=torch.int32, device=dev)
+
+    for i in range(args.warmup):
+        with torch.cuda.stream(stream):
+            flush.fill_(i)
+            g_step.replay()
+            g_serial.replay()
+            g_instr.replay()
+    stream.synchronize()
+
+    # ---------------- timed region (max over ranks) ----------------
+    if ws > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    clocks = ClockSampler(dev.index if ws == 1 else local).start()
+    step_ms = []
+    starts = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    ends = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    with torch.cuda.stream(stream):
+        for i in range(args.steps):
+            flush.fill_(i + 1)           # L2 flush, not timed
+            starts[i].record()
+            g_step.replay()
+            ends[i].record()
+    torch.cuda.synchronize()
+    step_ms = [s.elapsed_time(e) for s, e in zip(starts, ends)]
+    serial_ms = []
+    for i in range(args.steps):
+        with torch.cuda.stream(stream):
+            flush.fill_(i + 5)
+        serial_ms.append(time_graph(torch, g_serial, stream))
+    # instrumented replays (same inputs) for the per-kernel attribution
+    per_class = {"encode": [], "spmm": [], "sddmm": []}
+    per_launch = []
+    for i in range(args.steps):
+        with torch.cuda.stream(stream):
+            flush.fill_(i + 7)
+            g_instr.replay()
+        stream.synchronize()
+        row_ms = []
+        for b, row in zip(bufs, ev):
+            d = {name: s.elapsed_time(e) for name, s, e in row}
+            for k, v in d.items():
+                per_class[k].append(v)
+            row_ms.append(d)
+        per_launch.append(row_ms)
+    if ws > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    clk = clocks.stop()
+
+    total_ms = sum(step_ms)
+    if ws > 1:
+        t = torch.tensor([total_ms], device=dev, dtype=torch.float64)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        total_ms = float(t.item())
+    ms_per_step = total_ms / args.steps
+    value = ws * flops_step / (ms_per_step * 1e-3) / 1e12
+    ms_serial = sum(serial_ms) / args.steps
+
+    # ---------------- kernel attribution + roofline ----------------
+    nb = len(bufs)
+    cls_ms = {k: sum(v) / args.steps for k, v in per_class.items()}
+    instr_total = sum(cls_ms.values())
+    dominant = max(("spmm", "sddmm", "encode"), key=lambda k: cls_ms[k])
+    bytes_cls = {"encode": 0.0, "spmm": 0.0, "sddmm": 0.0}
+    for b in bufs:
+        for k, v in alg_bytes(b.p, b.nnz_v, b.k_ref).items():
+            bytes_cls[k] += v
+    flops_cls = {"encode": 0.0, "spmm": flops_spmm, "sddmm": flops_sddmm}
+    dom_avg_ms = cls_ms[dominant] / nb
+    achieved_gbs = (bytes_cls[dominant] / nb) / (dom_avg_ms * 1e-3) / 1e9
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tp):
+        traffic = json.load(open(tp)).get(f"{args.workload}:{dominant}")
+    roofline = {"bound": "hbm", "achieved": achieved_gbs, "peak": peaks["hbm_gbs"],
+                "unit": "GB/s", "frac": achieved_gbs / peaks["hbm_gbs"], "traffic": traffic,
+                "kernel": dominant, "peak_source": peaks["source"],
+                "algorithmic_bytes_per_launch": bytes_cls[dominant] / nb,
+                "avg_launch_us": dom_avg_ms * 1e3}
+    tensor_tf = (flops_cls[dominant] / nb) / (dom_avg_ms * 1e-3) / 1e12 if flops_cls[dominant] else 0.0
+    roofline_tensor = {"bound": "tensor", "achieved": tensor_tf, "peak": peaks["bf16_tflops"],
+                       "unit": "TFLOP/s", "frac": tensor_tf / peaks["bf16_tflops"],
+                       "kernel": dominant}
+
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": ws, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "f16", "data": "synthetic",
+        "config": {"workload": args.workload, "problems": nb,
+                   "shapes": "(M,K) in {(512,512),(2048,512),(512,2048),(2048,1024)} x V{2,4,8} "
+                             "x S{.5,.7,.9,.98} x N{64,128,256}" if args.workload == "dlmc_layer" else args.workload,
+                   "step": "per problem: encode W -> SpMM Y=WX -> SDDMM dW=(G X^T) o pattern(W)",
+                   "flops_per_step": flops_step, "l2": "flushed between timed steps (512 MiB write, untimed)",
+                   "launch": f"step replayed as one CUDA graph with {len(branches)} concurrent "
+                             "branches over the independent problems",
+                   "accumulate": "fp32"},
+        "serial": {"ms_per_step": ms_serial, "value": ws * flops_step / (ms_serial * 1e-3) / 1e12,
+                   "note": "same step as one serial graph (no cross-problem concurrency)"},
+        "roofline": roofline,
+        "roofline_tensor": roofline_tensor,
+        "kernels": {k: {"ms_per_step": v, "share": (v / instr_total if instr_total else None),
+                        "tflops": (flops_cls[k] / (v * 1e-3) / 1e12 if v and flops_cls[k] else None)}
+                    for k, v in cls_ms.items()},
+        "gpu_launches": launches_per_step * args.steps,
+        "clocks": clk,
+    }
+
+    detail = {"problems": [], "step_ms": step_ms}
+    for b in bufs:
+        detail["problems"].append({**b.p.asdict(), "nnz_v": b.nnz_v, "k_ref": b.k_ref})
+    for j in range(nb):
+        for k in ("encode", "spmm", "sddmm"):
+            detail["problems"][j][f"{k}_us"] = 1e3 * statistics.median(
+                per_launch[i][j][k] for i in range(args.steps))
+
+    # ---------------- end to end with host buffers ----------------
+    if not args.no_e2e:
+        def body_e2e(b):
+            b.Wd.copy_(b.h_Wd, non_blocking=True)
+            b.X.copy_(b.h_X, non_blocking=True)
+            b.G.copy_(b.h_G, non_blocking=True)
+            b.encode(vs)
+            b.spmm(vs)
+            b.sddmm(vs)
+            b.h_Y.copy_(b.Y, non_blocking=True)
+            b.h_dW.copy_(b.dW[:b.nnz_v * b.p.V], non_blocking=True)
+        g_e2e = capture(torch, forked(body_e2e), stream)
+        with torch.cuda.stream(stream):
+            g_e2e.replay()
+        stream.synchronize()
+        e2e_ms = []
+        for i in range(args.steps):
+            with torch.cuda.stream(stream):
+                flush.fill_(i + 3)
+            e2e_ms.append(time_graph(torch, g_e2e, stream))
+        e2e_total = sum(e2e_ms)
+        if ws > 1:
+            t = torch.tensor([e2e_total], device=dev, dtype=torch.float64)
+            torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+            e2e_total = float(t.item())
+        h2d = sum(2 * (b.p.M * b.p.K + b.p.K * b.p.N + b.p.M * b.p.N) for b in bufs)
+        d2h = sum(2 * (b.p.M * b.p.N + b.nnz_v * b.p.V) for b in bufs)
+        line["e2e"] = {"value": ws * flops_step / (e2e_total / args.steps * 1e-3) / 1e12,
+                       "unit": UNIT, "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+                       "ms_per_step": e2e_total / args.steps,
+                       "path": "pinned host -> device copies, C-ABI calls, device -> pinned host, one CUDA graph"}
+
+    # ---------------- same-box library baselines, per cell ----------------
+    if not args.no_baselines and rank == 0:
+        try:
+            line.update(library_baselines(args, torch, vs, bufs, stream, detail))
+        except Exception as exc:  # baselines are context; never fail the bench on them
+            line["baselines_error"] = repr(exc)[:300]
+
+    # ---------------- CPU oracle baseline ----------------
+    if not args.no_cpu and rank == 0 and ws == 1:
+        import oracle
+        f, t, n = oracle_sample_run(sample_order(problems), args.cpu_seconds)
+        line["cpu_baseline"] = {"value": f / t / 1e12, "unit": UNIT, "cores": oracle.num_threads(),
+                                "kind": "oracle",
+                                "sample": f"{n} of {nb} problems (encode+SpMM+SDDMM, fp64 C oracle, "
+                                          f"{t:.1f} s), interleaved order"}
+    if rank == 0:
+        os.makedirs(os.path.dirname(args.detail), exist_ok=True)
+        json.dump(detail, open(args.detail, "w"), indent=1)
+        print(json.dumps(line), flush=True)
+    if ws > 1:
+        torch.distributed.destroy_process_group()
+    return 0
+
+
+def geomean(xs):
+    xs = [x for x in xs if x and x > 0 and math.isfinite(x)]
+    return math.exp(sum(math.log(x) for x in xs) / len(xs)) if xs else None
+
+
+def library_baselines(args, torch, vs, bufs, stream, detail):
+    """Per-cell micro timings (each implementation captured as a graph of `reps` launches,
+    L2 warm, same protocol for all): ours SpMM / SDDMM vs cublasHgemm / GemmEx on the dense
+    M x K x N problem, cusparseSpMM (Blocked-ELL, CSR) and cusparseSDDMM (CSR)."""
+    import numpy as np
+    import baselines
+    from synth import gen
+    L = baselines.lib()
+    h = L.bl_create()
+    reps = args.reps
+    sptr = stream.cuda_stream
+    cells = {}
+    for j, b in enumerate(bufs):
+        p = b.p
+        d = detail["problems"][j]
+        Cd = torch.empty((p.M, p.N), dtype=torch.float16, device=b.X.device)
+
+        def rep(fn):
+            with torch.cuda.stream(stream):
+                fn()  # eager warm-up (library workspaces are set up outside capture)
+            stream.synchronize()
+
+            def run():
+                for _ in range(reps):
+                    fn()
+            g = capture(torch, run, stream)
+            with torch.cuda.stream(stream):
+                g.replay()
+            return 1e3 * time_graph(torch, g, stream, reps=3) / reps  # us per launch
+
+        t_spmm = rep(lambda: b.spmm(vs))
+        t_sddmm = rep(lambda: b.sddmm(vs))
+        ptr = lambda t: t.data_ptr()
+        t_h = rep(lambda: L.bl_hgemm(h, p.M, p.N, p.K, ptr(b.Wd), ptr(b.X), ptr(Cd),
+                                     torch.cuda.current_stream().cuda_stream))
+        t_gx = rep(lambda: L.bl_gemmex(h, p.M, p.N, p.K, ptr(b.Wd), ptr(b.X), ptr(Cd),
+                                       torch.cuda.current_stream().cuda_stream))
+        d.update({"spmm_us_warm": t_spmm, "sddmm_us_warm": t_sddmm, "hgemm_us": t_h, "gemmex_us": t_gx})
+        # cuSPARSE Blocked-ELL with block = V (reading R12)
+        try:
+            rng = gen.make_rng("bell_" + p.id)
+            nb = max(1, int(round(p.K / p.V * (1.0 - p.S))))
+            nbr = p.M // p.V
+            ci = np.stack([np.sort(rng.choice(p.K // p.V, size=nb, replace=False)) for _ in range(nbr)]).astype(np.int32)
+            ev = gen.fp16_values(rng, (p.M, nb * p.V))
+            d_ci, d_ev = torch.from_numpy(ci).cuda(), torch.from_numpy(ev).cuda()
+            st = ctypes_int()
+            plan = L.bl_spmm_bell_plan(h, p.M, p.K, p.N, p.V, nb * p.V, ptr(d_ci), ptr(d_ev),
+                                       ptr(b.X), ptr(Cd), sptr, st)
+            if plan:
+                t_bell = rep(lambda: L.bl_plan_run(plan))
+                d["cusparse_bell_us"] = t_bell
+                L.bl_plan_free(plan)
+            else:
+                d["cusparse_bell_status"] = st.value
+        except Exception as exc:
+            d["cusparse_bell_error"] = repr(exc)[:200]
+        # scalar CSR (V-expanded) for cusparseSpMM / SDDMM
+        try:
+            rp = b.row_ptr.cpu().numpy().astype(np.int64)
+            ci = b.col_idx[:b.nnz_v].cpu().numpy()
+            W = len(rp) - 1
+            rows_rp = [0]
+            cols = []
+            for w in range(W):
+                seg = ci[rp[w]:rp[w + 1]]
+                for r in range(p.V):
+                    if w * p.V + r < p.M:
+                        cols.append(seg)
+                        rows_rp.append(rows_rp[-1] + seg.size)
+            s_rp = torch.from_numpy(np.asarray(rows_rp, np.int32)).cuda()
+            s_ci = torch.from_numpy(np.concatenate(cols).astype(np.int32) if cols else np.zeros(0, np.int32)).cuda()
+            nnz_s = int(rows_rp[-1])
+            s_v = torch.ones(max(nnz_s, 1), dtype=torch.float16, device=b.X.device)
+            st = ctypes_int()
+            plan = L.bl_spmm_csr_plan(h, p.M, p.K, p.N, nnz_s, ptr(s_rp), ptr(s_ci), ptr(s_v),
+                                      ptr(b.X), ptr(Cd), sptr, st)
+            if plan:
+                d["cusparse_csr_spmm_us"] = rep(lambda: L.bl_plan_run(plan))
+                L.bl_plan_free(plan)
+            else:
+                d["cusparse_csr_spmm_status"] = st.value
+            Xt = b.X.t().contiguous()  # cuSPARSE SDDMM B operand [N x K] row-major
+            for vt, tag, A_, B_ in ((0, "fp16", b.G, Xt), (1, "fp32", b.G.float(), Xt.float())):
+                out = torch.empty(max(nnz_s, 1), dtype=A_.dtype, device=b.X.device)
+                st = ctypes_int()
+                plan = L.bl_sddmm_csr_plan(h, p.M, p.K, p.N, nnz_s, ptr(s_rp), ptr(s_ci), ptr(out),
+                                           ptr(A_), ptr(B_), vt, sptr, st)
+                if plan:
+                    d[f"cusparse_sddmm_{tag}_us"] = rep(lambda: L.bl_plan_run(plan))
+                    L.bl_plan_free(plan)
+                    break
+                d[f"cusparse_sddmm_{tag}_status"] = st.value
+        except Exception as exc:
+            d["cusparse_csr_error"] = repr(exc)[:200]
+        key = (p.V, p.S)
+        c = cells.setdefault(key, {"spmm_vs_h": [], "sddmm_vs_h": [], "spmm_vs_bell": [],
+                                   "spmm_vs_best_cublas": [], "sddmm_vs_cusparse": []})
+        c["spmm_vs_h"].append(t_h / t_spmm)
+        c["sddmm_vs_h"].append(t_h / t_sddmm)
+        c["spmm_vs_best_cublas"].append(min(t_h, t_gx) / t_spmm)
+        if "cusparse_bell_us" in d:
+            c["spmm_vs_bell"].append(d["cusparse_bell_us"] / t_spmm)
+        sd = d.get("cusparse_sddmm_fp16_us") or d.get("cusparse_sddmm_fp32_us")
+        if sd:
+            c["sddmm_vs_cusparse"].append(sd / t_sddmm)
+    L.bl_destroy(h)
+    summary = {}
+    for (V, S), c in sorted(cells.items()):
+        summary[f"V{V}_S{S:.2f}"] = {k: (round(geomean(v), 3) if geomean(v) else None) for k, v in c.items()}
+    all_spmm = [x for c in cells.values() for x in c["spmm_vs_h"]]
+    all_sddmm = [x for c in cells.values() for x in c["sddmm_vs_h"]]
+    return {"speedup_vs_cublas_hgemm": {
+        "geomean_spmm": geomean(all_spmm), "geomean_sddmm": geomean(all_sddmm),
+        "per_cell_geomean": summary,
+        "protocol": f"{args.reps} launches per CUDA graph, L2 warm, per-launch mean; dense "
+                    "counterpart = cublasHgemm M x K x N (both ops)"}}
+
+
+def ctypes_int():
+    import ctypes
+    return ctypes.c_int(0)
+
+
+def main(argv=None):
+    args = parse_args(argv)
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_ours(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

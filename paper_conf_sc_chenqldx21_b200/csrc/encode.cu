@@ -1,22 +1,18 @@
 // encode.cu — dense fp16 matrix / uint8 mask -> column-vector CSR (§4.2, Fig. 8).
 //
-// Three stream-ordered kernels:
-//   1. encode_count   : one warp per row window; each lane tests 8 consecutive columns per
-//                       step (one 16-byte load per row of the window), keep bit = any nonzero
-//                       fp16 bit pattern (or mask byte) over the window's V rows; the warp's
-//                       popcount total goes to row_ptr[w+1].
-//   2. scan_inplace   : one CTA turns the per-window counts into the inclusive prefix, so
-//                       row_ptr[w] is the first vector of window w (row_ptr[0] = 0).
-//   3. encode_compact : one warp per window again; a warp-wide exclusive scan of the lanes'
-//                       keep counts gives every kept column its slot; the lane writes col_idx
-//                       and the V values of the vector (transposed from the V row loads into
-//                       vector-major order).
+// One kernel (encode_fused, below) with one CTA per row window and one warp per 256-column
+// chunk (up to 8 warps); each lane tests 8 consecutive columns with one 16-byte load per
+// row of the window.  Keep bit = any nonzero fp16 bit pattern (or mask byte) over the
+// window's V rows.  Phase 1 counts the window; a decoupled look-back over row_ptr gives the
+// window's first slot (row_ptr becomes the CSR row pointer in place); phase 2 writes col_idx
+// and the V values of each kept vector (transposed from the V row loads into vector-major
+// order).
 // Columns are visited in ascending order, so col_idx ascends inside each window (Fig. 8).
 #include "common.cuh"
 
 namespace vs {
 
-constexpr int kEncWarps = 4;                     // warps (windows) per CTA
+constexpr int kEncMaxThreads = 256;              // threads per CTA (one CTA per window)
 constexpr int kColsPerLane = 8;                  // columns per lane per step
 constexpr int kColsPerStep = kColsPerLane * 32;  // 256 columns per warp step
 
@@ -96,101 +92,156 @@ __device__ __forceinline__ uint32_t window_keep8(const uint16_t* __restrict__ de
   return keep;
 }
 
-template <int V, bool VEC, bool HAS_MASK>
-__global__ void __launch_bounds__(kEncWarps * 32)
-    encode_count_kernel(int64_t M, int64_t K, int64_t W, const uint16_t* __restrict__ dense,
-                        const uint8_t* __restrict__ mask, int32_t* __restrict__ row_ptr) {
-  const int lane = lane_id();
-  const int64_t w = (int64_t)blockIdx.x * kEncWarps + (threadIdx.x >> 5);
-  if (w >= W) return;
-  uint32_t count = 0;
+// ---------------------------------------------------------------- single-pass encoder
+//
+// encode_fused: one kernel per call.  CTA w counts its window (phase 1), publishes the count,
+// obtains the exclusive prefix of all earlier windows by a decoupled look-back over
+// row_ptr itself, publishes its inclusive prefix, then (phase 2) writes col_idx / vals.
+// row_ptr[w+1] doubles as the look-back status of window w (it is preset to -1 by one
+// memset node):  -1 = nothing yet,  <= -2 = aggregate (count = -s-2) only,  >= 0 = inclusive
+// prefix (final value).  CTAs are dispatched in blockIdx order, so a CTA only waits on CTAs
+// that are already resident or finished.
+
+// The status word is the only data exchanged between CTAs, so relaxed gpu-scope accesses
+// suffice (no other memory is published through it); relaxed loads are not serialised the
+// way acquire loads are, so a thread's look-back loads are all in flight at once.
+__device__ __forceinline__ void st_status(int32_t* p, int32_t v) {
+  asm volatile("st.relaxed.gpu.global.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ int32_t ld_status(const int32_t* p) {
+  int32_t v;
+  asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+
+// Exclusive prefix of windows [0, w), computed by the whole CTA (all threads call it; all
+// get the result).  One round reads the statuses of the kLookback nearest predecessors at
+// once (all CTAs of a small problem run concurrently, so the nearest prefix is usually the
+// sentinel P(0) before window 0 and one round suffices); the nearest published prefix ends
+// the walk, aggregates before it are summed.
+constexpr int kLookback = 1024;
+
+__device__ __forceinline__ int64_t lookback(const int32_t* row_ptr, int64_t w, int32_t* s_min,
+                                            int64_t* s_sum) {
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5, nw = blockDim.x >> 5;
+  const int per = kLookback / blockDim.x;  // statuses per thread per round (<= 32)
+  int64_t excl = 0;
+  int64_t j = w - 1;  // nearest window not yet accounted for (its status is row_ptr[j + 1])
+  while (true) {
+    int32_t st[32];
+    int my_first = 0x7fffffff;  // smallest offset o (= j - idx) holding a prefix
+    // issue all loads, then re-poll only the statuses not yet published
+    bool pending = false;
+#pragma unroll
+    for (int q = 0; q < 32; ++q) {
+      if (q >= per) break;
+      const int64_t idx = j - (tid * per + q);
+      // idx == -1: the P(0) sentinel; idx < -1: beyond it, never summed
+      st[q] = idx >= 0 ? ld_status(row_ptr + idx + 1) : 0;
+    }
+#pragma unroll
+    for (int q = 0; q < 32; ++q) pending |= (q < per) && st[q] == -1;
+    while (pending) {
+      pending = false;
+#pragma unroll
+      for (int q = 0; q < 32; ++q) {
+        if (q >= per) break;
+        if (st[q] == -1) st[q] = ld_status(row_ptr + (j - (tid * per + q)) + 1);
+      }
+#pragma unroll
+      for (int q = 0; q < 32; ++q) pending |= (q < per) && st[q] == -1;
+    }
+#pragma unroll
+    for (int q = 0; q < 32; ++q) {
+      if (q >= per) break;
+      const int o = tid * per + q;
+      if (st[q] >= 0 && o < my_first) my_first = o;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) my_first = min(my_first, __shfl_xor_sync(0xffffffffu, my_first, o));
+    if (lane == 0) s_min[wid] = my_first;
+    __syncthreads();
+    int first = 0x7fffffff;
+    for (int i = 0; i < nw; ++i) first = min(first, s_min[i]);
+    int64_t part = 0;
+#pragma unroll
+    for (int q = 0; q < 32; ++q) {
+      if (q >= per) break;
+      const int o = tid * per + q;
+      const int32_t v = st[q];
+      if (o < first) part += (int64_t)(-v - 2);  // aggregate (only -x-2 values precede first)
+      else if (o == first) part += (int64_t)v;    // the nearest inclusive prefix
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
+    if (lane == 0) s_sum[wid] = part;
+    __syncthreads();
+    for (int i = 0; i < nw; ++i) excl += s_sum[i];
+    __syncthreads();  // s_min / s_sum reused next round
+    if (first != 0x7fffffff) return excl;
+    j -= kLookback;
+  }
+}
+
+template <int V, bool VEC, bool HAS_MASK, bool WRITE_IDX, bool WRITE_VALS, bool VEC_VALS>
+__global__ void __launch_bounds__(kEncMaxThreads)
+    encode_fused_kernel(int64_t M, int64_t K, const uint16_t* __restrict__ dense,
+                        const uint8_t* __restrict__ mask, int32_t* __restrict__ row_ptr,
+                        int32_t* __restrict__ col_idx, uint16_t* __restrict__ vals) {
+  __shared__ uint32_t warp_cnt[kEncMaxThreads / 32];
+  __shared__ int32_t s_min[kEncMaxThreads / 32];
+  __shared__ int64_t s_sum[kEncMaxThreads / 32];
+  const int lane = lane_id(), wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  const int64_t w = blockIdx.x;
   uint16_t h[V][8];
-  for (int64_t c0 = 0; c0 < K; c0 += kColsPerStep) {
-    int64_t c = c0 + lane * kColsPerLane;
-    uint32_t keep = window_keep8<V, VEC, HAS_MASK, false>(dense, mask, M, K, w, c, h);
-    count += __popc(keep);
+
+  // phase 1: count the window's kept vectors
+  uint32_t count = 0;
+  for (int64_t c0 = (int64_t)wid * kColsPerStep; c0 < K; c0 += (int64_t)nw * kColsPerStep) {
+    const int64_t c = c0 + lane * kColsPerLane;
+    count += __popc(window_keep8<V, VEC, HAS_MASK, false>(dense, mask, M, K, w, c, h));
   }
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) count += __shfl_xor_sync(0xffffffffu, count, o);
-  if (lane == 0) row_ptr[w + 1] = (int32_t)count;
-  if (w == 0 && lane == 0) row_ptr[0] = 0;
-}
-
-// In-place inclusive scan of row_ptr[1..W] (per-window counts) by one CTA of 1024 threads.
-constexpr int kScanThreads = 1024;
-constexpr int kScanPerThread = 4;
-__global__ void __launch_bounds__(kScanThreads) scan_inplace_kernel(int32_t* __restrict__ row_ptr,
-                                                                    int64_t W) {
-  __shared__ int32_t warp_sums[32];
-  __shared__ int32_t carry_s;
-  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-  if (tid == 0) carry_s = 0;
+  if (lane == 0) warp_cnt[wid] = count;
   __syncthreads();
-  int32_t* a = row_ptr + 1;
-  for (int64_t base = 0; base < W; base += (int64_t)kScanThreads * kScanPerThread) {
-    int32_t v[kScanPerThread];
-    int32_t local = 0;
-#pragma unroll
-    for (int j = 0; j < kScanPerThread; ++j) {
-      int64_t idx = base + (int64_t)tid * kScanPerThread + j;
-      v[j] = idx < W ? a[idx] : 0;
-      local += v[j];
+  uint32_t tot = 0;
+  for (int i = 0; i < nw; ++i) tot += warp_cnt[i];
+  int64_t base;
+  if (w == 0) {
+    if (threadIdx.x == 0) {
+      st_status(row_ptr + 1, (int32_t)tot);
+      row_ptr[0] = 0;
     }
-    int32_t incl = local;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      int32_t t = __shfl_up_sync(0xffffffffu, incl, o);
-      if (lane >= o) incl += t;
-    }
-    if (lane == 31) warp_sums[wid] = incl;
-    __syncthreads();
-    if (wid == 0) {
-      int32_t s = warp_sums[lane];
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        int32_t t = __shfl_up_sync(0xffffffffu, s, o);
-        if (lane >= o) s += t;
-      }
-      warp_sums[lane] = s;  // inclusive over warps
-    }
-    __syncthreads();
-    int32_t carry = carry_s;
-    int32_t run = carry + (wid > 0 ? warp_sums[wid - 1] : 0) + incl - local;
-#pragma unroll
-    for (int j = 0; j < kScanPerThread; ++j) {
-      int64_t idx = base + (int64_t)tid * kScanPerThread + j;
-      run += v[j];
-      if (idx < W) a[idx] = run;
-    }
-    __syncthreads();
-    if (tid == 0) carry_s = carry + warp_sums[31];
-    __syncthreads();
+    base = 0;
+  } else {
+    if (threadIdx.x == 0) st_status(row_ptr + w + 1, -(int32_t)tot - 2);  // aggregate
+    base = lookback(row_ptr, w, s_min, s_sum);
+    if (threadIdx.x == 0) st_status(row_ptr + w + 1, (int32_t)(base + tot));  // inclusive prefix
   }
-  if (tid == 0) row_ptr[0] = 0;
-}
+  if (!WRITE_IDX) return;
 
-// Writes col_idx and (optionally) vals of window w; needs the scanned row_ptr.
-template <int V, bool VEC, bool HAS_MASK, bool WRITE_VALS, bool VEC_VALS>
-__global__ void __launch_bounds__(kEncWarps * 32)
-    encode_compact_kernel(int64_t M, int64_t K, int64_t W, const uint16_t* __restrict__ dense,
-                          const uint8_t* __restrict__ mask, const int32_t* __restrict__ row_ptr,
-                          int32_t* __restrict__ col_idx, uint16_t* __restrict__ vals) {
-  const int lane = lane_id();
-  const int64_t w = (int64_t)blockIdx.x * kEncWarps + (threadIdx.x >> 5);
-  if (w >= W) return;
-  int64_t base = row_ptr[w];
-  uint16_t h[V][8];
-  for (int64_t c0 = 0; c0 < K; c0 += kColsPerStep) {
-    int64_t c = c0 + lane * kColsPerLane;
-    uint32_t keep = window_keep8<V, VEC, HAS_MASK, WRITE_VALS>(dense, mask, M, K, w, c, h);
-    uint32_t n = __popc(keep);
+  // phase 2: write col_idx / vals (re-reads the window, now L1/L2 resident)
+  for (int64_t r0 = 0; r0 < K; r0 += (int64_t)nw * kColsPerStep) {
+    const int64_t c = r0 + (int64_t)wid * kColsPerStep + lane * kColsPerLane;
+    const uint32_t keep = window_keep8<V, VEC, HAS_MASK, WRITE_VALS>(dense, mask, M, K, w, c, h);
+    const uint32_t n = __popc(keep);
     uint32_t incl = n;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
-      uint32_t t = __shfl_up_sync(0xffffffffu, incl, o);
+      const uint32_t t = __shfl_up_sync(0xffffffffu, incl, o);
       if (lane >= o) incl += t;
     }
-    int64_t slot = base + (incl - n);
+    __syncthreads();  // previous round's readers of warp_cnt are done
+    if (lane == 31) warp_cnt[wid] = incl;
+    __syncthreads();
+    uint32_t before = 0, total = 0;
+    for (int i = 0; i < nw; ++i) {
+      const uint32_t v = warp_cnt[i];
+      before += (i < wid) ? v : 0;
+      total += v;
+    }
+    int64_t slot = base + before + (incl - n);
 #pragma unroll
     for (int j = 0; j < 8; ++j) {
       if (keep & (1u << j)) {
@@ -213,11 +264,29 @@ __global__ void __launch_bounds__(kEncWarps * 32)
         ++slot;
       }
     }
-    base += __shfl_sync(0xffffffffu, incl, 31);
+    base += total;
   }
 }
 
 // ---------------------------------------------------------------- host-side launchers
+
+template <int V, bool VEC, bool MASKB>
+static void launch_fused(int64_t M, int64_t K, int64_t W, const uint16_t* dense, const uint8_t* mask,
+                         int32_t* row_ptr, int32_t* col_idx, uint16_t* vals, bool vec_vals,
+                         dim3 grid, dim3 block, cudaStream_t s) {
+  if (col_idx == nullptr)
+    encode_fused_kernel<V, VEC, MASKB, false, false, false><<<grid, block, 0, s>>>(
+        M, K, dense, mask, row_ptr, col_idx, vals);
+  else if (vals == nullptr)
+    encode_fused_kernel<V, VEC, MASKB, true, false, false><<<grid, block, 0, s>>>(
+        M, K, dense, mask, row_ptr, col_idx, vals);
+  else if (vec_vals)
+    encode_fused_kernel<V, VEC, MASKB, true, true, true><<<grid, block, 0, s>>>(
+        M, K, dense, mask, row_ptr, col_idx, vals);
+  else
+    encode_fused_kernel<V, VEC, MASKB, true, true, false><<<grid, block, 0, s>>>(
+        M, K, dense, mask, row_ptr, col_idx, vals);
+}
 
 template <int V>
 static cudaError_t launch_encode_v(int64_t M, int64_t K, const uint16_t* dense, const uint8_t* mask,
@@ -225,35 +294,23 @@ static cudaError_t launch_encode_v(int64_t M, int64_t K, const uint16_t* dense, 
                                    bool vec_vals, cudaStream_t s) {
   const int64_t W = ceil_div64(M, V);
   if (W == 0) return cudaSuccess;
-  dim3 grid((unsigned)ceil_div64(W, kEncWarps)), block(kEncWarps * 32);
+  if (W > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
+  // one CTA per window, one warp per 256-column chunk (up to 8 warps)
+  const int64_t chunks = ceil_div64(K, kColsPerStep);
+  const int threads =
+      (int)(32 * (chunks < 1 ? 1 : (chunks > kEncMaxThreads / 32 ? kEncMaxThreads / 32 : chunks)));
+  dim3 grid((unsigned)W), block(threads);
+  // look-back status: row_ptr[1..W] = -1 ("nothing published yet")
+  cudaError_t e = cudaMemsetAsync(row_ptr + 1, 0xFF, (size_t)W * sizeof(int32_t), s);
+  if (e != cudaSuccess) return e;
   const bool has_mask = mask != nullptr;
-#define VS_COUNT(VECB, MASKB) \
-  encode_count_kernel<V, VECB, MASKB><<<grid, block, 0, s>>>(M, K, W, dense, mask, row_ptr)
   if (vec) {
-    if (has_mask) VS_COUNT(true, true); else VS_COUNT(true, false);
+    if (has_mask) launch_fused<V, true, true>(M, K, W, dense, mask, row_ptr, col_idx, vals, vec_vals, grid, block, s);
+    else launch_fused<V, true, false>(M, K, W, dense, mask, row_ptr, col_idx, vals, vec_vals, grid, block, s);
   } else {
-    if (has_mask) VS_COUNT(false, true); else VS_COUNT(false, false);
+    if (has_mask) launch_fused<V, false, true>(M, K, W, dense, mask, row_ptr, col_idx, vals, vec_vals, grid, block, s);
+    else launch_fused<V, false, false>(M, K, W, dense, mask, row_ptr, col_idx, vals, vec_vals, grid, block, s);
   }
-#undef VS_COUNT
-  scan_inplace_kernel<<<1, kScanThreads, 0, s>>>(row_ptr, W);
-  if (col_idx == nullptr) return cudaGetLastError();
-  const bool wv = vals != nullptr;
-#define VS_COMPACT(VECB, MASKB, WVB, VVB)                                              \
-  encode_compact_kernel<V, VECB, MASKB, WVB, VVB><<<grid, block, 0, s>>>(M, K, W, dense, mask, \
-                                                                          row_ptr, col_idx, vals)
-#define VS_COMPACT2(VECB, MASKB)                                \
-  do {                                                          \
-    if (!wv) VS_COMPACT(VECB, MASKB, false, false);             \
-    else if (vec_vals) VS_COMPACT(VECB, MASKB, true, true);     \
-    else VS_COMPACT(VECB, MASKB, true, false);                  \
-  } while (0)
-  if (vec) {
-    if (has_mask) VS_COMPACT2(true, true); else VS_COMPACT2(true, false);
-  } else {
-    if (has_mask) VS_COMPACT2(false, true); else VS_COMPACT2(false, false);
-  }
-#undef VS_COMPACT2
-#undef VS_COMPACT
   return cudaGetLastError();
 }
 

@@ -86,47 +86,65 @@ __global__ void __launch_bounds__(kSddmmWarps * 32)
   const int64_t s_end = (s_begin + per < n_slices) ? s_begin + per : n_slices;
   if (s_begin >= s_end) return;
 
-  int64_t w = find_window(row_ptr, W, s_begin * 16);
-  int64_t w_end_p = row_ptr[w + 1];  // first vector after window w
+  const int64_t kt = 8 * t;
+  // Per slice: the two vectors (M rows g and g+8) whose Bt rows this thread loads.  Their
+  // column indices are fetched one slice ahead and the first K chunk of the next slice is
+  // loaded during the current slice's last chunk, so consecutive slices overlap.
+  int64_t v0 = s_begin * 16;
+  int64_t v_hi = (v0 + 16 < nnz) ? v0 + 16 : nnz;
+  bool oka = v0 + g < v_hi, okb = v0 + g + 8 < v_hi;
+  const uint16_t* rowa = Bt + (int64_t)(oka ? ldg32i(col_idx + v0 + g) : 0) * K;
+  const uint16_t* rowb = Bt + (int64_t)(okb ? ldg32i(col_idx + v0 + g + 8) : 0) * K;
+  uint4 a0, a1, b0, b1;  // Bt chunk [k0, k0 + 64) of vectors g and g+8
+  load_seg2<VEC>(rowa, K, kt, oka, a0, a1);
+  load_seg2<VEC>(rowb, K, kt, okb, b0, b1);
+  // the window search runs while the first gathered rows are in flight
+  int64_t w = find_window(row_ptr, W, v0);
+  int64_t w_end_p = row_ptr[w + 1];
 
   for (int64_t s = s_begin; s < s_end; ++s) {
-    const int64_t v0 = s * 16;
-    const int64_t v_hi = (v0 + 16 < nnz) ? v0 + 16 : nnz;
-    // the two vectors (M rows g and g+8) this thread loads Bt rows for
-    const int64_t va = v0 + g, vb = v0 + g + 8;
-    const bool oka = va < v_hi, okb = vb < v_hi;
-    const int ca = oka ? ldg32i(col_idx + va) : 0;
-    const int cb = okb ? ldg32i(col_idx + vb) : 0;
-    const uint16_t* rowa = Bt + (int64_t)ca * K;
-    const uint16_t* rowb = Bt + (int64_t)cb * K;
+    // next slice's column indices
+    const bool has_next = s + 1 < s_end;
+    const int64_t nv0 = v0 + 16;
+    const int64_t nv_hi = (nv0 + 16 < nnz) ? nv0 + 16 : nnz;
+    const bool noka = has_next && nv0 + g < nv_hi, nokb = has_next && nv0 + g + 8 < nv_hi;
+    const int nca = noka ? ldg32i(col_idx + nv0 + g) : 0;
+    const int ncb = nokb ? ldg32i(col_idx + nv0 + g + 8) : 0;
 
     int64_t v_cur = v0;
+    bool first_seg = true;
     while (v_cur < v_hi) {
       while (w_end_p <= v_cur) {  // advance to the window owning v_cur
         ++w;
         w_end_p = row_ptr[w + 1];
       }
       const int64_t seg_hi = w_end_p < v_hi ? w_end_p : v_hi;  // vectors [v_cur, seg_hi) in w
+      const bool last_seg = seg_hi == v_hi;
       const int64_t arow = w * V + g;
       const bool oka_row = (g < V) && (arow < M);
       const uint16_t* rowA = A + arow * K;
+      if (!first_seg) {  // the slice straddles windows: restart the Bt stream
+        load_seg2<VEC>(rowa, K, kt, oka, a0, a1);
+        load_seg2<VEC>(rowb, K, kt, okb, b0, b1);
+      }
+      first_seg = false;
 
       float acc[4] = {0.f, 0.f, 0.f, 0.f};
-      for (int64_t k0 = 0; k0 < K; k0 += 128) {
-        uint4 a0[2], a1[2], b0[2], b1[2], x0[2], x1[2];
-#pragma unroll
-        for (int h = 0; h < 2; ++h) {
-          const int64_t k = k0 + 64 * h + 8 * t;
-          load_seg2<VEC>(rowa, K, k, oka, a0[h], a1[h]);      // Bt row of vector g
-          load_seg2<VEC>(rowb, K, k, okb, b0[h], b1[h]);      // Bt row of vector g+8
-          load_seg2<VEC>(rowA, K, k, oka_row, x0[h], x1[h]);  // A row g of the window
+      for (int64_t k0 = 0; k0 < K; k0 += 64) {
+        uint4 x0, x1;  // A row g of the window, same K permutation
+        load_seg2<VEC>(rowA, K, k0 + kt, oka_row, x0, x1);
+        const uint4 ca0 = a0, ca1 = a1, cb0 = b0, cb1 = b1;
+        if (k0 + 64 < K) {  // prefetch the next chunk of the gathered rows
+          load_seg2<VEC>(rowa, K, k0 + 64 + kt, oka, a0, a1);
+          load_seg2<VEC>(rowb, K, k0 + 64 + kt, okb, b0, b1);
+        } else if (last_seg && has_next) {  // or the first chunk of the next slice
+          load_seg2<VEC>(Bt + (int64_t)nca * K, K, kt, noka, a0, a1);
+          load_seg2<VEC>(Bt + (int64_t)ncb * K, K, kt, nokb, b0, b1);
         }
 #pragma unroll
-        for (int h = 0; h < 2; ++h)
-#pragma unroll
-          for (int j = 0; j < 4; ++j)
-            mma_16816(acc, wordj(a0[h], j), wordj(b0[h], j), wordj(a1[h], j), wordj(b1[h], j),
-                      wordj(x0[h], j), wordj(x1[h], j));
+        for (int j = 0; j < 4; ++j)
+          mma_16816(acc, wordj(ca0, j), wordj(cb0, j), wordj(ca1, j), wordj(cb1, j),
+                    wordj(x0, j), wordj(x1, j));
       }
       // acc[0..1]: vector v0+g, rows 2t, 2t+1; acc[2..3]: vector v0+g+8, rows 2t, 2t+1.
 #pragma unroll
@@ -146,7 +164,27 @@ __global__ void __launch_bounds__(kSddmmWarps * 32)
       }
       v_cur = seg_hi;
     }
+    v0 = nv0;
+    v_hi = nv_hi;
+    oka = noka;
+    okb = nokb;
+    rowa = Bt + (int64_t)nca * K;
+    rowb = Bt + (int64_t)ncb * K;
   }
+}
+
+// Persistent grid: as many CTAs as can be resident at once (occupancy queried once per
+// kernel instantiation), so every warp's contiguous share of slices runs concurrently.
+template <int V, bool VEC>
+static int sddmm_ctas_per_sm() {
+  static const int n = [] {
+    int b = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, sddmm_kernel<V, VEC>, kSddmmWarps * 32, 0) !=
+            cudaSuccess || b < 1)
+      b = 1;
+    return b;
+  }();
+  return n;
 }
 
 template <int V>
@@ -156,12 +194,14 @@ static cudaError_t launch_sddmm_v(int64_t M, int64_t N, int64_t K, const int32_t
   (void)N;
   const int64_t W = ceil_div64(M, V);
   dim3 block(kSddmmWarps * 32);
-  dim3 grid((unsigned)(num_sms * 8));  // persistent: 8 CTAs (32 warps) per SM
   const bool out4 = (reinterpret_cast<uintptr_t>(out) & 3) == 0;
-  if (vec)
+  if (vec) {
+    dim3 grid((unsigned)(num_sms * sddmm_ctas_per_sm<V, true>()));
     sddmm_kernel<V, true><<<grid, block, 0, s>>>(M, K, W, row_ptr, col_idx, A, Bt, out, out4);
-  else
+  } else {
+    dim3 grid((unsigned)(num_sms * sddmm_ctas_per_sm<V, false>()));
     sddmm_kernel<V, false><<<grid, block, 0, s>>>(M, K, W, row_ptr, col_idx, A, Bt, out, out4);
+  }
   return cudaGetLastError();
 }
 

@@ -1,0 +1,125 @@
+"""Multi-GPU partitioning of the hot path (one process per GPU, torch.distributed).
+
+The paper is single-GPU; the sharding follows the north star: the two ops
+split into independent units, so ranks compute with NO data-path collective, and an NCCL
+all-gather runs only when the caller asks for a replicated output.
+
+  SpMM  (C = A B):  N-panels.  Rank p owns the columns [n_p, n_{p+1}) of B and C (panel
+        widths multiples of 64, the paper's TileN); A (column-vector CSR) is
+        replicated.  Per-element accumulation order does not depend on the panel, so the
+        sharded result equals the 1-GPU result bit for bit.
+  SDDMM (out = (A B^T) o D): row windows.  Rank p owns windows [w_p, w_{p+1}) chosen by a
+        binary search of row_ptr so that each rank gets ~nnz_v/P stored vectors; its A rows,
+        a rebased row_ptr slice, and the contiguous col_idx / out_vals slices.  Bt is
+        replicated.  The concatenated out_vals equal the unsharded ones bit for bit.
+
+Only host-side bookkeeping lives here; the per-shard compute is an ordinary vs_spmm /
+vs_sddmm call on the shard's buffers (``compute=`` hooks exist so the partition logic can
+be tested on CPU with a stand-in).
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass
+
+import numpy as np
+
+__all__ = ["panel_bounds", "window_bounds", "SddmmShard", "sddmm_shard", "spmm_npanel",
+           "sddmm_rowwin", "gather_panels", "gather_segments"]
+
+
+def panel_bounds(N: int, world: int, align: int = 64) -> list:
+    """Column boundaries [n_0 = 0, ..., n_P = N] of P panels whose widths are multiples of
+    ``align`` (except possibly the last), as equal as possible."""
+    units = -(-N // align) if N > 0 else 0
+    out = [0]
+    for p in range(1, world + 1):
+        out.append(min(N, (units * p // world) * align))
+    out[-1] = N
+    return out
+
+
+def window_bounds(row_ptr: np.ndarray, world: int) -> list:
+    """Window boundaries [w_0 = 0, ..., w_P = W] with row_ptr[w_p] ~ p * nnz_v / P
+    (balanced to within one window's vectors)."""
+    row_ptr = np.asarray(row_ptr, dtype=np.int64)
+    W = row_ptr.size - 1
+    nnz = int(row_ptr[-1])
+    out = [0]
+    for p in range(1, world):
+        target = (nnz * p) // world
+        w = int(np.searchsorted(row_ptr, target, side="left"))
+        out.append(min(max(w, out[-1]), W))
+    out.append(W)
+    return out
+
+
+@dataclass
+class SddmmShard:
+    w0: int           # first window
+    w1: int           # one past the last window
+    p0: int           # first stored vector (global index)
+    p1: int           # one past the last stored vector
+    row0: int         # first scalar row of A = w0 * V
+    row1: int         # one past the last scalar row (clipped to M)
+    row_ptr: np.ndarray  # rebased row_ptr slice, int32 [w1 - w0 + 1]
+
+
+def sddmm_shard(row_ptr: np.ndarray, M: int, V: int, bounds: list, rank: int) -> SddmmShard:
+    row_ptr = np.asarray(row_ptr, dtype=np.int64)
+    w0, w1 = bounds[rank], bounds[rank + 1]
+    p0, p1 = int(row_ptr[w0]), int(row_ptr[w1])
+    local = (row_ptr[w0:w1 + 1] - p0).astype(np.int32)
+    return SddmmShard(w0, w1, p0, p1, w0 * V, min(M, w1 * V), local)
+
+
+def spmm_npanel(row_ptr, col_idx, vals, B_panel, M: int, V: int, compute=None, out=None):
+    """This rank's panel of C = A B: an ordinary SpMM on the local [K x Np] panel of B.
+    ``compute(row_ptr, col_idx, vals, B_panel, M, V, out)`` defaults to the CUDA kernel."""
+    if compute is None:
+        from . import spmm as compute
+    return compute(row_ptr, col_idx, vals, B_panel, M, V, out=out)
+
+
+def sddmm_rowwin(shard: SddmmShard, row_ptr_local, col_idx_local, A_rows, Bt, V: int,
+                 compute=None, out=None):
+    """This rank's out_vals segment (vectors [p0, p1)) of the sampled product."""
+    if compute is None:
+        from . import sddmm as compute
+    return compute(row_ptr_local, col_idx_local, A_rows, Bt, V, nnz=shard.p1 - shard.p0, out=out)
+
+
+def gather_panels(C_panel, bounds: list, group=None, row_major: bool = True):
+    """All-gather of the C panels (optional replicated output).  Panels are padded to the
+    widest one, gathered with all_gather_into_tensor ([P, M, Np_max], panel-major) and, if
+    ``row_major``, permuted into the row-major [M, N] matrix."""
+    import torch
+    import torch.distributed as dist
+    world = len(bounds) - 1
+    widths = [bounds[i + 1] - bounds[i] for i in range(world)]
+    wmax = max(widths)
+    M = C_panel.shape[0]
+    send = C_panel
+    if C_panel.shape[1] != wmax:
+        send = torch.zeros((M, wmax), dtype=C_panel.dtype, device=C_panel.device)
+        send[:, :C_panel.shape[1]] = C_panel
+    recv = torch.empty((world * M, wmax), dtype=C_panel.dtype, device=C_panel.device)
+    dist.all_gather_into_tensor(recv, send.contiguous(), group=group)
+    recv = recv.view(world, M, wmax)
+    if not row_major:
+        return recv
+    return torch.cat([recv[i, :, :widths[i]] for i in range(world)], dim=1)
+
+
+def gather_segments(segment, counts: list, group=None):
+    """All-gather-v of contiguous out_vals segments (rank i contributes counts[i] values) into
+    the global array, via a padded all_gather_into_tensor."""
+    import torch
+    import torch.distributed as dist
+    world = len(counts)
+    cmax = max(counts) if counts else 0
+    send = torch.zeros(cmax, dtype=segment.dtype, device=segment.device)
+    send[:segment.numel()] = segment.reshape(-1)
+    recv = torch.empty(world * cmax, dtype=segment.dtype, device=segment.device)
+    dist.all_gather_into_tensor(recv, send, group=group)
+    recv = recv.view(world, cmax)
+    return torch.cat([recv[i, :counts[i]] for i in range(world)])

@@ -71,5 +71,7 @@ WORKLOADS = {
     "dlmc_layer": dlmc_layer_workload,
     "rn50_layer": rn50_workload,
     "c1": lambda: [c1_problem()],
+    # the paper's profiling case: A 2048x1024 x B 1024x256, 90% (Tables 2/3)
+    "profile": lambda: [Problem(2048, 1024, 256, 4, 0.9), Problem(2048, 1024, 256, 8, 0.9)],
     "c5": lambda: [c5_problem()],
 }

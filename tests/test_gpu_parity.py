@@ -324,3 +324,91 @@ def test_adjoint_identity_gpu(vs, V):
     scale = float((dev(np.abs(Wd.astype(np.float64))) @ dev(np.abs(X.astype(np.float64)))
                    * dev(np.abs(G.astype(np.float64)))).sum())
     assert abs(lhs - rhs) <= 2e-3 * scale
+
+
+# ------------------------------------------------ sharding invariants with the kernels
+
+@pytest.mark.parametrize("V", [2, 8])
+def test_sharded_equals_unsharded_spmm(vs, V):
+    """N-panel shards (dist.panel_bounds) computed separately == the full SpMM, bitwise."""
+    from paper_conf_sc_chenqldx21_b200 import dist as vsd
+    rng = gen.make_rng(f"gshard_spmm_{V}")
+    M, K, N = 512, 1024, 1000
+    A = gen.colvec_dense(rng, M, K, V, 0.1)
+    B = dev(gen.dense_operand(rng, K, N))
+    rp, ci, va = vs.encode(V, dense=dev(A))
+    full = vs.spmm(rp, ci, va, B, M, V)
+    for P in (2, 3, 8):
+        b = vsd.panel_bounds(N, P)
+        parts = [vs.spmm(rp, ci, va, B[:, b[i]:b[i + 1]].contiguous(), M, V) for i in range(P)]
+        assert torch.equal(torch.cat(parts, dim=1).view(torch.int16), full.view(torch.int16))
+
+
+@pytest.mark.parametrize("V", [2, 8])
+def test_sharded_equals_unsharded_sddmm(vs, V):
+    """Row-window shards (dist.window_bounds) computed separately == the full SDDMM, bitwise."""
+    from paper_conf_sc_chenqldx21_b200 import dist as vsd
+    rng = gen.make_rng(f"gshard_sddmm_{V}")
+    M, N, K = 600, 700, 256
+    mask = gen.colvec_mask(rng, M, N, V, 0.1)
+    A = dev(gen.dense_operand(rng, M, K))
+    Bt = dev(gen.dense_operand(rng, N, K))
+    rp, ci, _ = vs.encode(V, mask=dev(mask))
+    full = vs.sddmm(rp, ci, A, Bt, V)
+    rph = host(rp)
+    for P in (2, 3, 8):
+        wb = vsd.window_bounds(rph, P)
+        segs = []
+        for r in range(P):
+            sh = vsd.sddmm_shard(rph, M, V, wb, r)
+            segs.append(vs.sddmm(dev(sh.row_ptr), ci[sh.p0:sh.p1].contiguous(),
+                                 A[sh.row0:sh.row1].contiguous(), Bt, V, nnz=sh.p1 - sh.p0))
+        assert torch.equal(torch.cat(segs).view(torch.int16), full.view(torch.int16))
+
+
+# ------------------------------------------------- full-size (C5) sampled parity
+
+def test_c5_spmm_sampled(vs):
+    """C5 SpMM at full size (M=K=16384, N=65536, V=8, S=0.9), the launch the sharded bench
+    runs per panel; 4096 sampled outputs against the oracle, plus the adjoint check."""
+    M = K = 16384
+    N, V, S = 65536, 8, 0.9
+    A = gen.torch_colvec_dense(M, K, V, 1 - S, seed=501)
+    B = gen.torch_dense_operand(K, N, seed=502)
+    rp, ci, va = vs.encode(V, dense=A)
+    C = vs.spmm(rp, ci, va, B, M, V)
+    torch.cuda.synchronize()
+    nnz = int(rp[-1].item())
+    assert abs(nnz - (M // V) * K * (1 - S)) < 0.01 * nnz
+    rng = np.random.default_rng(7)
+    rows = rng.integers(0, M, 4096)
+    cols = rng.integers(0, N, 4096)
+    o, s = oracle.spmm_sample(M, K, N, V, host(rp), host(ci)[:nnz], host(va)[:nnz * V],
+                              host(B), rows, cols)
+    g = host(C[torch.from_numpy(rows).cuda(), torch.from_numpy(cols).cuda()])
+    assert_within(g, o, s, "C5 spmm sample")
+    # oracle-free encode check on a slice: GPU encode of the first 64 rows vs oracle encode
+    orp, oci, ova = oracle.encode(64, K, V, dense=host(A[:64]))
+    assert np.array_equal(host(rp[:9]), orp)
+    assert np.array_equal(host(ci[:orp[-1]]), oci)
+
+
+def test_c5_sddmm_sampled(vs):
+    """C5 SDDMM (mask 16384 x 65536, inner K=16384, V=8, S=0.9): 512 sampled vectors."""
+    M, N, K, V, S = 16384, 65536, 16384, 8, 0.9
+    g = torch.Generator(device="cuda")
+    g.manual_seed(503)
+    keep = (torch.rand((M // V, N), generator=g, device="cuda") < (1 - S))
+    mask = keep.repeat_interleave(V, dim=0).to(torch.uint8)
+    del keep
+    rp, ci, _ = vs.encode(V, mask=mask)
+    del mask
+    A = gen.torch_dense_operand(M, K, seed=504)
+    Bt = gen.torch_dense_operand(N, K, seed=505)
+    nnz = int(rp[-1].item())
+    out = vs.sddmm(rp, ci, A, Bt, V, nnz=nnz)
+    torch.cuda.synchronize()
+    ps = np.random.default_rng(8).integers(0, nnz, 512)
+    o, s = oracle.sddmm_sample(M, N, K, V, host(rp), host(ci)[:nnz], host(A), host(Bt), ps)
+    gv = host(out.view(-1, V)[torch.from_numpy(ps).cuda()])
+    assert_within(gv, o, s, "C5 sddmm sample")
