@@ -85,6 +85,71 @@ __device__ __forceinline__ void mma_16816(float (&d)[4], uint32_t a0, uint32_t a
       : "r"(a0), "r"(a1), "r"(a2), "r"(a3), "r"(b0), "r"(b1));
 }
 
+// ---- mbarrier + bulk async copy (global -> shared, completion counted in bytes) ----------
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "WAIT_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      "@!p bra WAIT_%=;\n"
+      "}\n" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+// bytes must be a multiple of 16; src and dst 16-byte aligned
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void cp_async16(void* dst, const void* src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_wait_all() {
+  asm volatile("cp.async.wait_all;" ::: "memory");
+}
+__device__ __forceinline__ uint4 lds128(const void* p) {
+  uint4 r;
+  asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+               : "r"(smem_u32(p)));
+  return r;
+}
+
+// Smallest i in [0, n] with a[i] >= target (a non-decreasing, a[n] treated as +inf).
+// Warp-cooperative 32-ary search; every lane returns the result.
+__device__ __forceinline__ int64_t warp_lower_bound(const int32_t* __restrict__ a, int64_t n,
+                                                    int64_t target) {
+  int64_t lo = 0, hi = n;  // answer in [lo, hi]
+  const int lane = lane_id();
+  while (lo < hi) {
+    const int64_t span = hi - lo;
+    const int64_t step = (span + 31) / 32;
+    const int64_t probe = lo + (int64_t)lane * step;
+    const bool less = (probe < hi) && (a[probe] < target);
+    const unsigned ballot = __ballot_sync(0xffffffffu, less);
+    if (ballot == 0) return lo;  // a[lo] >= target
+    const int last = 31 - __clz(ballot);  // a[lo + last*step] < target
+    lo = lo + (int64_t)last * step + 1;
+    const int64_t nhi = lo - 1 + step;  // probe last+1 (if any) is >= target
+    if (last < 31 && nhi < hi) hi = nhi;
+  }
+  return lo;
+}
+
 __host__ __device__ __forceinline__ int64_t ceil_div64(int64_t a, int64_t b) {
   return (a + b - 1) / b;
 }

@@ -1,12 +1,16 @@
 // encode.cu — dense fp16 matrix / uint8 mask -> column-vector CSR (§4.2, Fig. 8).
 //
-// One kernel (encode_fused, below) with one CTA per row window and one warp per 256-column
-// chunk (up to 8 warps); each lane tests 8 consecutive columns with one 16-byte load per
-// row of the window.  Keep bit = any nonzero fp16 bit pattern (or mask byte) over the
-// window's V rows.  Phase 1 counts the window; a decoupled look-back over row_ptr gives the
-// window's first slot (row_ptr becomes the CSR row pointer in place); phase 2 writes col_idx
-// and the V values of each kept vector (transposed from the V row loads into vector-major
-// order).
+// Two kernels (+ one memset node), both with one CTA per row window and one warp per
+// 256-column chunk (up to 8 warps); each lane tests 8 consecutive columns with one 16-byte
+// load per row of the window.  Keep bit = any nonzero fp16 bit pattern (or mask byte) over
+// the window's V rows.
+//   1. encode_count_scan : counts the window's kept vectors into row_ptr[w+1]; the LAST CTA
+//      to finish (a ticket taken with one atomic on row_ptr[0], preset to -1) turns the counts
+//      into the inclusive prefix in place and sets row_ptr[0] = 0.  No CTA ever waits for
+//      another, so any grid size and any concurrent work on the device are safe.
+//   2. encode_compact    : re-reads the window (L2-resident), block-scans the lanes' keep
+//      counts and writes col_idx and the V values of each kept vector (transposed from the V
+//      row loads into vector-major order) starting at row_ptr[w].
 // Columns are visited in ascending order, so col_idx ascends inside each window (Fig. 8).
 #include "common.cuh"
 
@@ -92,110 +96,59 @@ __device__ __forceinline__ uint32_t window_keep8(const uint16_t* __restrict__ de
   return keep;
 }
 
-// ---------------------------------------------------------------- single-pass encoder
-//
-// encode_fused: one kernel per call.  CTA w counts its window (phase 1), publishes the count,
-// obtains the exclusive prefix of all earlier windows by a decoupled look-back over
-// row_ptr itself, publishes its inclusive prefix, then (phase 2) writes col_idx / vals.
-// row_ptr[w+1] doubles as the look-back status of window w (it is preset to -1 by one
-// memset node):  -1 = nothing yet,  <= -2 = aggregate (count = -s-2) only,  >= 0 = inclusive
-// prefix (final value).  CTAs are dispatched in blockIdx order, so a CTA only waits on CTAs
-// that are already resident or finished.
+// ------------------------------------------------------------------------ kernels
 
-// The status word is the only data exchanged between CTAs, so relaxed gpu-scope accesses
-// suffice (no other memory is published through it); relaxed loads are not serialised the
-// way acquire loads are, so a thread's look-back loads are all in flight at once.
-__device__ __forceinline__ void st_status(int32_t* p, int32_t v) {
-  asm volatile("st.relaxed.gpu.global.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
-__device__ __forceinline__ int32_t ld_status(const int32_t* p) {
-  int32_t v;
-  asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-  return v;
-}
-
-// Exclusive prefix of windows [0, w), computed by the whole CTA (all threads call it; all
-// get the result).  One round reads the statuses of the kLookback nearest predecessors at
-// once (all CTAs of a small problem run concurrently, so the nearest prefix is usually the
-// sentinel P(0) before window 0 and one round suffices); the nearest published prefix ends
-// the walk, aggregates before it are summed.
-constexpr int kLookback = 1024;
-
-__device__ __forceinline__ int64_t lookback(const int32_t* row_ptr, int64_t w, int32_t* s_min,
-                                            int64_t* s_sum) {
+// Inclusive scan of a[0..n) in place by one CTA (all threads call it).
+__device__ void block_scan_inplace(int32_t* a, int64_t n, int32_t* s_warp, int32_t* s_carry) {
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5, nw = blockDim.x >> 5;
-  const int per = kLookback / blockDim.x;  // statuses per thread per round (<= 32)
-  int64_t excl = 0;
-  int64_t j = w - 1;  // nearest window not yet accounted for (its status is row_ptr[j + 1])
-  while (true) {
-    int32_t st[32];
-    int my_first = 0x7fffffff;  // smallest offset o (= j - idx) holding a prefix
-    // issue all loads, then re-poll only the statuses not yet published
-    bool pending = false;
+  if (tid == 0) *s_carry = 0;
+  __syncthreads();
+  constexpr int PER = 4;
+  for (int64_t base = 0; base < n; base += (int64_t)blockDim.x * PER) {
+    int32_t v[PER];
+    int32_t local = 0;
 #pragma unroll
-    for (int q = 0; q < 32; ++q) {
-      if (q >= per) break;
-      const int64_t idx = j - (tid * per + q);
-      // idx == -1: the P(0) sentinel; idx < -1: beyond it, never summed
-      st[q] = idx >= 0 ? ld_status(row_ptr + idx + 1) : 0;
+    for (int j = 0; j < PER; ++j) {
+      const int64_t idx = base + (int64_t)tid * PER + j;
+      v[j] = idx < n ? __ldcg(a + idx) : 0;
+      local += v[j];
     }
+    int32_t incl = local;
 #pragma unroll
-    for (int q = 0; q < 32; ++q) pending |= (q < per) && st[q] == -1;
-    while (pending) {
-      pending = false;
-#pragma unroll
-      for (int q = 0; q < 32; ++q) {
-        if (q >= per) break;
-        if (st[q] == -1) st[q] = ld_status(row_ptr + (j - (tid * per + q)) + 1);
-      }
-#pragma unroll
-      for (int q = 0; q < 32; ++q) pending |= (q < per) && st[q] == -1;
+    for (int o = 1; o < 32; o <<= 1) {
+      const int32_t t = __shfl_up_sync(0xffffffffu, incl, o);
+      if (lane >= o) incl += t;
     }
-#pragma unroll
-    for (int q = 0; q < 32; ++q) {
-      if (q >= per) break;
-      const int o = tid * per + q;
-      if (st[q] >= 0 && o < my_first) my_first = o;
-    }
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) my_first = min(my_first, __shfl_xor_sync(0xffffffffu, my_first, o));
-    if (lane == 0) s_min[wid] = my_first;
+    if (lane == 31) s_warp[wid] = incl;
     __syncthreads();
-    int first = 0x7fffffff;
-    for (int i = 0; i < nw; ++i) first = min(first, s_min[i]);
-    int64_t part = 0;
-#pragma unroll
-    for (int q = 0; q < 32; ++q) {
-      if (q >= per) break;
-      const int o = tid * per + q;
-      const int32_t v = st[q];
-      if (o < first) part += (int64_t)(-v - 2);  // aggregate (only -x-2 values precede first)
-      else if (o == first) part += (int64_t)v;    // the nearest inclusive prefix
+    int32_t before = *s_carry, total = 0;
+    for (int i = 0; i < nw; ++i) {
+      before += (i < wid) ? s_warp[i] : 0;
+      total += s_warp[i];
     }
+    int32_t run = before + incl - local;
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
-    if (lane == 0) s_sum[wid] = part;
+    for (int j = 0; j < PER; ++j) {
+      const int64_t idx = base + (int64_t)tid * PER + j;
+      run += v[j];
+      if (idx < n) a[idx] = run;
+    }
     __syncthreads();
-    for (int i = 0; i < nw; ++i) excl += s_sum[i];
-    __syncthreads();  // s_min / s_sum reused next round
-    if (first != 0x7fffffff) return excl;
-    j -= kLookback;
+    if (tid == 0) *s_carry += total;
+    __syncthreads();
   }
 }
 
-template <int V, bool VEC, bool HAS_MASK, bool WRITE_IDX, bool WRITE_VALS, bool VEC_VALS>
+template <int V, bool VEC, bool HAS_MASK>
 __global__ void __launch_bounds__(kEncMaxThreads)
-    encode_fused_kernel(int64_t M, int64_t K, const uint16_t* __restrict__ dense,
-                        const uint8_t* __restrict__ mask, int32_t* __restrict__ row_ptr,
-                        int32_t* __restrict__ col_idx, uint16_t* __restrict__ vals) {
-  __shared__ uint32_t warp_cnt[kEncMaxThreads / 32];
-  __shared__ int32_t s_min[kEncMaxThreads / 32];
-  __shared__ int64_t s_sum[kEncMaxThreads / 32];
+    encode_count_scan_kernel(int64_t M, int64_t K, int64_t W, const uint16_t* __restrict__ dense,
+                             const uint8_t* __restrict__ mask, int32_t* __restrict__ row_ptr) {
+  __shared__ int32_t s_warp[kEncMaxThreads / 32];
+  __shared__ int32_t s_carry;
+  __shared__ int s_last;
   const int lane = lane_id(), wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
   const int64_t w = blockIdx.x;
   uint16_t h[V][8];
-
-  // phase 1: count the window's kept vectors
   uint32_t count = 0;
   for (int64_t c0 = (int64_t)wid * kColsPerStep; c0 < K; c0 += (int64_t)nw * kColsPerStep) {
     const int64_t c = c0 + lane * kColsPerLane;
@@ -203,25 +156,36 @@ __global__ void __launch_bounds__(kEncMaxThreads)
   }
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) count += __shfl_xor_sync(0xffffffffu, count, o);
-  if (lane == 0) warp_cnt[wid] = count;
+  if (lane == 0) s_warp[wid] = (int32_t)count;
   __syncthreads();
-  uint32_t tot = 0;
-  for (int i = 0; i < nw; ++i) tot += warp_cnt[i];
-  int64_t base;
-  if (w == 0) {
-    if (threadIdx.x == 0) {
-      st_status(row_ptr + 1, (int32_t)tot);
-      row_ptr[0] = 0;
-    }
-    base = 0;
-  } else {
-    if (threadIdx.x == 0) st_status(row_ptr + w + 1, -(int32_t)tot - 2);  // aggregate
-    base = lookback(row_ptr, w, s_min, s_sum);
-    if (threadIdx.x == 0) st_status(row_ptr + w + 1, (int32_t)(base + tot));  // inclusive prefix
+  if (threadIdx.x == 0) {
+    int32_t tot = 0;
+    for (int i = 0; i < nw; ++i) tot += s_warp[i];
+    row_ptr[w + 1] = tot;
+    __threadfence();  // publish the count before taking the ticket
+    const int ticket = atomicAdd(row_ptr, 1);  // row_ptr[0] was preset to -1
+    s_last = (ticket == (int)(W - 2));
   }
-  if (!WRITE_IDX) return;
+  __syncthreads();
+  if (!s_last) return;
+  __threadfence();  // all counts are visible to the last CTA
+  block_scan_inplace(row_ptr + 1, W, s_warp, &s_carry);
+  if (threadIdx.x == 0) row_ptr[0] = 0;
+}
 
-  // phase 2: write col_idx / vals (re-reads the window, now L1/L2 resident)
+// Writes col_idx and (optionally) vals of window w from row_ptr[w] on.  Per round, warp i
+// takes chunk (round * nwarps + i); a block-wide exclusive scan of the warps' keep counts
+// gives each warp its slot range, so col_idx stays ascending.
+template <int V, bool VEC, bool HAS_MASK, bool WRITE_VALS, bool VEC_VALS>
+__global__ void __launch_bounds__(kEncMaxThreads)
+    encode_compact_kernel(int64_t M, int64_t K, const uint16_t* __restrict__ dense,
+                          const uint8_t* __restrict__ mask, const int32_t* __restrict__ row_ptr,
+                          int32_t* __restrict__ col_idx, uint16_t* __restrict__ vals) {
+  __shared__ uint32_t warp_cnt[kEncMaxThreads / 32];
+  const int lane = lane_id(), wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  const int64_t w = blockIdx.x;
+  int64_t base = row_ptr[w];
+  uint16_t h[V][8];
   for (int64_t r0 = 0; r0 < K; r0 += (int64_t)nw * kColsPerStep) {
     const int64_t c = r0 + (int64_t)wid * kColsPerStep + lane * kColsPerLane;
     const uint32_t keep = window_keep8<V, VEC, HAS_MASK, WRITE_VALS>(dense, mask, M, K, w, c, h);
@@ -232,7 +196,6 @@ __global__ void __launch_bounds__(kEncMaxThreads)
       const uint32_t t = __shfl_up_sync(0xffffffffu, incl, o);
       if (lane >= o) incl += t;
     }
-    __syncthreads();  // previous round's readers of warp_cnt are done
     if (lane == 31) warp_cnt[wid] = incl;
     __syncthreads();
     uint32_t before = 0, total = 0;
@@ -265,27 +228,24 @@ __global__ void __launch_bounds__(kEncMaxThreads)
       }
     }
     base += total;
+    __syncthreads();  // warp_cnt is rewritten next round
   }
 }
 
 // ---------------------------------------------------------------- host-side launchers
 
 template <int V, bool VEC, bool MASKB>
-static void launch_fused(int64_t M, int64_t K, int64_t W, const uint16_t* dense, const uint8_t* mask,
-                         int32_t* row_ptr, int32_t* col_idx, uint16_t* vals, bool vec_vals,
-                         dim3 grid, dim3 block, cudaStream_t s) {
-  if (col_idx == nullptr)
-    encode_fused_kernel<V, VEC, MASKB, false, false, false><<<grid, block, 0, s>>>(
-        M, K, dense, mask, row_ptr, col_idx, vals);
-  else if (vals == nullptr)
-    encode_fused_kernel<V, VEC, MASKB, true, false, false><<<grid, block, 0, s>>>(
-        M, K, dense, mask, row_ptr, col_idx, vals);
+static void launch_v(int64_t M, int64_t K, int64_t W, const uint16_t* dense, const uint8_t* mask,
+                     int32_t* row_ptr, int32_t* col_idx, uint16_t* vals, bool vec_vals, dim3 grid,
+                     dim3 block, cudaStream_t s) {
+  encode_count_scan_kernel<V, VEC, MASKB><<<grid, block, 0, s>>>(M, K, W, dense, mask, row_ptr);
+  if (col_idx == nullptr) return;
+  if (vals == nullptr)
+    encode_compact_kernel<V, VEC, MASKB, false, false><<<grid, block, 0, s>>>(M, K, dense, mask, row_ptr, col_idx, vals);
   else if (vec_vals)
-    encode_fused_kernel<V, VEC, MASKB, true, true, true><<<grid, block, 0, s>>>(
-        M, K, dense, mask, row_ptr, col_idx, vals);
+    encode_compact_kernel<V, VEC, MASKB, true, true><<<grid, block, 0, s>>>(M, K, dense, mask, row_ptr, col_idx, vals);
   else
-    encode_fused_kernel<V, VEC, MASKB, true, true, false><<<grid, block, 0, s>>>(
-        M, K, dense, mask, row_ptr, col_idx, vals);
+    encode_compact_kernel<V, VEC, MASKB, true, false><<<grid, block, 0, s>>>(M, K, dense, mask, row_ptr, col_idx, vals);
 }
 
 template <int V>
@@ -300,16 +260,16 @@ static cudaError_t launch_encode_v(int64_t M, int64_t K, const uint16_t* dense, 
   const int threads =
       (int)(32 * (chunks < 1 ? 1 : (chunks > kEncMaxThreads / 32 ? kEncMaxThreads / 32 : chunks)));
   dim3 grid((unsigned)W), block(threads);
-  // look-back status: row_ptr[1..W] = -1 ("nothing published yet")
-  cudaError_t e = cudaMemsetAsync(row_ptr + 1, 0xFF, (size_t)W * sizeof(int32_t), s);
+  // row_ptr[0] = -1: the ticket counter of encode_count_scan (reset to 0 by the last CTA)
+  cudaError_t e = cudaMemsetAsync(row_ptr, 0xFF, sizeof(int32_t), s);
   if (e != cudaSuccess) return e;
   const bool has_mask = mask != nullptr;
   if (vec) {
-    if (has_mask) launch_fused<V, true, true>(M, K, W, dense, mask, row_ptr, col_idx, vals, vec_vals, grid, block, s);
-    else launch_fused<V, true, false>(M, K, W, dense, mask, row_ptr, col_idx, vals, vec_vals, grid, block, s);
+    if (has_mask) launch_v<V, true, true>(M, K, W, dense, mask, row_ptr, col_idx, vals, vec_vals, grid, block, s);
+    else launch_v<V, true, false>(M, K, W, dense, mask, row_ptr, col_idx, vals, vec_vals, grid, block, s);
   } else {
-    if (has_mask) launch_fused<V, false, true>(M, K, W, dense, mask, row_ptr, col_idx, vals, vec_vals, grid, block, s);
-    else launch_fused<V, false, false>(M, K, W, dense, mask, row_ptr, col_idx, vals, vec_vals, grid, block, s);
+    if (has_mask) launch_v<V, false, true>(M, K, W, dense, mask, row_ptr, col_idx, vals, vec_vals, grid, block, s);
+    else launch_v<V, false, false>(M, K, W, dense, mask, row_ptr, col_idx, vals, vec_vals, grid, block, s);
   }
   return cudaGetLastError();
 }

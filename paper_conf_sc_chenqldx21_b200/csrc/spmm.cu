@@ -214,7 +214,7 @@ static void launch_cfg(int64_t M, int64_t N, int64_t W, const int32_t* row_ptr,
 // the shipped configuration): VS_SPMM_UNROLL in {1,2}, VS_SPMM_NC in {0 (auto),1,2},
 // VS_SPMM_SPLIT_SHIFT (SPLIT = K >> shift, clamped to [1,16] and rounded down to a power of 2).
 struct SpmmTune {
-  int unroll = 2, nc = 1, split_shift = 8;
+  int unroll = 1, nc = 0, split_shift = 8;
 };
 static const SpmmTune& spmm_tune() {
   static const SpmmTune t = [] {
@@ -260,8 +260,9 @@ static void launch_unroll(int64_t M, int64_t K, int64_t N, int64_t W, const int3
 template <int V>
 static cudaError_t launch_spmm_v(int64_t M, int64_t K, int64_t N, const int32_t* row_ptr,
                                  const int32_t* col_idx, const uint16_t* vals, const uint16_t* B,
-                                 uint16_t* C, bool vec, cudaStream_t s) {
+                                 uint16_t* C, bool vec, int num_sms, cudaStream_t s) {
   const int64_t W = ceil_div64(M, V);
+  (void)num_sms;
   const int NC = spmm_tune().nc == 0 ? ((N <= 64) ? 1 : 2) : (spmm_tune().nc == 2 && N > 64 ? 2 : 1);
   if (ceil_div64(N, 64 * NC) * W > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
   if (NC == 1) {
@@ -276,17 +277,17 @@ static cudaError_t launch_spmm_v(int64_t M, int64_t K, int64_t N, const int32_t*
 
 cudaError_t launch_spmm(int64_t M, int64_t K, int64_t N, int V, const int32_t* row_ptr,
                         const int32_t* col_idx, const void* vals, const void* B, void* C,
-                        cudaStream_t s) {
+                        int num_sms, cudaStream_t s) {
   const uint16_t* v = static_cast<const uint16_t*>(vals);
   const uint16_t* b = static_cast<const uint16_t*>(B);
   uint16_t* c = static_cast<uint16_t*>(C);
   const bool vec = (N % 8 == 0) && ((reinterpret_cast<uintptr_t>(B) & 15) == 0) &&
                    ((reinterpret_cast<uintptr_t>(C) & 15) == 0);
   switch (V) {
-    case 1: return launch_spmm_v<1>(M, K, N, row_ptr, col_idx, v, b, c, vec, s);
-    case 2: return launch_spmm_v<2>(M, K, N, row_ptr, col_idx, v, b, c, vec, s);
-    case 4: return launch_spmm_v<4>(M, K, N, row_ptr, col_idx, v, b, c, vec, s);
-    case 8: return launch_spmm_v<8>(M, K, N, row_ptr, col_idx, v, b, c, vec, s);
+    case 1: return launch_spmm_v<1>(M, K, N, row_ptr, col_idx, v, b, c, vec, num_sms, s);
+    case 2: return launch_spmm_v<2>(M, K, N, row_ptr, col_idx, v, b, c, vec, num_sms, s);
+    case 4: return launch_spmm_v<4>(M, K, N, row_ptr, col_idx, v, b, c, vec, num_sms, s);
+    case 8: return launch_spmm_v<8>(M, K, N, row_ptr, col_idx, v, b, c, vec, num_sms, s);
   }
   return cudaErrorInvalidValue;
 }

@@ -10,7 +10,7 @@ cudaError_t launch_encode(int64_t M, int64_t K, int V, const void* dense, const 
                           int32_t* row_ptr, int32_t* col_idx, void* vals, cudaStream_t s);
 cudaError_t launch_spmm(int64_t M, int64_t K, int64_t N, int V, const int32_t* row_ptr,
                         const int32_t* col_idx, const void* vals, const void* B, void* C,
-                        cudaStream_t s);
+                        int num_sms, cudaStream_t s);
 cudaError_t launch_sddmm(int64_t M, int64_t N, int64_t K, int V, const int32_t* row_ptr,
                          const int32_t* col_idx, const void* A, const void* Bt, void* out,
                          int num_sms, cudaStream_t s);
@@ -115,7 +115,7 @@ vs_status_t vs_spmm(int64_t M, int64_t K, int64_t N, int V, const int32_t* row_p
   if (st != VS_SUCCESS) return st;
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   if (K == 0) return from_cuda(cudaMemsetAsync(C, 0, (size_t)(M * N) * 2, s));
-  return from_cuda(vs::launch_spmm(M, K, N, V, row_ptr, col_idx, vals, B, C, s));
+  return from_cuda(vs::launch_spmm(M, K, N, V, row_ptr, col_idx, vals, B, C, info.num_sms, s));
 }
 
 vs_status_t vs_sddmm(int64_t M, int64_t N, int64_t K, int V, const int32_t* row_ptr,

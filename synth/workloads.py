@@ -67,7 +67,18 @@ def c5_problem():
     return Problem(16384, 16384, 65536, 8, 0.9)
 
 
+def custom_workload():
+    """Problems from the environment: VS_PROBLEMS="M,K,N,V,S;M,K,N,V,S" (tuning/profiling)."""
+    import os
+    out = []
+    for item in filter(None, os.environ.get("VS_PROBLEMS", "").split(";")):
+        M, K, N, V, S = item.split(",")
+        out.append(Problem(int(M), int(K), int(N), int(V), float(S)))
+    return out
+
+
 WORKLOADS = {
+    "custom": custom_workload,
     "dlmc_layer": dlmc_layer_workload,
     "rn50_layer": rn50_workload,
     "c1": lambda: [c1_problem()],
