@@ -169,6 +169,25 @@ def alg_bytes(p, nnz_v, k_ref):
     return {"encode": encode, "spmm": spmm, "sddmm": sddmm}
 
 
+def count_launches(bufs):
+    """Kernel launches of one batched step, by the library's grouping rules (vs_api.cu):
+    encode groups by V (3 kernels per group of <= 128 problems: ticket init, count+scan,
+    compact), SpMM by (V, panel width NC from N, SPLIT from K), SDDMM by V (1 kernel per
+    group of <= 128)."""
+    import math as _m
+    from collections import Counter
+    def split(K):
+        q = K >> 8
+        return 16 if q >= 16 else 8 if q >= 8 else 4 if q >= 4 else 2 if q >= 2 else 1
+    enc = Counter(b.p.V for b in bufs)
+    sp = Counter((b.p.V, 1 if b.p.N <= 64 else 2, split(b.p.K)) for b in bufs)
+    sd = Counter(b.p.V for b in bufs)
+    per = {"encode": sum(3 * _m.ceil(n / 128) for n in enc.values()),
+           "spmm": sum(_m.ceil(n / 128) for n in sp.values()),
+           "sddmm": sum(_m.ceil(n / 128) for n in sd.values())}
+    return {"per_class": per, "total": sum(per.values())}
+
+
 # --------------------------------------------------------------- reference (oracle) arm
 
 _INPUT_CACHE = {}
@@ -342,54 +361,62 @@ def run_ours(args):
     flops_spmm = sum(problem_flops(b.nnz_v, b.p)[0] for b in bufs)
     flops_sddmm = sum(problem_flops(b.nnz_v, b.p)[1] for b in bufs)
     flops_step = flops_spmm + flops_sddmm
-    launches_per_step = len(bufs) * 3  # encode_fused (+ one memset node), spmm, sddmm
+    launches_per_step = count_launches(bufs)
 
-    def step_serial():
-        for b in bufs:
-            b.encode(vs)
-            b.spmm(vs)
-            b.sddmm(vs)
+    # the step through the batched C ABI: one encode batch, then the SpMM batch and (on a
+    # forked graph branch, it only needs the encoding) the SDDMM batch
+    enc_arr = vs.make_encode_batch([(b.p.M, b.p.K, b.p.V, b.Wd, None, b.row_ptr, b.col_idx, b.vals)
+                                    for b in bufs])
+    spmm_arr = vs.make_spmm_batch([(b.p.M, b.p.K, b.p.N, b.p.V, b.row_ptr, b.col_idx, b.vals, b.X, b.Y)
+                                   for b in bufs])
+    sddmm_arr = vs.make_sddmm_batch([(b.p.M, b.p.K, b.p.N, b.p.V, b.row_ptr, b.col_idx, b.G, b.X, b.dW)
+                                     for b in bufs])
+    side = torch.cuda.Stream()
 
+    def step_batched(pre=None, post=None):
+        cur = torch.cuda.current_stream()
+        if pre:
+            pre()
+        vs.vs_encode_colvec_batched(enc_arr)
+        side.wait_stream(cur)
+        vs.vs_spmm_batched(spmm_arr)
+        with torch.cuda.stream(side):
+            vs.vs_sddmm_batched(sddmm_arr)
+        cur.wait_stream(side)
+        if post:
+            post()
+
+    # per-problem calls (single entry points) on 8 concurrent graph branches: comparison only
     branches = [torch.cuda.Stream() for _ in range(max(1, args.streams))]
 
-    def forked(body):
-        """Runs body(b) for every problem, problem i on branch i % S (independent problems
-        become parallel branches of the captured graph)."""
-        def run():
-            cur = torch.cuda.current_stream()
-            for st in branches:
-                st.wait_stream(cur)
-            for i, b in enumerate(bufs):
-                with torch.cuda.stream(branches[i % len(branches)]):
-                    body(b)
-            for st in branches:
-                cur.wait_stream(st)
-        return run
+    def step_per_problem():
+        cur = torch.cuda.current_stream()
+        for st in branches:
+            st.wait_stream(cur)
+        for i, b in enumerate(bufs):
+            with torch.cuda.stream(branches[i % len(branches)]):
+                b.encode(vs)
+                b.spmm(vs)
+                b.sddmm(vs)
+        for st in branches:
+            cur.wait_stream(st)
 
-    def body(b):
-        b.encode(vs)
-        b.spmm(vs)
-        b.sddmm(vs)
-
-    step = forked(body)
-
-    # instrumented copy of the step: external events around every ABI call
+    # instrumented serial copy of the batched step: external events around each batched call
     ev = []
 
     def step_instr():
-        for b in bufs:
-            row = []
-            for name, fn in (("encode", b.encode), ("spmm", b.spmm), ("sddmm", b.sddmm)):
-                s = torch.cuda.Event(enable_timing=True, external=True)
-                e = torch.cuda.Event(enable_timing=True, external=True)
-                s.record()
-                fn(vs)
-                e.record()
-                row.append((name, s, e))
-            ev.append(row)
+        for name, fn in (("encode", lambda: vs.vs_encode_colvec_batched(enc_arr)),
+                         ("spmm", lambda: vs.vs_spmm_batched(spmm_arr)),
+                         ("sddmm", lambda: vs.vs_sddmm_batched(sddmm_arr))):
+            s0 = torch.cuda.Event(enable_timing=True, external=True)
+            e0 = torch.cuda.Event(enable_timing=True, external=True)
+            s0.record()
+            fn()
+            e0.record()
+            ev.append((name, s0, e0))
 
-    g_step = capture(torch, step, stream)
-    g_serial = capture(torch, step_serial, stream)
+    g_step = capture(torch, step_batched, stream)
+    g_pp = capture(torch, step_per_problem, stream)
     g_instr = capture(torch, step_instr, stream)
     flush = torch.empty(512 * 1024 * 1024 // 4, dtype=torch.int32, device=dev)
 
@@ -397,7 +424,7 @@ def run_ours(args):
         with torch.cuda.stream(stream):
             flush.fill_(i)
             g_step.replay()
-            g_serial.replay()
+            g_pp.replay()
             g_instr.replay()
     stream.synchronize()
 
@@ -411,7 +438,6 @@ def run_ours(args):
         bus = "%08X:%02X:%02X.0" % (getattr(props, "pci_domain_id", 0), props.pci_bus_id,
                                    getattr(props, "pci_device_id", 0))
     clocks = ClockSampler(dev.index if ws == 1 else local, bus).start()
-    step_ms = []
     starts = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
     ends = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
     with torch.cuda.stream(stream):
@@ -421,27 +447,21 @@ def run_ours(args):
             g_step.replay()
             ends[i].record()
     torch.cuda.synchronize()
-    step_ms = [s.elapsed_time(e) for s, e in zip(starts, ends)]
-    serial_ms = []
+    step_ms = [s0.elapsed_time(e0) for s0, e0 in zip(starts, ends)]
+    pp_ms = []
     for i in range(args.steps):
         with torch.cuda.stream(stream):
             flush.fill_(i + 5)
-        serial_ms.append(time_graph(torch, g_serial, stream))
+        pp_ms.append(time_graph(torch, g_pp, stream))
     # instrumented replays (same inputs) for the per-kernel attribution
     per_class = {"encode": [], "spmm": [], "sddmm": []}
-    per_launch = []
     for i in range(args.steps):
         with torch.cuda.stream(stream):
             flush.fill_(i + 7)
             g_instr.replay()
         stream.synchronize()
-        row_ms = []
-        for b, row in zip(bufs, ev):
-            d = {name: s.elapsed_time(e) for name, s, e in row}
-            for k, v in d.items():
-                per_class[k].append(v)
-            row_ms.append(d)
-        per_launch.append(row_ms)
+        for name, s0, e0 in ev:
+            per_class[name].append(s0.elapsed_time(e0))
     if ws > 1:
         torch.distributed.barrier()
     torch.cuda.synchronize()
@@ -454,7 +474,7 @@ def run_ours(args):
         total_ms = float(t.item())
     ms_per_step = total_ms / args.steps
     value = ws * flops_step / (ms_per_step * 1e-3) / 1e12
-    ms_serial = sum(serial_ms) / args.steps
+    ms_pp = sum(pp_ms) / args.steps
 
     # ---------------- kernel attribution + roofline ----------------
     nb = len(bufs)
@@ -466,18 +486,22 @@ def run_ours(args):
         for k, v in alg_bytes(b.p, b.nnz_v, b.k_ref).items():
             bytes_cls[k] += v
     flops_cls = {"encode": 0.0, "spmm": flops_spmm, "sddmm": flops_sddmm}
-    dom_avg_ms = cls_ms[dominant] / nb
-    achieved_gbs = (bytes_cls[dominant] / nb) / (dom_avg_ms * 1e-3) / 1e9
+    n_launch = launches_per_step["per_class"][dominant]
+    dom_avg_ms = cls_ms[dominant] / n_launch
+    achieved_gbs = (bytes_cls[dominant] / n_launch) / (dom_avg_ms * 1e-3) / 1e9
     traffic = None
     tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(tp):
-        traffic = json.load(open(tp)).get(f"{args.workload}:{dominant}")
+        tr = json.load(open(tp)).get(f"{args.workload}:{dominant}")
+        if tr is not None:
+            traffic = tr / n_launch
     roofline = {"bound": "hbm", "achieved": achieved_gbs, "peak": peaks["hbm_gbs"],
                 "unit": "GB/s", "frac": achieved_gbs / peaks["hbm_gbs"], "traffic": traffic,
                 "kernel": dominant, "peak_source": peaks["source"],
-                "algorithmic_bytes_per_launch": bytes_cls[dominant] / nb,
+                "launches_per_step": n_launch,
+                "algorithmic_bytes_per_launch": bytes_cls[dominant] / n_launch,
                 "avg_launch_us": dom_avg_ms * 1e3}
-    tensor_tf = (flops_cls[dominant] / nb) / (dom_avg_ms * 1e-3) / 1e12 if flops_cls[dominant] else 0.0
+    tensor_tf = flops_cls[dominant] / (cls_ms[dominant] * 1e-3) / 1e12 if flops_cls[dominant] else 0.0
     roofline_tensor = {"bound": "tensor", "achieved": tensor_tf, "peak": peaks["bf16_tflops"],
                        "unit": "TFLOP/s", "frac": tensor_tf / peaks["bf16_tflops"],
                        "kernel": dominant}
@@ -491,40 +515,40 @@ def run_ours(args):
                              "x S{.5,.7,.9,.98} x N{64,128,256}" if args.workload == "dlmc_layer" else args.workload,
                    "step": "per problem: encode W -> SpMM Y=WX -> SDDMM dW=(G X^T) o pattern(W)",
                    "flops_per_step": flops_step, "l2": "flushed between timed steps (512 MiB write, untimed)",
-                   "launch": f"step replayed as one CUDA graph with {len(branches)} concurrent "
-                             "branches over the independent problems",
+                   "launch": "batched C ABI (vs_*_batched), step replayed as one CUDA graph; "
+                             "SDDMM batch on a forked branch concurrent with the SpMM batch",
                    "accumulate": "fp32"},
-        "serial": {"ms_per_step": ms_serial, "value": ws * flops_step / (ms_serial * 1e-3) / 1e12,
-                   "note": "same step as one serial graph (no cross-problem concurrency)"},
+        "per_problem_calls": {"ms_per_step": ms_pp, "value": ws * flops_step / (ms_pp * 1e-3) / 1e12,
+                              "note": "same step through the single-problem entry points, "
+                                      f"{len(branches)} concurrent graph branches"},
         "roofline": roofline,
         "roofline_tensor": roofline_tensor,
         "kernels": {k: {"ms_per_step": v, "share": (v / instr_total if instr_total else None),
-                        "tflops": (flops_cls[k] / (v * 1e-3) / 1e12 if v and flops_cls[k] else None)}
+                        "launches_per_step": launches_per_step["per_class"][k],
+                        "tflops": (flops_cls[k] / (v * 1e-3) / 1e12 if v and flops_cls[k] else None),
+                        "alg_GBps": bytes_cls[k] / (v * 1e-3) / 1e9 if v else None}
                     for k, v in cls_ms.items()},
-        "gpu_launches": launches_per_step * args.steps,
+        "gpu_launches": launches_per_step["total"] * args.steps,
         "clocks": clk,
     }
 
     detail = {"problems": [], "step_ms": step_ms}
     for b in bufs:
         detail["problems"].append({**b.p.asdict(), "nnz_v": b.nnz_v, "k_ref": b.k_ref})
-    for j in range(nb):
-        for k in ("encode", "spmm", "sddmm"):
-            detail["problems"][j][f"{k}_us"] = 1e3 * statistics.median(
-                per_launch[i][j][k] for i in range(args.steps))
 
     # ---------------- end to end with host buffers ----------------
     if not args.no_e2e:
-        def body_e2e(b):
-            b.Wd.copy_(b.h_Wd, non_blocking=True)
-            b.X.copy_(b.h_X, non_blocking=True)
-            b.G.copy_(b.h_G, non_blocking=True)
-            b.encode(vs)
-            b.spmm(vs)
-            b.sddmm(vs)
-            b.h_Y.copy_(b.Y, non_blocking=True)
-            b.h_dW.copy_(b.dW[:b.nnz_v * b.p.V], non_blocking=True)
-        g_e2e = capture(torch, forked(body_e2e), stream)
+        def h2d():
+            for b in bufs:
+                b.Wd.copy_(b.h_Wd, non_blocking=True)
+                b.X.copy_(b.h_X, non_blocking=True)
+                b.G.copy_(b.h_G, non_blocking=True)
+
+        def d2h():
+            for b in bufs:
+                b.h_Y.copy_(b.Y, non_blocking=True)
+                b.h_dW.copy_(b.dW[:b.nnz_v * b.p.V], non_blocking=True)
+        g_e2e = capture(torch, lambda: step_batched(h2d, d2h), stream)
         with torch.cuda.stream(stream):
             g_e2e.replay()
         stream.synchronize()
@@ -538,12 +562,13 @@ def run_ours(args):
             t = torch.tensor([e2e_total], device=dev, dtype=torch.float64)
             torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
             e2e_total = float(t.item())
-        h2d = sum(2 * (b.p.M * b.p.K + b.p.K * b.p.N + b.p.M * b.p.N) for b in bufs)
-        d2h = sum(2 * (b.p.M * b.p.N + b.nnz_v * b.p.V) for b in bufs)
+        h2d_b = sum(2 * (b.p.M * b.p.K + b.p.K * b.p.N + b.p.M * b.p.N) for b in bufs)
+        d2h_b = sum(2 * (b.p.M * b.p.N + b.nnz_v * b.p.V) for b in bufs)
         line["e2e"] = {"value": ws * flops_step / (e2e_total / args.steps * 1e-3) / 1e12,
-                       "unit": UNIT, "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+                       "unit": UNIT, "h2d_bytes_per_step": h2d_b, "d2h_bytes_per_step": d2h_b,
                        "ms_per_step": e2e_total / args.steps,
-                       "path": "pinned host -> device copies, C-ABI calls, device -> pinned host, one CUDA graph"}
+                       "path": "pinned host -> device copies, batched C-ABI calls, device -> "
+                               "pinned host, one CUDA graph"}
 
     # ---------------- same-box library baselines, per cell ----------------
     if not args.no_baselines and rank == 0:

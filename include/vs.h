@@ -133,6 +133,57 @@ vs_status_t vs_sddmm(int64_t M, int64_t N, int64_t K, int V,
                      const int32_t* row_ptr, const int32_t* col_idx,
                      const void* A, const void* Bt, void* out_vals, vs_stream_t stream);
 
+/*
+ * Batched entry points: many independent problems per call (SURVEY §8(f) rank 3 — the
+ * DLMC-sized problems of the paper's benchmarks, are launch-latency bound on
+ * B200 one at a time).
+ *
+ *   problems : HOST array of `count` descriptors, read during the call only.  Each entry has
+ *              exactly the semantics, preconditions and alignment rules of the single call;
+ *              problems may differ in every field and must not write overlapping outputs.
+ *   The library groups the problems by kernel configuration and launches one kernel per
+ *   group of up to 128 problems (the descriptors travel as a kernel parameter).  Results
+ *   are bitwise identical to calling the single entry point once per problem.
+ *   Errors: every entry is checked before anything is enqueued; the first invalid entry
+ *   makes the call return its status (VS_ERROR_INVALID_VALUE / VS_ERROR_MISALIGNED).
+ *   count == 0 is a no-op.  Asynchronous; the encoder batch never returns nnz_v.
+ */
+typedef struct {
+  int64_t M, K, N;
+  int32_t V, reserved;
+  const int32_t* row_ptr;
+  const int32_t* col_idx;
+  const void* vals;
+  const void* B;
+  void* C;
+} vs_spmm_problem_t;
+
+typedef struct {
+  int64_t M, N, K;
+  int32_t V, reserved;
+  const int32_t* row_ptr;
+  const int32_t* col_idx;
+  const void* A;
+  const void* Bt;
+  void* out_vals;
+} vs_sddmm_problem_t;
+
+typedef struct {
+  int64_t M, K;
+  int32_t V, reserved;
+  const void* dense;
+  const uint8_t* mask;
+  int32_t* row_ptr;
+  int32_t* col_idx; /* NULL: count mode (row_ptr only) */
+  void* vals;
+} vs_encode_problem_t;
+
+vs_status_t vs_spmm_batched(int64_t count, const vs_spmm_problem_t* problems, vs_stream_t stream);
+vs_status_t vs_sddmm_batched(int64_t count, const vs_sddmm_problem_t* problems,
+                             vs_stream_t stream);
+vs_status_t vs_encode_colvec_batched(int64_t count, const vs_encode_problem_t* problems,
+                                     vs_stream_t stream);
+
 #ifdef __cplusplus
 }
 #endif

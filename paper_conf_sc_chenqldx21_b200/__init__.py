@@ -22,6 +22,7 @@ import os
 import threading
 
 __all__ = ["VSError", "lib_path", "load", "vs_encode_colvec", "vs_spmm", "vs_sddmm",
+           "vs_encode_colvec_batched", "vs_spmm_batched", "vs_sddmm_batched",
            "encode", "spmm", "sddmm", "num_windows"]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
@@ -31,6 +32,29 @@ _lock = threading.Lock()
 
 _P = ctypes.c_void_p
 _I64 = ctypes.c_int64
+
+class SpmmProblem(ctypes.Structure):
+    """vs_spmm_problem_t"""
+    _fields_ = [("M", ctypes.c_int64), ("K", ctypes.c_int64), ("N", ctypes.c_int64),
+                ("V", ctypes.c_int32), ("reserved", ctypes.c_int32), ("row_ptr", ctypes.c_void_p),
+                ("col_idx", ctypes.c_void_p), ("vals", ctypes.c_void_p), ("B", ctypes.c_void_p),
+                ("C", ctypes.c_void_p)]
+
+
+class SddmmProblem(ctypes.Structure):
+    """vs_sddmm_problem_t"""
+    _fields_ = [("M", ctypes.c_int64), ("N", ctypes.c_int64), ("K", ctypes.c_int64),
+                ("V", ctypes.c_int32), ("reserved", ctypes.c_int32), ("row_ptr", ctypes.c_void_p),
+                ("col_idx", ctypes.c_void_p), ("A", ctypes.c_void_p), ("Bt", ctypes.c_void_p),
+                ("out_vals", ctypes.c_void_p)]
+
+
+class EncodeProblem(ctypes.Structure):
+    """vs_encode_problem_t"""
+    _fields_ = [("M", ctypes.c_int64), ("K", ctypes.c_int64), ("V", ctypes.c_int32),
+                ("reserved", ctypes.c_int32), ("dense", ctypes.c_void_p), ("mask", ctypes.c_void_p),
+                ("row_ptr", ctypes.c_void_p), ("col_idx", ctypes.c_void_p), ("vals", ctypes.c_void_p)]
+
 
 STATUS = {0: "VS_SUCCESS", 1: "VS_ERROR_INVALID_VALUE", 2: "VS_ERROR_NOT_SUPPORTED",
           3: "VS_ERROR_CUDA", 4: "VS_ERROR_MISALIGNED"}
@@ -62,6 +86,11 @@ def load():
             L.vs_spmm.argtypes = [_I64, _I64, _I64, ctypes.c_int, _P, _P, _P, _P, _P, _P]
             L.vs_sddmm.restype = ctypes.c_int
             L.vs_sddmm.argtypes = [_I64, _I64, _I64, ctypes.c_int, _P, _P, _P, _P, _P, _P]
+            for name, st in (("vs_spmm_batched", SpmmProblem), ("vs_sddmm_batched", SddmmProblem),
+                             ("vs_encode_colvec_batched", EncodeProblem)):
+                f = getattr(L, name)
+                f.restype = ctypes.c_int
+                f.argtypes = [_I64, ctypes.POINTER(st), _P]
             _lib = L
     return _lib
 
@@ -90,6 +119,12 @@ def _ptr(t, dtype=None, name="tensor"):
     if not t.is_contiguous():
         raise ValueError(f"{name} must be contiguous")
     return ctypes.c_void_p(t.data_ptr()) if t.numel() > 0 else None
+
+
+def _addr(t, dtype=None, name="tensor"):
+    """_ptr() as a plain integer (or None) for ctypes structure fields."""
+    p = _ptr(t, dtype, name)
+    return None if p is None else p.value
 
 
 def num_windows(M: int, V: int) -> int:
@@ -128,6 +163,64 @@ def vs_sddmm(M, N, K, V, row_ptr, col_idx, A, Bt, out_vals, stream=None):
                          _ptr(Bt, torch.float16, "Bt"), _ptr(out_vals, torch.float16, "out_vals"),
                          _stream(stream))
     _check(st, "vs_sddmm")
+
+
+# ------------------------------------------------------------------ batched mirrors
+#
+# Each takes a list of per-problem tuples in the order of the C struct fields (tensors for
+# pointers, None for NULL).  Build the ctypes array once with make_*_batch() and pass it to
+# the vs_*_batched() call to keep the per-call marshalling cost off a hot loop.
+
+def make_spmm_batch(problems):
+    """problems: [(M, K, N, V, row_ptr, col_idx, vals, B, C), ...]"""
+    import torch
+    arr = (SpmmProblem * len(problems))()
+    for i, (M, K, N, V, rp, ci, va, B, C) in enumerate(problems):
+        arr[i] = SpmmProblem(int(M), int(K), int(N), int(V), 0, _addr(rp, torch.int32, "row_ptr"),
+                             _addr(ci, torch.int32, "col_idx"), _addr(va, torch.float16, "vals"),
+                             _addr(B, torch.float16, "B"), _addr(C, torch.float16, "C"))
+    return arr
+
+
+def make_sddmm_batch(problems):
+    """problems: [(M, N, K, V, row_ptr, col_idx, A, Bt, out_vals), ...]"""
+    import torch
+    arr = (SddmmProblem * len(problems))()
+    for i, (M, N, K, V, rp, ci, A, Bt, out) in enumerate(problems):
+        arr[i] = SddmmProblem(int(M), int(N), int(K), int(V), 0, _addr(rp, torch.int32, "row_ptr"),
+                              _addr(ci, torch.int32, "col_idx"), _addr(A, torch.float16, "A"),
+                              _addr(Bt, torch.float16, "Bt"), _addr(out, torch.float16, "out_vals"))
+    return arr
+
+
+def make_encode_batch(problems):
+    """problems: [(M, K, V, dense, mask, row_ptr, col_idx, vals), ...]"""
+    import torch
+    arr = (EncodeProblem * len(problems))()
+    for i, (M, K, V, d, m, rp, ci, va) in enumerate(problems):
+        arr[i] = EncodeProblem(int(M), int(K), int(V), 0, _addr(d, torch.float16, "dense"),
+                               _addr(m, torch.uint8, "mask"), _addr(rp, torch.int32, "row_ptr"),
+                               _addr(ci, torch.int32, "col_idx"), _addr(va, torch.float16, "vals"))
+    return arr
+
+
+def vs_spmm_batched(batch, stream=None):
+    if isinstance(batch, list):
+        batch = make_spmm_batch(batch)
+    _check(load().vs_spmm_batched(len(batch), batch, _stream(stream)), "vs_spmm_batched")
+
+
+def vs_sddmm_batched(batch, stream=None):
+    if isinstance(batch, list):
+        batch = make_sddmm_batch(batch)
+    _check(load().vs_sddmm_batched(len(batch), batch, _stream(stream)), "vs_sddmm_batched")
+
+
+def vs_encode_colvec_batched(batch, stream=None):
+    if isinstance(batch, list):
+        batch = make_encode_batch(batch)
+    _check(load().vs_encode_colvec_batched(len(batch), batch, _stream(stream)),
+           "vs_encode_colvec_batched")
 
 
 # ------------------------------------------------------------------ conveniences

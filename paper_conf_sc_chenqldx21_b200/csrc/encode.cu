@@ -12,6 +12,10 @@
 //      counts and writes col_idx and the V values of each kept vector (transposed from the V
 //      row loads into vector-major order) starting at row_ptr[w].
 // Columns are visited in ascending order, so col_idx ascends inside each window (Fig. 8).
+#include <algorithm>
+#include <utility>
+#include <vector>
+
 #include "common.cuh"
 
 namespace vs {
@@ -140,14 +144,14 @@ __device__ void block_scan_inplace(int32_t* a, int64_t n, int32_t* s_warp, int32
 }
 
 template <int V, bool VEC, bool HAS_MASK>
-__global__ void __launch_bounds__(kEncMaxThreads)
-    encode_count_scan_kernel(int64_t M, int64_t K, int64_t W, const uint16_t* __restrict__ dense,
-                             const uint8_t* __restrict__ mask, int32_t* __restrict__ row_ptr) {
+__device__ __forceinline__ void count_scan_body(int64_t M, int64_t K, int64_t W, int64_t w,
+                                                const uint16_t* __restrict__ dense,
+                                                const uint8_t* __restrict__ mask,
+                                                int32_t* __restrict__ row_ptr) {
   __shared__ int32_t s_warp[kEncMaxThreads / 32];
   __shared__ int32_t s_carry;
   __shared__ int s_last;
   const int lane = lane_id(), wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
-  const int64_t w = blockIdx.x;
   uint16_t h[V][8];
   uint32_t count = 0;
   for (int64_t c0 = (int64_t)wid * kColsPerStep; c0 < K; c0 += (int64_t)nw * kColsPerStep) {
@@ -177,13 +181,14 @@ __global__ void __launch_bounds__(kEncMaxThreads)
 // takes chunk (round * nwarps + i); a block-wide exclusive scan of the warps' keep counts
 // gives each warp its slot range, so col_idx stays ascending.
 template <int V, bool VEC, bool HAS_MASK, bool WRITE_VALS, bool VEC_VALS>
-__global__ void __launch_bounds__(kEncMaxThreads)
-    encode_compact_kernel(int64_t M, int64_t K, const uint16_t* __restrict__ dense,
-                          const uint8_t* __restrict__ mask, const int32_t* __restrict__ row_ptr,
-                          int32_t* __restrict__ col_idx, uint16_t* __restrict__ vals) {
+__device__ __forceinline__ void compact_body(int64_t M, int64_t K, int64_t w,
+                                             const uint16_t* __restrict__ dense,
+                                             const uint8_t* __restrict__ mask,
+                                             const int32_t* __restrict__ row_ptr,
+                                             int32_t* __restrict__ col_idx,
+                                             uint16_t* __restrict__ vals) {
   __shared__ uint32_t warp_cnt[kEncMaxThreads / 32];
   const int lane = lane_id(), wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
-  const int64_t w = blockIdx.x;
   int64_t base = row_ptr[w];
   uint16_t h[V][8];
   for (int64_t r0 = 0; r0 < K; r0 += (int64_t)nw * kColsPerStep) {
@@ -232,64 +237,201 @@ __global__ void __launch_bounds__(kEncMaxThreads)
   }
 }
 
-// ---------------------------------------------------------------- host-side launchers
+// --------------------------------------------------------------- kernels and launchers
+//
+// Template flags: V, VEC (16-byte row loads: K % 8 == 0 and aligned rows), HAS_MASK, and for
+// the compact kernel WRITE_VALS and VEC_VALS (vector stores of a whole vector).
+
+template <int V, bool VEC, bool HAS_MASK>
+__global__ void __launch_bounds__(kEncMaxThreads)
+    encode_count_scan_kernel(int64_t M, int64_t K, int64_t W, const uint16_t* __restrict__ dense,
+                             const uint8_t* __restrict__ mask, int32_t* __restrict__ row_ptr) {
+  count_scan_body<V, VEC, HAS_MASK>(M, K, W, blockIdx.x, dense, mask, row_ptr);
+}
+
+template <int V, bool VEC, bool HAS_MASK, bool WRITE_VALS, bool VEC_VALS>
+__global__ void __launch_bounds__(kEncMaxThreads)
+    encode_compact_kernel(int64_t M, int64_t K, const uint16_t* __restrict__ dense,
+                          const uint8_t* __restrict__ mask, const int32_t* __restrict__ row_ptr,
+                          int32_t* __restrict__ col_idx, uint16_t* __restrict__ vals) {
+  compact_body<V, VEC, HAS_MASK, WRITE_VALS, VEC_VALS>(M, K, blockIdx.x, dense, mask, row_ptr,
+                                                       col_idx, vals);
+}
+
+// Batched: one grid over the windows of up to kEncMaxBatch problems of one configuration
+// (descriptors as a __grid_constant__ parameter; a CTA finds its problem by binary search).
+struct EncDesc {
+  int64_t M, K, W;
+  const uint16_t* dense;
+  const uint8_t* mask;
+  int32_t* row_ptr;
+  int32_t* col_idx;
+  uint16_t* vals;
+};
+constexpr int kEncMaxBatch = 128;
+struct EncBatch {
+  int count;
+  int64_t first_block[kEncMaxBatch + 1];
+  EncDesc d[kEncMaxBatch];
+};
+
+__device__ __forceinline__ int find_problem(const EncBatch& b, int64_t bid) {
+  int lo = 0, hi = b.count - 1;
+  while (lo < hi) {
+    const int mid = (lo + hi + 1) >> 1;
+    if (b.first_block[mid] <= bid) lo = mid; else hi = mid - 1;
+  }
+  return lo;
+}
+
+__global__ void ticket_init_kernel(const __grid_constant__ EncBatch b) {
+  for (int p = threadIdx.x; p < b.count; p += blockDim.x) b.d[p].row_ptr[0] = -1;
+}
+
+template <int V, bool VEC, bool HAS_MASK>
+__global__ void __launch_bounds__(kEncMaxThreads)
+    encode_count_scan_batched_kernel(const __grid_constant__ EncBatch b) {
+  const int p = find_problem(b, blockIdx.x);
+  const EncDesc& d = b.d[p];
+  count_scan_body<V, VEC, HAS_MASK>(d.M, d.K, d.W, blockIdx.x - b.first_block[p], d.dense, d.mask,
+                                    d.row_ptr);
+}
+
+template <int V, bool VEC, bool HAS_MASK, bool WRITE_VALS, bool VEC_VALS>
+__global__ void __launch_bounds__(kEncMaxThreads)
+    encode_compact_batched_kernel(const __grid_constant__ EncBatch b) {
+  const int p = find_problem(b, blockIdx.x);
+  const EncDesc& d = b.d[p];
+  compact_body<V, VEC, HAS_MASK, WRITE_VALS, VEC_VALS>(d.M, d.K, blockIdx.x - b.first_block[p],
+                                                       d.dense, d.mask, d.row_ptr, d.col_idx, d.vals);
+}
+
+struct EncCfg {
+  int V;
+  bool VEC, MASK, IDX, VALS, VEC_VALS;
+  int key() const { return (((((V * 2 + VEC) * 2 + MASK) * 2 + IDX) * 2 + VALS) * 2 + VEC_VALS); }
+};
+
+static EncCfg enc_config(int64_t K, int V, const void* dense, const uint8_t* mask,
+                         const int32_t* col_idx, const void* vals) {
+  EncCfg c;
+  c.V = V;
+  // vector path: 16-byte rows (fp16) / 8-byte rows (mask)
+  c.VEC = (K % 8 == 0) && !(dense && (reinterpret_cast<uintptr_t>(dense) & 15)) &&
+          !(mask && (reinterpret_cast<uintptr_t>(mask) & 7));
+  c.MASK = mask != nullptr;
+  c.IDX = col_idx != nullptr;
+  c.VALS = c.IDX && vals != nullptr;
+  c.VEC_VALS = c.VALS && ((reinterpret_cast<uintptr_t>(vals) & (2 * V - 1)) == 0);
+  return c;
+}
+
+static int enc_threads(int64_t K) {  // one warp per 256-column chunk, up to 8 warps
+  const int64_t chunks = ceil_div64(K, kColsPerStep);
+  return (int)(32 * (chunks < 1 ? 1 : (chunks > kEncMaxThreads / 32 ? kEncMaxThreads / 32 : chunks)));
+}
+
+struct EncKernels {
+  void (*count_single)(int64_t, int64_t, int64_t, const uint16_t*, const uint8_t*, int32_t*);
+  void (*compact_single)(int64_t, int64_t, const uint16_t*, const uint8_t*, const int32_t*, int32_t*,
+                         uint16_t*);
+  void (*count_batched)(EncBatch);
+  void (*compact_batched)(EncBatch);
+};
 
 template <int V, bool VEC, bool MASKB>
-static void launch_v(int64_t M, int64_t K, int64_t W, const uint16_t* dense, const uint8_t* mask,
-                     int32_t* row_ptr, int32_t* col_idx, uint16_t* vals, bool vec_vals, dim3 grid,
-                     dim3 block, cudaStream_t s) {
-  encode_count_scan_kernel<V, VEC, MASKB><<<grid, block, 0, s>>>(M, K, W, dense, mask, row_ptr);
-  if (col_idx == nullptr) return;
-  if (vals == nullptr)
-    encode_compact_kernel<V, VEC, MASKB, false, false><<<grid, block, 0, s>>>(M, K, dense, mask, row_ptr, col_idx, vals);
-  else if (vec_vals)
-    encode_compact_kernel<V, VEC, MASKB, true, true><<<grid, block, 0, s>>>(M, K, dense, mask, row_ptr, col_idx, vals);
-  else
-    encode_compact_kernel<V, VEC, MASKB, true, false><<<grid, block, 0, s>>>(M, K, dense, mask, row_ptr, col_idx, vals);
+static EncKernels enc_kernels_vm(const EncCfg& c) {
+  EncKernels k;
+  k.count_single = encode_count_scan_kernel<V, VEC, MASKB>;
+  k.count_batched = encode_count_scan_batched_kernel<V, VEC, MASKB>;
+  if (!c.VALS) {
+    k.compact_single = encode_compact_kernel<V, VEC, MASKB, false, false>;
+    k.compact_batched = encode_compact_batched_kernel<V, VEC, MASKB, false, false>;
+  } else if (c.VEC_VALS) {
+    k.compact_single = encode_compact_kernel<V, VEC, MASKB, true, true>;
+    k.compact_batched = encode_compact_batched_kernel<V, VEC, MASKB, true, true>;
+  } else {
+    k.compact_single = encode_compact_kernel<V, VEC, MASKB, true, false>;
+    k.compact_batched = encode_compact_batched_kernel<V, VEC, MASKB, true, false>;
+  }
+  return k;
 }
 
 template <int V>
-static cudaError_t launch_encode_v(int64_t M, int64_t K, const uint16_t* dense, const uint8_t* mask,
-                                   int32_t* row_ptr, int32_t* col_idx, uint16_t* vals, bool vec,
-                                   bool vec_vals, cudaStream_t s) {
-  const int64_t W = ceil_div64(M, V);
-  if (W == 0) return cudaSuccess;
-  if (W > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
-  // one CTA per window, one warp per 256-column chunk (up to 8 warps)
-  const int64_t chunks = ceil_div64(K, kColsPerStep);
-  const int threads =
-      (int)(32 * (chunks < 1 ? 1 : (chunks > kEncMaxThreads / 32 ? kEncMaxThreads / 32 : chunks)));
-  dim3 grid((unsigned)W), block(threads);
-  // row_ptr[0] = -1: the ticket counter of encode_count_scan (reset to 0 by the last CTA)
-  cudaError_t e = cudaMemsetAsync(row_ptr, 0xFF, sizeof(int32_t), s);
-  if (e != cudaSuccess) return e;
-  const bool has_mask = mask != nullptr;
-  if (vec) {
-    if (has_mask) launch_v<V, true, true>(M, K, W, dense, mask, row_ptr, col_idx, vals, vec_vals, grid, block, s);
-    else launch_v<V, true, false>(M, K, W, dense, mask, row_ptr, col_idx, vals, vec_vals, grid, block, s);
-  } else {
-    if (has_mask) launch_v<V, false, true>(M, K, W, dense, mask, row_ptr, col_idx, vals, vec_vals, grid, block, s);
-    else launch_v<V, false, false>(M, K, W, dense, mask, row_ptr, col_idx, vals, vec_vals, grid, block, s);
+static EncKernels enc_kernels_v(const EncCfg& c) {
+  if (c.VEC) return c.MASK ? enc_kernels_vm<V, true, true>(c) : enc_kernels_vm<V, true, false>(c);
+  return c.MASK ? enc_kernels_vm<V, false, true>(c) : enc_kernels_vm<V, false, false>(c);
+}
+
+static EncKernels enc_kernels(const EncCfg& c) {
+  switch (c.V) {
+    case 1: return enc_kernels_v<1>(c);
+    case 2: return enc_kernels_v<2>(c);
+    case 4: return enc_kernels_v<4>(c);
+    default: return enc_kernels_v<8>(c);
   }
-  return cudaGetLastError();
 }
 
 cudaError_t launch_encode(int64_t M, int64_t K, int V, const void* dense, const uint8_t* mask,
                           int32_t* row_ptr, int32_t* col_idx, void* vals, cudaStream_t s) {
+  const int64_t W = ceil_div64(M, V);
+  if (W == 0) return cudaSuccess;
+  if (W > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
+  const EncCfg c = enc_config(K, V, dense, mask, col_idx, vals);
+  const EncKernels k = enc_kernels(c);
+  const dim3 grid((unsigned)W), block(enc_threads(K));
   const uint16_t* d = static_cast<const uint16_t*>(dense);
-  // vector path: 16-byte rows (fp16) / 8-byte rows (mask)
-  bool vec = (K % 8 == 0);
-  if (d && (reinterpret_cast<uintptr_t>(d) & 15)) vec = false;
-  if (mask && (reinterpret_cast<uintptr_t>(mask) & 7)) vec = false;
-  bool vec_vals = vals && ((reinterpret_cast<uintptr_t>(vals) & (2 * V - 1)) == 0);
-  uint16_t* v = static_cast<uint16_t*>(vals);
-  switch (V) {
-    case 1: return launch_encode_v<1>(M, K, d, mask, row_ptr, col_idx, v, vec, vec_vals, s);
-    case 2: return launch_encode_v<2>(M, K, d, mask, row_ptr, col_idx, v, vec, vec_vals, s);
-    case 4: return launch_encode_v<4>(M, K, d, mask, row_ptr, col_idx, v, vec, vec_vals, s);
-    case 8: return launch_encode_v<8>(M, K, d, mask, row_ptr, col_idx, v, vec, vec_vals, s);
+  // row_ptr[0] = -1: the ticket counter of encode_count_scan (reset to 0 by the last CTA)
+  cudaError_t e = cudaMemsetAsync(row_ptr, 0xFF, sizeof(int32_t), s);
+  if (e != cudaSuccess) return e;
+  k.count_single<<<grid, block, 0, s>>>(M, K, W, d, mask, row_ptr);
+  if (c.IDX)
+    k.compact_single<<<grid, block, 0, s>>>(M, K, d, mask, row_ptr, col_idx,
+                                            static_cast<uint16_t*>(vals));
+  return cudaGetLastError();
+}
+
+// Problems with W == 0 are handled by the caller.
+cudaError_t launch_encode_batched(int64_t count, const int64_t* M, const int64_t* K, const int* V,
+                                  const void* const* dense, const uint8_t* const* mask,
+                                  int32_t* const* row_ptr, int32_t* const* col_idx,
+                                  void* const* vals, cudaStream_t s) {
+  std::vector<std::pair<int, int64_t>> order;
+  for (int64_t i = 0; i < count; ++i)
+    order.push_back({enc_config(K[i], V[i], dense[i], mask[i], col_idx[i], vals[i]).key(), i});
+  std::stable_sort(order.begin(), order.end(),
+                   [](const auto& a, const auto& b) { return a.first < b.first; });
+  EncBatch batch;
+  size_t i = 0;
+  while (i < order.size()) {
+    const int key = order[i].first;
+    const int64_t p0 = order[i].second;
+    const EncCfg c = enc_config(K[p0], V[p0], dense[p0], mask[p0], col_idx[p0], vals[p0]);
+    const EncKernels k = enc_kernels(c);
+    batch.count = 0;
+    int64_t blocks = 0;
+    int threads = 32;
+    while (i < order.size() && order[i].first == key && batch.count < kEncMaxBatch) {
+      const int64_t p = order[i].second;
+      const int64_t W = ceil_div64(M[p], V[p]);
+      if (blocks + W > 0x7fffffffLL) break;
+      batch.d[batch.count] = {M[p], K[p], W, static_cast<const uint16_t*>(dense[p]), mask[p],
+                              row_ptr[p], col_idx[p], static_cast<uint16_t*>(vals[p])};
+      batch.first_block[batch.count++] = blocks;
+      blocks += W;
+      const int th = enc_threads(K[p]);
+      threads = th > threads ? th : threads;
+      ++i;
+    }
+    if (batch.count == 0) return cudaErrorInvalidConfiguration;
+    batch.first_block[batch.count] = blocks;
+    ticket_init_kernel<<<1, 128, 0, s>>>(batch);
+    k.count_batched<<<(unsigned)blocks, threads, 0, s>>>(batch);
+    if (c.IDX) k.compact_batched<<<(unsigned)blocks, threads, 0, s>>>(batch);
+    const cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return e;
   }
-  return cudaErrorInvalidValue;
+  return cudaSuccess;
 }
 
 }  // namespace vs

@@ -17,6 +17,10 @@
 // k0 + 8t + 2j (resp. k0 + 32 + 8t + 2j), the same permutation on both operands.  Every
 // partial sum stays inside one MMA accumulator, so the paper's cross-octet shuffle+FADD
 // reduction (17-30% of instructions) disappears.
+#include <algorithm>
+#include <utility>
+#include <vector>
+
 #include "common.cuh"
 
 namespace vs {
@@ -70,13 +74,98 @@ __device__ __forceinline__ int64_t find_window(const int32_t* __restrict__ row_p
   return lo;
 }
 
+// Stores the two vectors (M rows g, g+8) of a 16-vector slice held in acc, restricted to the
+// vectors [lo, hi) of window w.
+template <int V>
+__device__ __forceinline__ void store_slice(const float (&acc)[4], int64_t v0, int64_t lo,
+                                            int64_t hi, int64_t w, int64_t M, int g, int t,
+                                            uint16_t* __restrict__ out, bool out4) {
+#pragma unroll
+  for (int q = 0; q < 2; ++q) {
+    const int64_t v = v0 + g + 8 * q;
+    if (v < lo || v >= hi) continue;
+    const int r = 2 * t;
+    const float f0 = (w * V + r < M) ? acc[2 * q] : 0.f;
+    const float f1 = (w * V + r + 1 < M) ? acc[2 * q + 1] : 0.f;
+    uint16_t* dst = out + v * V + r;
+    if (V >= 2 && out4) {
+      if (r < V) *reinterpret_cast<uint32_t*>(dst) = f2_to_h2(f0, f1);
+    } else {
+      if (r < V) dst[0] = f_to_h(f0);
+      if (r + 1 < V) dst[1] = f_to_h(f1);
+    }
+  }
+}
+
+// One warp computes the 16-vector slices [s_begin, s_end) of one problem (nnz stored
+// vectors in total); s_begin < s_end.  A slice that straddles windows is finished window by
+// window; the next 64-wide K chunk of the gathered rows is prefetched while the current
+// chunk's MMAs run.  (A variant that processed 2 or 4 slices of one window together to share
+// the A fragment measured no faster, tools/tune.py, and was dropped.)
+template <int V, bool VEC>
+__device__ __forceinline__ void sddmm_range(int64_t M, int64_t K, int64_t W,
+                                            const int32_t* __restrict__ row_ptr,
+                                            const int32_t* __restrict__ col_idx,
+                                            const uint16_t* __restrict__ A,
+                                            const uint16_t* __restrict__ Bt,
+                                            uint16_t* __restrict__ out, bool out4, int64_t s_begin,
+                                            int64_t s_end, int64_t nnz) {
+  const int lane = lane_id();
+  const int g = lane >> 2, t = lane & 3;
+  const int64_t kt = 8 * t;
+  int64_t w = find_window(row_ptr, W, s_begin * 16);
+  int64_t w_end_p = row_ptr[w + 1];
+
+  int64_t s = s_begin;
+  while (s < s_end) {
+    const int64_t v0 = s * 16;
+    while (w_end_p <= v0) {  // advance to the window owning v0
+      ++w;
+      w_end_p = row_ptr[w + 1];
+    }
+    const int64_t v_hi = (v0 + 16 < nnz) ? v0 + 16 : nnz;
+    const bool oka = v0 + g < v_hi, okb = v0 + g + 8 < v_hi;
+    const uint16_t* rowa = Bt + (int64_t)(oka ? ldg32i(col_idx + v0 + g) : 0) * K;
+    const uint16_t* rowb = Bt + (int64_t)(okb ? ldg32i(col_idx + v0 + g + 8) : 0) * K;
+    int64_t v_cur = v0;
+    while (v_cur < v_hi) {
+      while (w_end_p <= v_cur) {
+        ++w;
+        w_end_p = row_ptr[w + 1];
+      }
+      const int64_t seg_hi = w_end_p < v_hi ? w_end_p : v_hi;  // vectors [v_cur, seg_hi) in w
+      const int64_t srow = w * V + g;
+      const bool sok_row = (g < V) && (srow < M);
+      const uint16_t* srowA = A + srow * K;
+      uint4 a0, a1, b0, b1;  // Bt chunk [k0, k0 + 64) of vectors g and g+8
+      load_seg2<VEC>(rowa, K, kt, oka, a0, a1);
+      load_seg2<VEC>(rowb, K, kt, okb, b0, b1);
+      float acc[4] = {0.f, 0.f, 0.f, 0.f};
+      for (int64_t k0 = 0; k0 < K; k0 += 64) {
+        uint4 x0, x1;  // A row g of the window, same K permutation
+        load_seg2<VEC>(srowA, K, k0 + kt, sok_row, x0, x1);
+        const uint4 ca0 = a0, ca1 = a1, cb0 = b0, cb1 = b1;
+        if (k0 + 64 < K) {  // prefetch the next chunk of the gathered rows
+          load_seg2<VEC>(rowa, K, k0 + 64 + kt, oka, a0, a1);
+          load_seg2<VEC>(rowb, K, k0 + 64 + kt, okb, b0, b1);
+        }
+#pragma unroll
+        for (int j = 0; j < 4; ++j)
+          mma_16816(acc, wordj(ca0, j), wordj(cb0, j), wordj(ca1, j), wordj(cb1, j),
+                    wordj(x0, j), wordj(x1, j));
+      }
+      store_slice<V>(acc, v0, v_cur, seg_hi, w, M, g, t, out, out4);
+      v_cur = seg_hi;
+    }
+    s += 1;
+  }
+}
+
 template <int V, bool VEC>
 __global__ void __launch_bounds__(kSddmmWarps * 32)
     sddmm_kernel(int64_t M, int64_t K, int64_t W, const int32_t* __restrict__ row_ptr,
                  const int32_t* __restrict__ col_idx, const uint16_t* __restrict__ A,
                  const uint16_t* __restrict__ Bt, uint16_t* __restrict__ out, bool out4) {
-  const int lane = lane_id();
-  const int g = lane >> 2, t = lane & 3;
   const int64_t nnz = row_ptr[W];
   const int64_t n_slices = ceil_div64(nnz, 16);
   const int64_t n_warps = (int64_t)gridDim.x * kSddmmWarps;
@@ -85,105 +174,108 @@ __global__ void __launch_bounds__(kSddmmWarps * 32)
   const int64_t s_begin = gw * per;
   const int64_t s_end = (s_begin + per < n_slices) ? s_begin + per : n_slices;
   if (s_begin >= s_end) return;
+  sddmm_range<V, VEC>(M, K, W, row_ptr, col_idx, A, Bt, out, out4, s_begin, s_end, nnz);
+}
 
-  const int64_t kt = 8 * t;
-  // Per slice: the two vectors (M rows g and g+8) whose Bt rows this thread loads.  Their
-  // column indices are fetched one slice ahead and the first K chunk of the next slice is
-  // loaded during the current slice's last chunk, so consecutive slices overlap.
-  int64_t v0 = s_begin * 16;
-  int64_t v_hi = (v0 + 16 < nnz) ? v0 + 16 : nnz;
-  bool oka = v0 + g < v_hi, okb = v0 + g + 8 < v_hi;
-  const uint16_t* rowa = Bt + (int64_t)(oka ? ldg32i(col_idx + v0 + g) : 0) * K;
-  const uint16_t* rowb = Bt + (int64_t)(okb ? ldg32i(col_idx + v0 + g + 8) : 0) * K;
-  uint4 a0, a1, b0, b1;  // Bt chunk [k0, k0 + 64) of vectors g and g+8
-  load_seg2<VEC>(rowa, K, kt, oka, a0, a1);
-  load_seg2<VEC>(rowb, K, kt, okb, b0, b1);
-  // the window search runs while the first gathered rows are in flight
-  int64_t w = find_window(row_ptr, W, v0);
-  int64_t w_end_p = row_ptr[w + 1];
+// Batched launch over up to kSddmmMaxBatch problems of one configuration.  The work of a
+// problem is its slice count times its number of 64-wide K chunks (slice counts from each
+// problem's row_ptr[W], read on the device and prefix-summed per CTA in shared memory); the
+// total work is split evenly over the persistent warps, a warp's share of a problem being
+// the slices whose work offsets fall in the warp's range, so problems with different K are
+// balanced and every slice is computed exactly once.  A warp's run may cross into the next
+// problem.
+struct SddmmDesc {
+  int64_t M, K, W;
+  const int32_t* row_ptr;
+  const int32_t* col_idx;
+  const uint16_t* A;
+  const uint16_t* Bt;
+  uint16_t* out;
+  int64_t out4;
+};
+constexpr int kSddmmMaxBatch = 128;
+struct SddmmBatch {
+  int count;
+  SddmmDesc d[kSddmmMaxBatch];
+};
 
-  for (int64_t s = s_begin; s < s_end; ++s) {
-    // next slice's column indices
-    const bool has_next = s + 1 < s_end;
-    const int64_t nv0 = v0 + 16;
-    const int64_t nv_hi = (nv0 + 16 < nnz) ? nv0 + 16 : nnz;
-    const bool noka = has_next && nv0 + g < nv_hi, nokb = has_next && nv0 + g + 8 < nv_hi;
-    const int nca = noka ? ldg32i(col_idx + nv0 + g) : 0;
-    const int ncb = nokb ? ldg32i(col_idx + nv0 + g + 8) : 0;
-
-    int64_t v_cur = v0;
-    bool first_seg = true;
-    while (v_cur < v_hi) {
-      while (w_end_p <= v_cur) {  // advance to the window owning v_cur
-        ++w;
-        w_end_p = row_ptr[w + 1];
-      }
-      const int64_t seg_hi = w_end_p < v_hi ? w_end_p : v_hi;  // vectors [v_cur, seg_hi) in w
-      const bool last_seg = seg_hi == v_hi;
-      const int64_t arow = w * V + g;
-      const bool oka_row = (g < V) && (arow < M);
-      const uint16_t* rowA = A + arow * K;
-      if (!first_seg) {  // the slice straddles windows: restart the Bt stream
-        load_seg2<VEC>(rowa, K, kt, oka, a0, a1);
-        load_seg2<VEC>(rowb, K, kt, okb, b0, b1);
-      }
-      first_seg = false;
-
-      float acc[4] = {0.f, 0.f, 0.f, 0.f};
-      for (int64_t k0 = 0; k0 < K; k0 += 64) {
-        uint4 x0, x1;  // A row g of the window, same K permutation
-        load_seg2<VEC>(rowA, K, k0 + kt, oka_row, x0, x1);
-        const uint4 ca0 = a0, ca1 = a1, cb0 = b0, cb1 = b1;
-        if (k0 + 64 < K) {  // prefetch the next chunk of the gathered rows
-          load_seg2<VEC>(rowa, K, k0 + 64 + kt, oka, a0, a1);
-          load_seg2<VEC>(rowb, K, k0 + 64 + kt, okb, b0, b1);
-        } else if (last_seg && has_next) {  // or the first chunk of the next slice
-          load_seg2<VEC>(Bt + (int64_t)nca * K, K, kt, noka, a0, a1);
-          load_seg2<VEC>(Bt + (int64_t)ncb * K, K, kt, nokb, b0, b1);
-        }
+template <int V, bool VEC>
+__global__ void __launch_bounds__(kSddmmWarps * 32)
+    sddmm_batched_kernel(const __grid_constant__ SddmmBatch b) {
+  __shared__ int64_t pre[kSddmmMaxBatch + 1];  // work prefix (slices * chunks)
+  __shared__ int64_t nnzs[kSddmmMaxBatch];
+  __shared__ int32_t nks[kSddmmMaxBatch];      // 64-wide K chunks per slice (>= 1)
+  const int lane = lane_id();
+  if (threadIdx.x < 32) {
+    int64_t carry = 0;
+    for (int base = 0; base < b.count; base += 32) {
+      const int p = base + lane;
+      const int64_t nz = p < b.count ? (int64_t)b.d[p].row_ptr[b.d[p].W] : 0;
+      const int64_t nk = p < b.count ? (b.d[p].K > 64 ? ceil_div64(b.d[p].K, 64) : 1) : 1;
+      const int64_t v = ceil_div64(nz, 16) * nk;
+      int64_t incl = v;
 #pragma unroll
-        for (int j = 0; j < 4; ++j)
-          mma_16816(acc, wordj(ca0, j), wordj(cb0, j), wordj(ca1, j), wordj(cb1, j),
-                    wordj(x0, j), wordj(x1, j));
+      for (int o = 1; o < 32; o <<= 1) {
+        const int64_t x = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += x;
       }
-      // acc[0..1]: vector v0+g, rows 2t, 2t+1; acc[2..3]: vector v0+g+8, rows 2t, 2t+1.
-#pragma unroll
-      for (int q = 0; q < 2; ++q) {
-        const int64_t v = v0 + g + 8 * q;
-        if (v < v_cur || v >= seg_hi) continue;
-        const int r = 2 * t;
-        const float f0 = (w * V + r < M) ? acc[2 * q] : 0.f;
-        const float f1 = (w * V + r + 1 < M) ? acc[2 * q + 1] : 0.f;
-        uint16_t* dst = out + v * V + r;
-        if (V >= 2 && out4) {
-          if (r < V) *reinterpret_cast<uint32_t*>(dst) = f2_to_h2(f0, f1);
-        } else {
-          if (r < V) dst[0] = f_to_h(f0);
-          if (r + 1 < V) dst[1] = f_to_h(f1);
-        }
+      if (p < b.count) {
+        pre[p] = carry + incl - v;
+        nnzs[p] = nz;
+        nks[p] = (int32_t)nk;
       }
-      v_cur = seg_hi;
+      carry += __shfl_sync(0xffffffffu, incl, 31);
     }
-    v0 = nv0;
-    v_hi = nv_hi;
-    oka = noka;
-    okb = nokb;
-    rowa = Bt + (int64_t)nca * K;
-    rowb = Bt + (int64_t)ncb * K;
+    if (lane == 0) pre[b.count] = carry;
+  }
+  __syncthreads();
+  const int64_t total = pre[b.count];
+  const int64_t n_warps = (int64_t)gridDim.x * kSddmmWarps;
+  const int64_t gw = (int64_t)blockIdx.x * kSddmmWarps + (threadIdx.x >> 5);
+  const int64_t per = ceil_div64(total, n_warps);
+  const int64_t wb = gw * per;
+  const int64_t we = (wb + per < total) ? wb + per : total;
+  if (wb >= we) return;
+  int p = 0;
+  {
+    int lo = 0, hi = b.count - 1;  // last problem with pre[p] <= wb
+    while (lo < hi) {
+      const int mid = (lo + hi + 1) >> 1;
+      if (pre[mid] <= wb) lo = mid; else hi = mid - 1;
+    }
+    p = lo;
+  }
+  for (; p < b.count && pre[p] < we; ++p) {
+    // this warp's slices of problem p: those whose work offset s*nk lies in [wb, we)
+    const int64_t nk = nks[p];
+    const int64_t lo = wb > pre[p] ? wb - pre[p] : 0;
+    const int64_t hi = (we < pre[p + 1] ? we : pre[p + 1]) - pre[p];
+    const int64_t s0 = ceil_div64(lo, nk), s1 = ceil_div64(hi, nk);
+    if (s0 >= s1) continue;
+    const SddmmDesc& d = b.d[p];
+    sddmm_range<V, VEC>(d.M, d.K, d.W, d.row_ptr, d.col_idx, d.A, d.Bt, d.out, d.out4 != 0, s0, s1,
+                        nnzs[p]);
   }
 }
 
 // Persistent grid: as many CTAs as can be resident at once (occupancy queried once per
 // kernel instantiation), so every warp's contiguous share of slices runs concurrently.
+template <typename Kern>
+static int ctas_per_sm(Kern k) {
+  int b = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k, kSddmmWarps * 32, 0) != cudaSuccess || b < 1)
+    b = 1;
+  return b;
+}
+
 template <int V, bool VEC>
 static int sddmm_ctas_per_sm() {
-  static const int n = [] {
-    int b = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, sddmm_kernel<V, VEC>, kSddmmWarps * 32, 0) !=
-            cudaSuccess || b < 1)
-      b = 1;
-    return b;
-  }();
+  static const int n = ctas_per_sm(sddmm_kernel<V, VEC>);
+  return n;
+}
+template <int V, bool VEC>
+static int sddmm_batched_ctas_per_sm() {
+  static const int n = ctas_per_sm(sddmm_batched_kernel<V, VEC>);
   return n;
 }
 
@@ -203,6 +295,51 @@ static cudaError_t launch_sddmm_v(int64_t M, int64_t N, int64_t K, const int32_t
     sddmm_kernel<V, false><<<grid, block, 0, s>>>(M, K, W, row_ptr, col_idx, A, Bt, out, out4);
   }
   return cudaGetLastError();
+}
+
+template <int V, bool VEC>
+static void launch_sddmm_batch(const SddmmBatch& b, int num_sms, cudaStream_t s) {
+  dim3 grid((unsigned)(num_sms * sddmm_batched_ctas_per_sm<V, VEC>()));
+  sddmm_batched_kernel<V, VEC><<<grid, kSddmmWarps * 32, 0, s>>>(b);
+}
+
+cudaError_t launch_sddmm_batched(int64_t count, const int64_t* M, const int64_t* K, const int* V,
+                                 const int32_t* const* row_ptr, const int32_t* const* col_idx,
+                                 const void* const* A, const void* const* Bt, void* const* out,
+                                 int num_sms, cudaStream_t s) {
+  // group by (V, vector path); keep the caller's order inside a group
+  std::vector<std::pair<int, int64_t>> order;
+  for (int64_t i = 0; i < count; ++i) {
+    const bool vec = (K[i] % 8 == 0) && ((reinterpret_cast<uintptr_t>(A[i]) & 15) == 0) &&
+                     ((reinterpret_cast<uintptr_t>(Bt[i]) & 15) == 0);
+    order.push_back({V[i] * 2 + (vec ? 1 : 0), i});
+  }
+  std::stable_sort(order.begin(), order.end(),
+                   [](const auto& a, const auto& b) { return a.first < b.first; });
+  SddmmBatch batch;
+  size_t i = 0;
+  while (i < order.size()) {
+    const int key = order[i].first;
+    batch.count = 0;
+    while (i < order.size() && order[i].first == key && batch.count < kSddmmMaxBatch) {
+      const int64_t p = order[i].second;
+      SddmmDesc& d = batch.d[batch.count++];
+      d = {M[p], K[p], ceil_div64(M[p], V[p]), row_ptr[p], col_idx[p],
+           static_cast<const uint16_t*>(A[p]), static_cast<const uint16_t*>(Bt[p]),
+           static_cast<uint16_t*>(out[p]), (reinterpret_cast<uintptr_t>(out[p]) & 3) == 0 ? 1 : 0};
+      ++i;
+    }
+    const bool vec = key & 1;
+    switch (key >> 1) {
+      case 1: vec ? launch_sddmm_batch<1, true>(batch, num_sms, s) : launch_sddmm_batch<1, false>(batch, num_sms, s); break;
+      case 2: vec ? launch_sddmm_batch<2, true>(batch, num_sms, s) : launch_sddmm_batch<2, false>(batch, num_sms, s); break;
+      case 4: vec ? launch_sddmm_batch<4, true>(batch, num_sms, s) : launch_sddmm_batch<4, false>(batch, num_sms, s); break;
+      default: vec ? launch_sddmm_batch<8, true>(batch, num_sms, s) : launch_sddmm_batch<8, false>(batch, num_sms, s); break;
+    }
+    const cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
 }
 
 cudaError_t launch_sddmm(int64_t M, int64_t N, int64_t K, int V, const int32_t* row_ptr,

@@ -18,7 +18,9 @@
 //   words and the accumulators of a thread cover 8 consecutive columns of output rows
 //   2t and 2t+1: the epilogue stores 16 bytes per row with no shuffles.
 //   B fragment (k = vector slot, n = row r < V) is vals[p*V + g].
-#include <cstdlib>
+#include <algorithm>
+#include <utility>
+#include <vector>
 
 #include "common.cuh"
 
@@ -59,11 +61,11 @@ struct SpmmCta {
 };
 
 template <int V, int NC, bool VEC, int SPLIT, int UNROLL>
-__global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32)
-    spmm_kernel(int64_t M, int64_t N, int64_t W, int64_t n_wgroups,
-                const int32_t* __restrict__ row_ptr, const int32_t* __restrict__ col_idx,
-                const uint16_t* __restrict__ vals, const uint16_t* __restrict__ B,
-                uint16_t* __restrict__ C) {
+__device__ __forceinline__ void spmm_body(int64_t M, int64_t N, int64_t W, int64_t n_wgroups,
+                                          int64_t bid, const int32_t* __restrict__ row_ptr,
+                                          const int32_t* __restrict__ col_idx,
+                                          const uint16_t* __restrict__ vals,
+                                          const uint16_t* __restrict__ B, uint16_t* __restrict__ C) {
   constexpr int UPC = SpmmCta<SPLIT>::kUnits;  // units per CTA
   constexpr int NACC = NC * 16;                // accumulator floats per thread
   constexpr int HALF = SPLIT > 1 ? SPLIT / 2 : 1;
@@ -73,7 +75,6 @@ __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32)
   const int wid = threadIdx.x >> 5;
   const int part = wid % SPLIT;
   // panel-major CTA order: consecutive CTAs share a B panel (L1/L2 locality)
-  const int64_t bid = blockIdx.x;
   const int64_t pn = bid / n_wgroups;
   const int64_t w = (bid - pn * n_wgroups) * UPC + wid / SPLIT;
   const bool active = w < W;
@@ -198,98 +199,177 @@ __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32)
   }
 }
 
+// ------------------------------------------------------------------ kernels + launch
+
 template <int V, int NC, bool VEC, int SPLIT, int UNROLL>
-static void launch_cfg(int64_t M, int64_t N, int64_t W, const int32_t* row_ptr,
-                       const int32_t* col_idx, const uint16_t* vals, const uint16_t* B,
-                       uint16_t* C, cudaStream_t s) {
-  constexpr int UPC = SpmmCta<SPLIT>::kUnits;
-  const int64_t n_panels = ceil_div64(N, 64 * NC);
-  const int64_t n_wgroups = ceil_div64(W, UPC);
-  const int64_t grid = n_panels * n_wgroups;
-  spmm_kernel<V, NC, VEC, SPLIT, UNROLL><<<(unsigned)grid, SpmmCta<SPLIT>::kWarps * 32, 0, s>>>(
-      M, N, W, n_wgroups, row_ptr, col_idx, vals, B, C);
+__global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32)
+    spmm_kernel(int64_t M, int64_t N, int64_t W, int64_t n_wgroups,
+                const int32_t* __restrict__ row_ptr, const int32_t* __restrict__ col_idx,
+                const uint16_t* __restrict__ vals, const uint16_t* __restrict__ B,
+                uint16_t* __restrict__ C) {
+  spmm_body<V, NC, VEC, SPLIT, UNROLL>(M, N, W, n_wgroups, blockIdx.x, row_ptr, col_idx, vals, B, C);
 }
 
-// Tuning knobs (read once from the environment; for experiments only -- the defaults are
-// the shipped configuration): VS_SPMM_UNROLL in {1,2}, VS_SPMM_NC in {0 (auto),1,2},
-// VS_SPMM_SPLIT_SHIFT (SPLIT = K >> shift, clamped to [1,16] and rounded down to a power of 2).
-struct SpmmTune {
-  int unroll = 1, nc = 0, split_shift = 8;
+// Batched launch: one grid over the units of up to kSpmmMaxBatch problems that share a
+// kernel configuration; the descriptors travel as a __grid_constant__ kernel parameter and a
+// CTA finds its problem by binary search of the per-problem first-block table.
+struct SpmmDesc {
+  int64_t M, N, W, n_wgroups;
+  const int32_t* row_ptr;
+  const int32_t* col_idx;
+  const uint16_t* vals;
+  const uint16_t* B;
+  uint16_t* C;
 };
-static const SpmmTune& spmm_tune() {
-  static const SpmmTune t = [] {
-    SpmmTune r;
-    if (const char* e = std::getenv("VS_SPMM_UNROLL")) r.unroll = std::atoi(e) == 1 ? 1 : 2;
-    if (const char* e = std::getenv("VS_SPMM_NC")) r.nc = std::atoi(e);
-    if (const char* e = std::getenv("VS_SPMM_SPLIT_SHIFT")) r.split_shift = std::atoi(e);
-    return r;
-  }();
-  return t;
+constexpr int kSpmmMaxBatch = 128;
+struct SpmmBatch {
+  int count;
+  int64_t first_block[kSpmmMaxBatch + 1];
+  SpmmDesc d[kSpmmMaxBatch];
+};
+
+template <int V, int NC, bool VEC, int SPLIT, int UNROLL>
+__global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32)
+    spmm_batched_kernel(const __grid_constant__ SpmmBatch b) {
+  const int64_t bid = blockIdx.x;
+  int lo = 0, hi = b.count - 1;
+  while (lo < hi) {
+    const int mid = (lo + hi + 1) >> 1;
+    if (b.first_block[mid] <= bid) lo = mid; else hi = mid - 1;
+  }
+  const SpmmDesc& d = b.d[lo];
+  spmm_body<V, NC, VEC, SPLIT, UNROLL>(d.M, d.N, d.W, d.n_wgroups, bid - b.first_block[lo],
+                                       d.row_ptr, d.col_idx, d.vals, d.B, d.C);
 }
 
-template <int V, int NC, bool VEC, int UNROLL>
-static void launch_split(int64_t M, int64_t K, int64_t N, int64_t W, const int32_t* row_ptr,
-                         const int32_t* col_idx, const uint16_t* vals, const uint16_t* B,
-                         uint16_t* C, cudaStream_t s) {
-  // Warps per (window, panel) unit, from K (the bound on a window's vector count): about
-  // one warp per 2^shift possible vectors, up to 16.  It must not depend on N, so that N-panel
-  // shards accumulate in exactly the order of the full problem.
-  const int64_t q = K >> spmm_tune().split_shift;
-  if (q >= 16)
-    launch_cfg<V, NC, VEC, 16, UNROLL>(M, N, W, row_ptr, col_idx, vals, B, C, s);
-  else if (q >= 8)
-    launch_cfg<V, NC, VEC, 8, UNROLL>(M, N, W, row_ptr, col_idx, vals, B, C, s);
-  else if (q >= 4)
-    launch_cfg<V, NC, VEC, 4, UNROLL>(M, N, W, row_ptr, col_idx, vals, B, C, s);
-  else if (q >= 2)
-    launch_cfg<V, NC, VEC, 2, UNROLL>(M, N, W, row_ptr, col_idx, vals, B, C, s);
-  else
-    launch_cfg<V, NC, VEC, 1, UNROLL>(M, N, W, row_ptr, col_idx, vals, B, C, s);
+// Kernel configuration of one problem.  NC (64- or 128-column panels) follows N; SPLIT
+// (warps per unit, about one per 256 possible vectors of a window, up to 16) follows K only,
+// so N-panel shards of a problem run with exactly the same per-element accumulation order
+// as the full problem.  UNROLL = 1 (one 16-vector group in flight per warp and iteration,
+// metadata one group ahead) won the sweep of profiles/ (tools/tune.py).
+struct SpmmCfg {
+  int V, NC, SPLIT;
+  bool VEC;
+  bool operator<(const SpmmCfg& o) const {
+    return V != o.V ? V < o.V : NC != o.NC ? NC < o.NC : SPLIT != o.SPLIT ? SPLIT < o.SPLIT : VEC < o.VEC;
+  }
+};
+
+SpmmCfg spmm_config(int64_t K, int64_t N, int V, const void* B, const void* C) {
+  SpmmCfg c;
+  c.V = V;
+  c.NC = N <= 64 ? 1 : 2;
+  const int64_t q = K >> 8;
+  c.SPLIT = q >= 16 ? 16 : q >= 8 ? 8 : q >= 4 ? 4 : q >= 2 ? 2 : 1;
+  c.VEC = (N % 8 == 0) && ((reinterpret_cast<uintptr_t>(B) & 15) == 0) &&
+          ((reinterpret_cast<uintptr_t>(C) & 15) == 0);
+  return c;
+}
+
+struct SpmmKernels {
+  void (*single)(int64_t, int64_t, int64_t, int64_t, const int32_t*, const int32_t*,
+                 const uint16_t*, const uint16_t*, uint16_t*);
+  void (*batched)(SpmmBatch);
+  int threads, units_per_cta;
+};
+
+template <int V, int NC, bool VEC, int SPLIT>
+static SpmmKernels kernels_of() {
+  return {spmm_kernel<V, NC, VEC, SPLIT, 1>, spmm_batched_kernel<V, NC, VEC, SPLIT, 1>,
+          SpmmCta<SPLIT>::kWarps * 32, SpmmCta<SPLIT>::kUnits};
 }
 
 template <int V, int NC, bool VEC>
-static void launch_unroll(int64_t M, int64_t K, int64_t N, int64_t W, const int32_t* row_ptr,
-                          const int32_t* col_idx, const uint16_t* vals, const uint16_t* B,
-                          uint16_t* C, cudaStream_t s) {
-  if (spmm_tune().unroll == 1)
-    launch_split<V, NC, VEC, 1>(M, K, N, W, row_ptr, col_idx, vals, B, C, s);
-  else
-    launch_split<V, NC, VEC, 2>(M, K, N, W, row_ptr, col_idx, vals, B, C, s);
+static SpmmKernels pick_split(int split) {
+  switch (split) {
+    case 16: return kernels_of<V, NC, VEC, 16>();
+    case 8: return kernels_of<V, NC, VEC, 8>();
+    case 4: return kernels_of<V, NC, VEC, 4>();
+    case 2: return kernels_of<V, NC, VEC, 2>();
+    default: return kernels_of<V, NC, VEC, 1>();
+  }
 }
 
 template <int V>
-static cudaError_t launch_spmm_v(int64_t M, int64_t K, int64_t N, const int32_t* row_ptr,
-                                 const int32_t* col_idx, const uint16_t* vals, const uint16_t* B,
-                                 uint16_t* C, bool vec, int num_sms, cudaStream_t s) {
-  const int64_t W = ceil_div64(M, V);
-  (void)num_sms;
-  const int NC = spmm_tune().nc == 0 ? ((N <= 64) ? 1 : 2) : (spmm_tune().nc == 2 && N > 64 ? 2 : 1);
-  if (ceil_div64(N, 64 * NC) * W > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
-  if (NC == 1) {
-    if (vec) launch_unroll<V, 1, true>(M, K, N, W, row_ptr, col_idx, vals, B, C, s);
-    else launch_unroll<V, 1, false>(M, K, N, W, row_ptr, col_idx, vals, B, C, s);
-  } else {
-    if (vec) launch_unroll<V, 2, true>(M, K, N, W, row_ptr, col_idx, vals, B, C, s);
-    else launch_unroll<V, 2, false>(M, K, N, W, row_ptr, col_idx, vals, B, C, s);
+static SpmmKernels pick_v(const SpmmCfg& c) {
+  if (c.NC == 1) return c.VEC ? pick_split<V, 1, true>(c.SPLIT) : pick_split<V, 1, false>(c.SPLIT);
+  return c.VEC ? pick_split<V, 2, true>(c.SPLIT) : pick_split<V, 2, false>(c.SPLIT);
+}
+
+static SpmmKernels pick(const SpmmCfg& c) {
+  switch (c.V) {
+    case 1: return pick_v<1>(c);
+    case 2: return pick_v<2>(c);
+    case 4: return pick_v<4>(c);
+    default: return pick_v<8>(c);
   }
-  return cudaGetLastError();
+}
+
+static int64_t spmm_blocks(const SpmmKernels& k, const SpmmCfg& c, int64_t M, int64_t N, int V,
+                           int64_t* W_out, int64_t* nwg_out) {
+  const int64_t W = ceil_div64(M, V);
+  const int64_t nwg = ceil_div64(W, k.units_per_cta);
+  *W_out = W;
+  *nwg_out = nwg;
+  return ceil_div64(N, 64 * c.NC) * nwg;
 }
 
 cudaError_t launch_spmm(int64_t M, int64_t K, int64_t N, int V, const int32_t* row_ptr,
                         const int32_t* col_idx, const void* vals, const void* B, void* C,
                         int num_sms, cudaStream_t s) {
-  const uint16_t* v = static_cast<const uint16_t*>(vals);
-  const uint16_t* b = static_cast<const uint16_t*>(B);
-  uint16_t* c = static_cast<uint16_t*>(C);
-  const bool vec = (N % 8 == 0) && ((reinterpret_cast<uintptr_t>(B) & 15) == 0) &&
-                   ((reinterpret_cast<uintptr_t>(C) & 15) == 0);
-  switch (V) {
-    case 1: return launch_spmm_v<1>(M, K, N, row_ptr, col_idx, v, b, c, vec, num_sms, s);
-    case 2: return launch_spmm_v<2>(M, K, N, row_ptr, col_idx, v, b, c, vec, num_sms, s);
-    case 4: return launch_spmm_v<4>(M, K, N, row_ptr, col_idx, v, b, c, vec, num_sms, s);
-    case 8: return launch_spmm_v<8>(M, K, N, row_ptr, col_idx, v, b, c, vec, num_sms, s);
+  (void)num_sms;
+  const SpmmCfg c = spmm_config(K, N, V, B, C);
+  const SpmmKernels k = pick(c);
+  int64_t W, nwg;
+  const int64_t grid = spmm_blocks(k, c, M, N, V, &W, &nwg);
+  if (grid > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
+  k.single<<<(unsigned)grid, k.threads, 0, s>>>(M, N, W, nwg, row_ptr, col_idx,
+                                                static_cast<const uint16_t*>(vals),
+                                                static_cast<const uint16_t*>(B),
+                                                static_cast<uint16_t*>(C));
+  return cudaGetLastError();
+}
+
+// problems with K == 0 are handled by the caller (zero fill); M == 0 or N == 0 skipped.
+cudaError_t launch_spmm_batched(int64_t count, const int64_t* M, const int64_t* K, const int64_t* N,
+                                const int* V, const int32_t* const* row_ptr,
+                                const int32_t* const* col_idx, const void* const* vals,
+                                const void* const* B, void* const* C, cudaStream_t s) {
+  // group problem indices by configuration (stable: keeps the caller's order inside a group)
+  std::vector<std::pair<SpmmCfg, int64_t>> order;
+  order.reserve(count);
+  for (int64_t i = 0; i < count; ++i)
+    order.push_back({spmm_config(K[i], N[i], V[i], B[i], C[i]), i});
+  std::stable_sort(order.begin(), order.end(),
+                   [](const auto& a, const auto& b) { return a.first < b.first; });
+  SpmmBatch batch;
+  size_t i = 0;
+  while (i < order.size()) {
+    const SpmmCfg c = order[i].first;
+    const SpmmKernels k = pick(c);
+    batch.count = 0;
+    int64_t blocks = 0;
+    while (i < order.size() && !(c < order[i].first) && !(order[i].first < c) &&
+           batch.count < kSpmmMaxBatch) {
+      const int64_t p = order[i].second;
+      int64_t W, nwg;
+      const int64_t nb = spmm_blocks(k, c, M[p], N[p], V[p], &W, &nwg);
+      if (blocks + nb > 0x7fffffffLL) break;
+      SpmmDesc& d = batch.d[batch.count];
+      d = {M[p], N[p], W, nwg, row_ptr[p], col_idx[p], static_cast<const uint16_t*>(vals[p]),
+           static_cast<const uint16_t*>(B[p]), static_cast<uint16_t*>(C[p])};
+      batch.first_block[batch.count] = blocks;
+      blocks += nb;
+      ++batch.count;
+      ++i;
+    }
+    if (batch.count == 0) return cudaErrorInvalidConfiguration;
+    batch.first_block[batch.count] = blocks;
+    if (blocks > 0) k.batched<<<(unsigned)blocks, k.threads, 0, s>>>(batch);
+    const cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return e;
   }
-  return cudaErrorInvalidValue;
+  return cudaSuccess;
 }
 
 }  // namespace vs

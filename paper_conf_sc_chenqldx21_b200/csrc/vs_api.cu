@@ -1,6 +1,7 @@
 // vs_api.cu — the C ABI of include/vs.h: argument checks, dispatch, launch status.
 // No exception crosses this boundary; every entry point returns a vs_status_t.
 #include <mutex>
+#include <vector>
 
 #include "../../include/vs.h"
 #include "common.cuh"
@@ -14,6 +15,18 @@ cudaError_t launch_spmm(int64_t M, int64_t K, int64_t N, int V, const int32_t* r
 cudaError_t launch_sddmm(int64_t M, int64_t N, int64_t K, int V, const int32_t* row_ptr,
                          const int32_t* col_idx, const void* A, const void* Bt, void* out,
                          int num_sms, cudaStream_t s);
+cudaError_t launch_spmm_batched(int64_t count, const int64_t* M, const int64_t* K, const int64_t* N,
+                                const int* V, const int32_t* const* row_ptr,
+                                const int32_t* const* col_idx, const void* const* vals,
+                                const void* const* B, void* const* C, cudaStream_t s);
+cudaError_t launch_sddmm_batched(int64_t count, const int64_t* M, const int64_t* K, const int* V,
+                                 const int32_t* const* row_ptr, const int32_t* const* col_idx,
+                                 const void* const* A, const void* const* Bt, void* const* out,
+                                 int num_sms, cudaStream_t s);
+cudaError_t launch_encode_batched(int64_t count, const int64_t* M, const int64_t* K, const int* V,
+                                  const void* const* dense, const uint8_t* const* mask,
+                                  int32_t* const* row_ptr, int32_t* const* col_idx,
+                                  void* const* vals, cudaStream_t s);
 }  // namespace vs
 
 namespace {
@@ -52,6 +65,41 @@ vs_status_t check_device(DevInfo* info) {
   return info->ok ? VS_SUCCESS : VS_ERROR_NOT_SUPPORTED;
 }
 
+// Host-side argument checks shared by the single and batched entry points.
+vs_status_t check_encode(int64_t M, int64_t K, int V, const void* dense, const uint8_t* mask,
+                         int32_t* row_ptr, int32_t* col_idx, void* vals) {
+  if (!valid_v(V) || M < 0 || K < 0) return VS_ERROR_INVALID_VALUE;
+  // dense / mask may be NULL only for an empty matrix (M * K == 0)
+  if (M * K > 0 && dense == nullptr && mask == nullptr) return VS_ERROR_INVALID_VALUE;
+  if (row_ptr == nullptr) return VS_ERROR_INVALID_VALUE;
+  if (M * K > 0 && vals != nullptr && dense == nullptr) return VS_ERROR_INVALID_VALUE;
+  if (!al(row_ptr, 4) || (col_idx && !al(col_idx, 4))) return VS_ERROR_MISALIGNED;
+  if ((dense && !al(dense, 2)) || (vals && !al(vals, 2))) return VS_ERROR_MISALIGNED;
+  return VS_SUCCESS;
+}
+
+vs_status_t check_spmm(int64_t M, int64_t K, int64_t N, int V, const int32_t* row_ptr,
+                       const int32_t* col_idx, const void* vals, const void* B, const void* C) {
+  if (!valid_v(V) || M < 0 || K < 0 || N < 0) return VS_ERROR_INVALID_VALUE;
+  if (M == 0 || N == 0) return VS_SUCCESS;
+  // col_idx / vals / B may be NULL only when they are never read (nnz_v == 0 or K == 0)
+  if (row_ptr == nullptr || C == nullptr) return VS_ERROR_INVALID_VALUE;
+  if (!al(row_ptr, 4) || (col_idx && !al(col_idx, 4))) return VS_ERROR_MISALIGNED;
+  if ((vals && !al(vals, 2)) || (B && !al(B, 2)) || !al(C, 2)) return VS_ERROR_MISALIGNED;
+  return VS_SUCCESS;
+}
+
+vs_status_t check_sddmm(int64_t M, int64_t N, int64_t K, int V, const int32_t* row_ptr,
+                        const int32_t* col_idx, const void* A, const void* Bt, const void* out) {
+  if (!valid_v(V) || M < 0 || K < 0 || N < 0) return VS_ERROR_INVALID_VALUE;
+  if (M == 0 || N == 0) return VS_SUCCESS;
+  // col_idx / A / Bt / out_vals may be NULL only when never touched (nnz_v == 0)
+  if (row_ptr == nullptr) return VS_ERROR_INVALID_VALUE;
+  if (!al(row_ptr, 4) || (col_idx && !al(col_idx, 4))) return VS_ERROR_MISALIGNED;
+  if ((A && !al(A, 2)) || (Bt && !al(Bt, 2)) || (out && !al(out, 2))) return VS_ERROR_MISALIGNED;
+  return VS_SUCCESS;
+}
+
 }  // namespace
 
 extern "C" {
@@ -72,12 +120,8 @@ int vs_version(void) { return 100; /* 0.1.0 */ }
 vs_status_t vs_encode_colvec(int64_t M, int64_t K, int V, const void* dense, const uint8_t* mask,
                              int32_t* row_ptr, int32_t* col_idx, void* vals,
                              int64_t* nnz_vec_host, vs_stream_t stream) {
-  if (!valid_v(V) || M < 0 || K < 0) return VS_ERROR_INVALID_VALUE;
-  if (dense == nullptr && mask == nullptr) return VS_ERROR_INVALID_VALUE;
-  if (row_ptr == nullptr) return VS_ERROR_INVALID_VALUE;
-  if (vals != nullptr && dense == nullptr) return VS_ERROR_INVALID_VALUE;
-  if (!al(row_ptr, 4) || (col_idx && !al(col_idx, 4))) return VS_ERROR_MISALIGNED;
-  if ((dense && !al(dense, 2)) || (vals && !al(vals, 2))) return VS_ERROR_MISALIGNED;
+  vs_status_t st0 = check_encode(M, K, V, dense, mask, row_ptr, col_idx, vals);
+  if (st0 != VS_SUCCESS) return st0;
   DevInfo info;
   vs_status_t st = check_device(&info);
   if (st != VS_SUCCESS) return st;
@@ -104,12 +148,8 @@ vs_status_t vs_encode_colvec(int64_t M, int64_t K, int V, const void* dense, con
 vs_status_t vs_spmm(int64_t M, int64_t K, int64_t N, int V, const int32_t* row_ptr,
                     const int32_t* col_idx, const void* vals, const void* B, void* C,
                     vs_stream_t stream) {
-  if (!valid_v(V) || M < 0 || K < 0 || N < 0) return VS_ERROR_INVALID_VALUE;
-  if (M == 0 || N == 0) return VS_SUCCESS;
-  // col_idx / vals / B may be NULL only when they are never read (nnz_v == 0 or K == 0)
-  if (row_ptr == nullptr || C == nullptr) return VS_ERROR_INVALID_VALUE;
-  if (!al(row_ptr, 4) || (col_idx && !al(col_idx, 4))) return VS_ERROR_MISALIGNED;
-  if ((vals && !al(vals, 2)) || (B && !al(B, 2)) || !al(C, 2)) return VS_ERROR_MISALIGNED;
+  vs_status_t st0 = check_spmm(M, K, N, V, row_ptr, col_idx, vals, B, C);
+  if (st0 != VS_SUCCESS || M == 0 || N == 0) return st0;
   DevInfo info;
   vs_status_t st = check_device(&info);
   if (st != VS_SUCCESS) return st;
@@ -121,18 +161,110 @@ vs_status_t vs_spmm(int64_t M, int64_t K, int64_t N, int V, const int32_t* row_p
 vs_status_t vs_sddmm(int64_t M, int64_t N, int64_t K, int V, const int32_t* row_ptr,
                      const int32_t* col_idx, const void* A, const void* Bt, void* out_vals,
                      vs_stream_t stream) {
-  if (!valid_v(V) || M < 0 || K < 0 || N < 0) return VS_ERROR_INVALID_VALUE;
-  if (M == 0 || N == 0) return VS_SUCCESS;
-  // col_idx / A / Bt / out_vals may be NULL only when never touched (nnz_v == 0)
-  if (row_ptr == nullptr) return VS_ERROR_INVALID_VALUE;
-  if (!al(row_ptr, 4) || (col_idx && !al(col_idx, 4))) return VS_ERROR_MISALIGNED;
-  if ((A && !al(A, 2)) || (Bt && !al(Bt, 2)) || (out_vals && !al(out_vals, 2)))
-    return VS_ERROR_MISALIGNED;
+  vs_status_t st0 = check_sddmm(M, N, K, V, row_ptr, col_idx, A, Bt, out_vals);
+  if (st0 != VS_SUCCESS || M == 0 || N == 0) return st0;
   DevInfo info;
   vs_status_t st = check_device(&info);
   if (st != VS_SUCCESS) return st;
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   return from_cuda(vs::launch_sddmm(M, N, K, V, row_ptr, col_idx, A, Bt, out_vals, info.num_sms, s));
+}
+
+vs_status_t vs_spmm_batched(int64_t count, const vs_spmm_problem_t* problems, vs_stream_t stream) {
+  if (count < 0 || (count > 0 && problems == nullptr)) return VS_ERROR_INVALID_VALUE;
+  for (int64_t i = 0; i < count; ++i) {
+    const vs_spmm_problem_t& p = problems[i];
+    const vs_status_t st = check_spmm(p.M, p.K, p.N, p.V, p.row_ptr, p.col_idx, p.vals, p.B, p.C);
+    if (st != VS_SUCCESS) return st;
+  }
+  if (count == 0) return VS_SUCCESS;
+  DevInfo info;
+  vs_status_t st = check_device(&info);
+  if (st != VS_SUCCESS) return st;
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  std::vector<int64_t> M, K, N;
+  std::vector<int> V;
+  std::vector<const int32_t*> rp, ci;
+  std::vector<const void*> va, B;
+  std::vector<void*> C;
+  for (int64_t i = 0; i < count; ++i) {
+    const vs_spmm_problem_t& p = problems[i];
+    if (p.M == 0 || p.N == 0) continue;
+    if (p.K == 0) {
+      if (cudaMemsetAsync(p.C, 0, (size_t)(p.M * p.N) * 2, s) != cudaSuccess) return VS_ERROR_CUDA;
+      continue;
+    }
+    M.push_back(p.M); K.push_back(p.K); N.push_back(p.N); V.push_back(p.V);
+    rp.push_back(p.row_ptr); ci.push_back(p.col_idx); va.push_back(p.vals); B.push_back(p.B);
+    C.push_back(p.C);
+  }
+  if (M.empty()) return VS_SUCCESS;
+  return from_cuda(vs::launch_spmm_batched((int64_t)M.size(), M.data(), K.data(), N.data(), V.data(),
+                                           rp.data(), ci.data(), va.data(), B.data(), C.data(), s));
+}
+
+vs_status_t vs_sddmm_batched(int64_t count, const vs_sddmm_problem_t* problems,
+                             vs_stream_t stream) {
+  if (count < 0 || (count > 0 && problems == nullptr)) return VS_ERROR_INVALID_VALUE;
+  for (int64_t i = 0; i < count; ++i) {
+    const vs_sddmm_problem_t& p = problems[i];
+    const vs_status_t st = check_sddmm(p.M, p.N, p.K, p.V, p.row_ptr, p.col_idx, p.A, p.Bt, p.out_vals);
+    if (st != VS_SUCCESS) return st;
+  }
+  if (count == 0) return VS_SUCCESS;
+  DevInfo info;
+  vs_status_t st = check_device(&info);
+  if (st != VS_SUCCESS) return st;
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  std::vector<int64_t> M, K;
+  std::vector<int> V;
+  std::vector<const int32_t*> rp, ci;
+  std::vector<const void*> A, Bt;
+  std::vector<void*> out;
+  for (int64_t i = 0; i < count; ++i) {
+    const vs_sddmm_problem_t& p = problems[i];
+    if (p.M == 0 || p.N == 0) continue;
+    M.push_back(p.M); K.push_back(p.K); V.push_back(p.V); rp.push_back(p.row_ptr);
+    ci.push_back(p.col_idx); A.push_back(p.A); Bt.push_back(p.Bt); out.push_back(p.out_vals);
+  }
+  if (M.empty()) return VS_SUCCESS;
+  return from_cuda(vs::launch_sddmm_batched((int64_t)M.size(), M.data(), K.data(), V.data(), rp.data(),
+                                            ci.data(), A.data(), Bt.data(), out.data(),
+                                            info.num_sms, s));
+}
+
+vs_status_t vs_encode_colvec_batched(int64_t count, const vs_encode_problem_t* problems,
+                                     vs_stream_t stream) {
+  if (count < 0 || (count > 0 && problems == nullptr)) return VS_ERROR_INVALID_VALUE;
+  for (int64_t i = 0; i < count; ++i) {
+    const vs_encode_problem_t& p = problems[i];
+    const vs_status_t st = check_encode(p.M, p.K, p.V, p.dense, p.mask, p.row_ptr, p.col_idx, p.vals);
+    if (st != VS_SUCCESS) return st;
+  }
+  if (count == 0) return VS_SUCCESS;
+  DevInfo info;
+  vs_status_t st = check_device(&info);
+  if (st != VS_SUCCESS) return st;
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  std::vector<int64_t> M, K;
+  std::vector<int> V;
+  std::vector<const void*> dense;
+  std::vector<const uint8_t*> mask;
+  std::vector<int32_t*> rp, ci;
+  std::vector<void*> vals;
+  for (int64_t i = 0; i < count; ++i) {
+    const vs_encode_problem_t& p = problems[i];
+    if (p.M == 0) {  // W == 0: row_ptr = [0]
+      if (cudaMemsetAsync(p.row_ptr, 0, sizeof(int32_t), s) != cudaSuccess) return VS_ERROR_CUDA;
+      continue;
+    }
+    M.push_back(p.M); K.push_back(p.K); V.push_back(p.V); dense.push_back(p.dense);
+    mask.push_back(p.mask); rp.push_back(p.row_ptr); ci.push_back(p.col_idx); vals.push_back(p.vals);
+  }
+  if (M.empty()) return VS_SUCCESS;
+  return from_cuda(vs::launch_encode_batched((int64_t)M.size(), M.data(), K.data(), V.data(),
+                                             dense.data(), mask.data(), rp.data(), ci.data(),
+                                             vals.data(), s));
 }
 
 }  // extern "C"

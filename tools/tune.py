@@ -21,7 +21,53 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 
 
+def child_batched(op, workload, reps):
+    """Times one batched call over the whole workload (CUDA graph of `reps` calls)."""
+    import torch
+    import paper_conf_sc_chenqldx21_b200 as vs
+    from synth.workloads import WORKLOADS
+    from bench import layer_inputs
+    torch.cuda.set_device(0)
+    st = torch.cuda.Stream()
+    enc, sp, sd = [], [], []
+    for p in WORKLOADS[workload]():
+        Wd, X, G = layer_inputs(p)
+        Wd, X, G = (torch.from_numpy(a).cuda() for a in (Wd, X, G))
+        rp, ci, va = vs.encode(p.V, dense=Wd)
+        nnz = int(rp[-1].item())
+        Y = torch.empty((p.M, p.N), dtype=torch.float16, device="cuda")
+        dW = torch.empty(max(nnz, 1) * p.V, dtype=torch.float16, device="cuda")
+        enc.append((p.M, p.K, p.V, Wd, None, rp, ci, va))
+        sp.append((p.M, p.K, p.N, p.V, rp, ci, va, X, Y))
+        sd.append((p.M, p.K, p.N, p.V, rp, ci, G, X, dW))
+    arr = {"encode": vs.make_encode_batch(enc), "spmm": vs.make_spmm_batch(sp),
+           "sddmm": vs.make_sddmm_batch(sd)}[op]
+    call = {"encode": vs.vs_encode_colvec_batched, "spmm": vs.vs_spmm_batched,
+            "sddmm": vs.vs_sddmm_batched}[op]
+    with torch.cuda.stream(st):
+        call(arr)
+    st.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=st):
+        for _ in range(reps):
+            call(arr)
+    with torch.cuda.stream(st):
+        g.replay()
+    best = 1e30
+    for _ in range(3):
+        s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        with torch.cuda.stream(st):
+            s.record()
+            g.replay()
+            e.record()
+        e.synchronize()
+        best = min(best, s.elapsed_time(e) * 1e3 / reps)
+    print("JSON" + json.dumps([{"id": f"{workload}:{op}_batched", "us": best, "nnz_v": 0}]))
+
+
 def child(op, workload, reps):
+    if op.endswith("_batched"):
+        return child_batched(op[:-8], workload, reps)
     import torch
     import paper_conf_sc_chenqldx21_b200 as vs
     from synth.workloads import WORKLOADS
