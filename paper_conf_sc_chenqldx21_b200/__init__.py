@@ -26,7 +26,8 @@ __all__ = ["VSError", "lib_path", "load", "vs_encode_colvec", "vs_spmm", "vs_sdd
            "encode", "spmm", "sddmm", "num_windows"]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-lib_path = os.path.join(_PKG, "libvs.so")
+# VS_LIB_PATH overrides the library location (used to compare kernel build variants)
+lib_path = os.environ.get("VS_LIB_PATH") or os.path.join(_PKG, "libvs.so")
 _lib = None
 _lock = threading.Lock()
 

@@ -42,9 +42,22 @@ def up_to_date() -> bool:
     return all(os.path.getmtime(d) <= t for d in _deps())
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
+def build(force: bool = False, verbose: bool = False, out: str = None, defines=()) -> str:
+    """Builds libvs.so (or, with ``out``/``defines``, an experimental variant elsewhere)."""
+    global LIB, BUILD_DIR
+    if out is not None:
+        saved = (LIB, BUILD_DIR)
+        LIB, BUILD_DIR = out, out + ".build"
+        try:
+            return _build(True, verbose, list(defines))
+        finally:
+            LIB, BUILD_DIR = saved
     if not force and up_to_date():
         return LIB
+    return _build(force, verbose, [])
+
+
+def _build(force: bool, verbose: bool, defines) -> str:
     nvcc = nvcc_path()
     os.makedirs(BUILD_DIR, exist_ok=True)
     procs = []
@@ -53,7 +66,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
         name = os.path.splitext(os.path.basename(src))[0]
         obj = os.path.join(BUILD_DIR, name + ".o")
         log = open(os.path.join(BUILD_DIR, f"ptxas_{name}.log"), "w")
-        cmd = [nvcc, *ARCH, *NVCC_FLAGS, "-c", src, "-o", obj]
+        cmd = [nvcc, *ARCH, *NVCC_FLAGS, *("-D" + d for d in defines), "-c", src, "-o", obj]
         procs.append((subprocess.Popen(cmd, stdout=log, stderr=subprocess.STDOUT), log, src))
         objs.append(obj)
     failed = []

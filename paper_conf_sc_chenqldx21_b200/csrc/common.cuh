@@ -13,12 +13,26 @@ constexpr int kWarp = 32;
 __device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
 
 // 16-byte read-only global load, cached in L1 (gathered rows are re-read by other warps
-// of the same SM, so we want them to stay in L1).
+// of the same SM, so we want them to stay in L1).  VS_GATHER_HINT selects a cache-policy
+// variant for experiments (0: default, 1: L1::evict_last, 2: L1::no_allocate).
+#ifndef VS_GATHER_HINT
+#define VS_GATHER_HINT 0
+#endif
 __device__ __forceinline__ uint4 ldg128(const void* p) {
   uint4 r;
+#if VS_GATHER_HINT == 1
+  asm volatile("ld.global.nc.L1::evict_last.v4.u32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+               : "l"(p));
+#elif VS_GATHER_HINT == 2
+  asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+               : "l"(p));
+#else
   asm volatile("ld.global.nc.v4.u32 {%0,%1,%2,%3}, [%4];"
                : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
                : "l"(p));
+#endif
   return r;
 }
 
@@ -146,6 +160,16 @@ __device__ __forceinline__ int64_t warp_lower_bound(const int32_t* __restrict__ 
     lo = lo + (int64_t)last * step + 1;
     const int64_t nhi = lo - 1 + step;  // probe last+1 (if any) is >= target
     if (last < 31 && nhi < hi) hi = nhi;
+  }
+  return lo;
+}
+
+// Last index p in [0, count) with first[p] <= x (first[] non-decreasing, first[0] = 0).
+__device__ __forceinline__ int first_problem(const int64_t* first, int count, int64_t x) {
+  int lo = 0, hi = count - 1;
+  while (lo < hi) {
+    const int mid = (lo + hi + 1) >> 1;
+    if (first[mid] <= x) lo = mid; else hi = mid - 1;
   }
   return lo;
 }

@@ -1,16 +1,15 @@
 // encode.cu — dense fp16 matrix / uint8 mask -> column-vector CSR (§4.2, Fig. 8).
 //
-// Two kernels (+ one memset node), both with one CTA per row window and one warp per
-// 256-column chunk (up to 8 warps); each lane tests 8 consecutive columns with one 16-byte
-// load per row of the window.  Keep bit = any nonzero fp16 bit pattern (or mask byte) over
-// the window's V rows.
-//   1. encode_count_scan : counts the window's kept vectors into row_ptr[w+1]; the LAST CTA
-//      to finish (a ticket taken with one atomic on row_ptr[0], preset to -1) turns the counts
-//      into the inclusive prefix in place and sets row_ptr[0] = 0.  No CTA ever waits for
-//      another, so any grid size and any concurrent work on the device are safe.
-//   2. encode_compact    : re-reads the window (L2-resident), block-scans the lanes' keep
-//      counts and writes col_idx and the V values of each kept vector (transposed from the V
-//      row loads into vector-major order) starting at row_ptr[w].
+// Three kernels (+ one memset node), count and compact with one CTA per row window and one
+// warp per 256-column chunk (up to 8 warps); each lane tests 8 consecutive columns with one
+// 16-byte load per row of the window.  Keep bit = any nonzero fp16 bit pattern (or mask
+// byte) over the window's V rows.
+//   1. encode_count   : each warp adds its chunk's count to row_ptr[w+1] (zeroed by the
+//      memset) with one reduction atomic: no barrier, no waiting, order-independent.
+//   2. encode_scan    : one CTA turns the counts into the inclusive prefix in place.
+//   3. encode_compact : re-reads the window (L2-resident), block-scans the lanes' keep counts
+//      and writes col_idx and the V values of each kept vector (transposed from the V row
+//      loads into vector-major order) starting at row_ptr[w].
 // Columns are visited in ascending order, so col_idx ascends inside each window (Fig. 8).
 #include <algorithm>
 #include <utility>
@@ -143,14 +142,14 @@ __device__ void block_scan_inplace(int32_t* a, int64_t n, int32_t* s_warp, int32
   }
 }
 
+// Phase 1: each warp counts the kept vectors of its 256-column chunks of window w and adds
+// them to row_ptr[w+1] (zeroed beforehand) with one reduction atomic -- no barrier, no
+// waiting; integer addition makes the result independent of the order.
 template <int V, bool VEC, bool HAS_MASK>
-__device__ __forceinline__ void count_scan_body(int64_t M, int64_t K, int64_t W, int64_t w,
-                                                const uint16_t* __restrict__ dense,
-                                                const uint8_t* __restrict__ mask,
-                                                int32_t* __restrict__ row_ptr) {
-  __shared__ int32_t s_warp[kEncMaxThreads / 32];
-  __shared__ int32_t s_carry;
-  __shared__ int s_last;
+__device__ __forceinline__ void count_body(int64_t M, int64_t K, int64_t w,
+                                           const uint16_t* __restrict__ dense,
+                                           const uint8_t* __restrict__ mask,
+                                           int32_t* __restrict__ row_ptr) {
   const int lane = lane_id(), wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
   uint16_t h[V][8];
   uint32_t count = 0;
@@ -160,21 +159,7 @@ __device__ __forceinline__ void count_scan_body(int64_t M, int64_t K, int64_t W,
   }
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) count += __shfl_xor_sync(0xffffffffu, count, o);
-  if (lane == 0) s_warp[wid] = (int32_t)count;
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    int32_t tot = 0;
-    for (int i = 0; i < nw; ++i) tot += s_warp[i];
-    row_ptr[w + 1] = tot;
-    __threadfence();  // publish the count before taking the ticket
-    const int ticket = atomicAdd(row_ptr, 1);  // row_ptr[0] was preset to -1
-    s_last = (ticket == (int)(W - 2));
-  }
-  __syncthreads();
-  if (!s_last) return;
-  __threadfence();  // all counts are visible to the last CTA
-  block_scan_inplace(row_ptr + 1, W, s_warp, &s_carry);
-  if (threadIdx.x == 0) row_ptr[0] = 0;
+  if (lane == 0 && count) atomicAdd(row_ptr + w + 1, (int32_t)count);
 }
 
 // Writes col_idx and (optionally) vals of window w from row_ptr[w] on.  Per round, warp i
@@ -244,9 +229,18 @@ __device__ __forceinline__ void compact_body(int64_t M, int64_t K, int64_t w,
 
 template <int V, bool VEC, bool HAS_MASK>
 __global__ void __launch_bounds__(kEncMaxThreads)
-    encode_count_scan_kernel(int64_t M, int64_t K, int64_t W, const uint16_t* __restrict__ dense,
-                             const uint8_t* __restrict__ mask, int32_t* __restrict__ row_ptr) {
-  count_scan_body<V, VEC, HAS_MASK>(M, K, W, blockIdx.x, dense, mask, row_ptr);
+    encode_count_kernel(int64_t M, int64_t K, const uint16_t* __restrict__ dense,
+                        const uint8_t* __restrict__ mask, int32_t* __restrict__ row_ptr) {
+  count_body<V, VEC, HAS_MASK>(M, K, blockIdx.x, dense, mask, row_ptr);
+}
+
+// Phase 2: counts -> inclusive prefix, in place (one CTA).
+constexpr int kScanThreads = 1024;
+__global__ void __launch_bounds__(kScanThreads) encode_scan_kernel(int32_t* __restrict__ row_ptr,
+                                                                   int64_t W) {
+  __shared__ int32_t s_warp[32];
+  __shared__ int32_t s_carry;
+  block_scan_inplace(row_ptr + 1, W, s_warp, &s_carry);
 }
 
 template <int V, bool VEC, bool HAS_MASK, bool WRITE_VALS, bool VEC_VALS>
@@ -275,35 +269,48 @@ struct EncBatch {
   EncDesc d[kEncMaxBatch];
 };
 
-__device__ __forceinline__ int find_problem(const EncBatch& b, int64_t bid) {
-  int lo = 0, hi = b.count - 1;
-  while (lo < hi) {
-    const int mid = (lo + hi + 1) >> 1;
-    if (b.first_block[mid] <= bid) lo = mid; else hi = mid - 1;
-  }
-  return lo;
+// zero row_ptr[0..W] of every problem of the batch
+__global__ void zero_row_ptr_kernel(const __grid_constant__ EncBatch b) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int p = 0; p < b.count; ++p)
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i <= b.d[p].W; i += stride)
+      b.d[p].row_ptr[i] = 0;
 }
 
-__global__ void ticket_init_kernel(const __grid_constant__ EncBatch b) {
-  for (int p = threadIdx.x; p < b.count; p += blockDim.x) b.d[p].row_ptr[0] = -1;
-}
-
+// Batched kernels: grid-stride loop over the windows of all problems (launched with one CTA
+// per window, so usually one iteration); first problem by binary search, then a forward
+// linear advance.
 template <int V, bool VEC, bool HAS_MASK>
 __global__ void __launch_bounds__(kEncMaxThreads)
-    encode_count_scan_batched_kernel(const __grid_constant__ EncBatch b) {
-  const int p = find_problem(b, blockIdx.x);
-  const EncDesc& d = b.d[p];
-  count_scan_body<V, VEC, HAS_MASK>(d.M, d.K, d.W, blockIdx.x - b.first_block[p], d.dense, d.mask,
-                                    d.row_ptr);
+    encode_count_batched_kernel(const __grid_constant__ EncBatch b) {
+  const int64_t total = b.first_block[b.count];
+  int p = first_problem(b.first_block, b.count, (int64_t)blockIdx.x);
+  for (int64_t bid = blockIdx.x; bid < total; bid += gridDim.x) {
+    while (b.first_block[p + 1] <= bid) ++p;
+    const EncDesc& d = b.d[p];
+    count_body<V, VEC, HAS_MASK>(d.M, d.K, bid - b.first_block[p], d.dense, d.mask, d.row_ptr);
+  }
+}
+
+// one CTA per problem
+__global__ void __launch_bounds__(kScanThreads) encode_scan_batched_kernel(const __grid_constant__ EncBatch b) {
+  __shared__ int32_t s_warp[32];
+  __shared__ int32_t s_carry;
+  const EncDesc& d = b.d[blockIdx.x];
+  block_scan_inplace(d.row_ptr + 1, d.W, s_warp, &s_carry);
 }
 
 template <int V, bool VEC, bool HAS_MASK, bool WRITE_VALS, bool VEC_VALS>
 __global__ void __launch_bounds__(kEncMaxThreads)
     encode_compact_batched_kernel(const __grid_constant__ EncBatch b) {
-  const int p = find_problem(b, blockIdx.x);
-  const EncDesc& d = b.d[p];
-  compact_body<V, VEC, HAS_MASK, WRITE_VALS, VEC_VALS>(d.M, d.K, blockIdx.x - b.first_block[p],
-                                                       d.dense, d.mask, d.row_ptr, d.col_idx, d.vals);
+  const int64_t total = b.first_block[b.count];
+  int p = first_problem(b.first_block, b.count, (int64_t)blockIdx.x);
+  for (int64_t bid = blockIdx.x; bid < total; bid += gridDim.x) {
+    while (b.first_block[p + 1] <= bid) ++p;
+    const EncDesc& d = b.d[p];
+    compact_body<V, VEC, HAS_MASK, WRITE_VALS, VEC_VALS>(d.M, d.K, bid - b.first_block[p], d.dense,
+                                                         d.mask, d.row_ptr, d.col_idx, d.vals);
+  }
 }
 
 struct EncCfg {
@@ -332,7 +339,7 @@ static int enc_threads(int64_t K) {  // one warp per 256-column chunk, up to 8 w
 }
 
 struct EncKernels {
-  void (*count_single)(int64_t, int64_t, int64_t, const uint16_t*, const uint8_t*, int32_t*);
+  void (*count_single)(int64_t, int64_t, const uint16_t*, const uint8_t*, int32_t*);
   void (*compact_single)(int64_t, int64_t, const uint16_t*, const uint8_t*, const int32_t*, int32_t*,
                          uint16_t*);
   void (*count_batched)(EncBatch);
@@ -342,8 +349,8 @@ struct EncKernels {
 template <int V, bool VEC, bool MASKB>
 static EncKernels enc_kernels_vm(const EncCfg& c) {
   EncKernels k;
-  k.count_single = encode_count_scan_kernel<V, VEC, MASKB>;
-  k.count_batched = encode_count_scan_batched_kernel<V, VEC, MASKB>;
+  k.count_single = encode_count_kernel<V, VEC, MASKB>;
+  k.count_batched = encode_count_batched_kernel<V, VEC, MASKB>;
   if (!c.VALS) {
     k.compact_single = encode_compact_kernel<V, VEC, MASKB, false, false>;
     k.compact_batched = encode_compact_batched_kernel<V, VEC, MASKB, false, false>;
@@ -381,10 +388,10 @@ cudaError_t launch_encode(int64_t M, int64_t K, int V, const void* dense, const 
   const EncKernels k = enc_kernels(c);
   const dim3 grid((unsigned)W), block(enc_threads(K));
   const uint16_t* d = static_cast<const uint16_t*>(dense);
-  // row_ptr[0] = -1: the ticket counter of encode_count_scan (reset to 0 by the last CTA)
-  cudaError_t e = cudaMemsetAsync(row_ptr, 0xFF, sizeof(int32_t), s);
+  cudaError_t e = cudaMemsetAsync(row_ptr, 0, (size_t)(W + 1) * sizeof(int32_t), s);
   if (e != cudaSuccess) return e;
-  k.count_single<<<grid, block, 0, s>>>(M, K, W, d, mask, row_ptr);
+  k.count_single<<<grid, block, 0, s>>>(M, K, d, mask, row_ptr);
+  encode_scan_kernel<<<1, kScanThreads, 0, s>>>(row_ptr, W);
   if (c.IDX)
     k.compact_single<<<grid, block, 0, s>>>(M, K, d, mask, row_ptr, col_idx,
                                             static_cast<uint16_t*>(vals));
@@ -395,7 +402,7 @@ cudaError_t launch_encode(int64_t M, int64_t K, int V, const void* dense, const 
 cudaError_t launch_encode_batched(int64_t count, const int64_t* M, const int64_t* K, const int* V,
                                   const void* const* dense, const uint8_t* const* mask,
                                   int32_t* const* row_ptr, int32_t* const* col_idx,
-                                  void* const* vals, cudaStream_t s) {
+                                  void* const* vals, int num_sms, cudaStream_t s) {
   std::vector<std::pair<int, int64_t>> order;
   for (int64_t i = 0; i < count; ++i)
     order.push_back({enc_config(K[i], V[i], dense[i], mask[i], col_idx[i], vals[i]).key(), i});
@@ -425,8 +432,11 @@ cudaError_t launch_encode_batched(int64_t count, const int64_t* M, const int64_t
     }
     if (batch.count == 0) return cudaErrorInvalidConfiguration;
     batch.first_block[batch.count] = blocks;
-    ticket_init_kernel<<<1, 128, 0, s>>>(batch);
+    zero_row_ptr_kernel<<<64, 256, 0, s>>>(batch);
+    // one CTA per window (measured slightly faster than a resident-sized grid-stride grid)
+    (void)num_sms;
     k.count_batched<<<(unsigned)blocks, threads, 0, s>>>(batch);
+    encode_scan_batched_kernel<<<batch.count, kScanThreads, 0, s>>>(batch);
     if (c.IDX) k.compact_batched<<<(unsigned)blocks, threads, 0, s>>>(batch);
     const cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;

@@ -98,10 +98,13 @@ __device__ __forceinline__ void store_slice(const float (&acc)[4], int64_t v0, i
 }
 
 // One warp computes the 16-vector slices [s_begin, s_end) of one problem (nnz stored
-// vectors in total); s_begin < s_end.  A slice that straddles windows is finished window by
-// window; the next 64-wide K chunk of the gathered rows is prefetched while the current
-// chunk's MMAs run.  (A variant that processed 2 or 4 slices of one window together to share
-// the A fragment measured no faster, tools/tune.py, and was dropped.)
+// vectors in total); s_begin < s_end.  The work is one stream of 64-wide K chunks (slice by
+// slice; a slice that straddles windows is finished window by window, re-reading its rows),
+// software-pipelined one chunk ahead: while the MMAs of a chunk run, the gathered Bt rows of
+// the next chunk -- possibly the first chunk of the next segment or slice -- are in flight,
+// and the column indices of the next slice are fetched one slice ahead.  The first loads are
+// issued before the window search, which does not affect them.  (Processing 2 or 4 slices of
+// one window together to share the A fragment measured no faster, tools/tune.py.)
 template <int V, bool VEC>
 __device__ __forceinline__ void sddmm_range(int64_t M, int64_t K, int64_t W,
                                             const int32_t* __restrict__ row_ptr,
@@ -113,41 +116,51 @@ __device__ __forceinline__ void sddmm_range(int64_t M, int64_t K, int64_t W,
   const int lane = lane_id();
   const int g = lane >> 2, t = lane & 3;
   const int64_t kt = 8 * t;
-  int64_t w = find_window(row_ptr, W, s_begin * 16);
+  int64_t v0 = s_begin * 16;
+  int64_t v_hi = (v0 + 16 < nnz) ? v0 + 16 : nnz;
+  bool oka = v0 + g < v_hi, okb = v0 + g + 8 < v_hi;
+  const uint16_t* rowa = Bt + (int64_t)(oka ? ldg32i(col_idx + v0 + g) : 0) * K;
+  const uint16_t* rowb = Bt + (int64_t)(okb ? ldg32i(col_idx + v0 + g + 8) : 0) * K;
+  uint4 a0, a1, b0, b1;  // Bt chunk [k0, k0 + 64) of vectors g and g+8 (the next one to use)
+  load_seg2<VEC>(rowa, K, kt, oka, a0, a1);
+  load_seg2<VEC>(rowb, K, kt, okb, b0, b1);
+  int64_t w = find_window(row_ptr, W, v0);
   int64_t w_end_p = row_ptr[w + 1];
 
-  int64_t s = s_begin;
-  while (s < s_end) {
-    const int64_t v0 = s * 16;
-    while (w_end_p <= v0) {  // advance to the window owning v0
-      ++w;
-      w_end_p = row_ptr[w + 1];
-    }
-    const int64_t v_hi = (v0 + 16 < nnz) ? v0 + 16 : nnz;
-    const bool oka = v0 + g < v_hi, okb = v0 + g + 8 < v_hi;
-    const uint16_t* rowa = Bt + (int64_t)(oka ? ldg32i(col_idx + v0 + g) : 0) * K;
-    const uint16_t* rowb = Bt + (int64_t)(okb ? ldg32i(col_idx + v0 + g + 8) : 0) * K;
+  for (int64_t s = s_begin; s < s_end; ++s) {
+    // next slice's column indices, one slice ahead
+    const bool has_next = s + 1 < s_end;
+    const int64_t nv0 = v0 + 16;
+    const int64_t nv_hi = (nv0 + 16 < nnz) ? nv0 + 16 : nnz;
+    const bool noka = has_next && nv0 + g < nv_hi, nokb = has_next && nv0 + g + 8 < nv_hi;
+    const int nca = noka ? ldg32i(col_idx + nv0 + g) : 0;
+    const int ncb = nokb ? ldg32i(col_idx + nv0 + g + 8) : 0;
+
     int64_t v_cur = v0;
     while (v_cur < v_hi) {
-      while (w_end_p <= v_cur) {
+      while (w_end_p <= v_cur) {  // advance to the window owning v_cur
         ++w;
         w_end_p = row_ptr[w + 1];
       }
       const int64_t seg_hi = w_end_p < v_hi ? w_end_p : v_hi;  // vectors [v_cur, seg_hi) in w
-      const int64_t srow = w * V + g;
-      const bool sok_row = (g < V) && (srow < M);
-      const uint16_t* srowA = A + srow * K;
-      uint4 a0, a1, b0, b1;  // Bt chunk [k0, k0 + 64) of vectors g and g+8
-      load_seg2<VEC>(rowa, K, kt, oka, a0, a1);
-      load_seg2<VEC>(rowb, K, kt, okb, b0, b1);
+      const bool last_seg = seg_hi == v_hi;
+      const int64_t arow = w * V + g;
+      const bool ok_row = (g < V) && (arow < M);
+      const uint16_t* rowA = A + arow * K;
       float acc[4] = {0.f, 0.f, 0.f, 0.f};
       for (int64_t k0 = 0; k0 < K; k0 += 64) {
         uint4 x0, x1;  // A row g of the window, same K permutation
-        load_seg2<VEC>(srowA, K, k0 + kt, sok_row, x0, x1);
+        load_seg2<VEC>(rowA, K, k0 + kt, ok_row, x0, x1);
         const uint4 ca0 = a0, ca1 = a1, cb0 = b0, cb1 = b1;
-        if (k0 + 64 < K) {  // prefetch the next chunk of the gathered rows
+        if (k0 + 64 < K) {  // next chunk of the same rows
           load_seg2<VEC>(rowa, K, k0 + 64 + kt, oka, a0, a1);
           load_seg2<VEC>(rowb, K, k0 + 64 + kt, okb, b0, b1);
+        } else if (!last_seg) {  // the same rows again, for the slice's next window
+          load_seg2<VEC>(rowa, K, kt, oka, a0, a1);
+          load_seg2<VEC>(rowb, K, kt, okb, b0, b1);
+        } else if (has_next) {  // first chunk of the next slice
+          load_seg2<VEC>(Bt + (int64_t)nca * K, K, kt, noka, a0, a1);
+          load_seg2<VEC>(Bt + (int64_t)ncb * K, K, kt, nokb, b0, b1);
         }
 #pragma unroll
         for (int j = 0; j < 4; ++j)
@@ -157,7 +170,12 @@ __device__ __forceinline__ void sddmm_range(int64_t M, int64_t K, int64_t W,
       store_slice<V>(acc, v0, v_cur, seg_hi, w, M, g, t, out, out4);
       v_cur = seg_hi;
     }
-    s += 1;
+    v0 = nv0;
+    v_hi = nv_hi;
+    oka = noka;
+    okb = nokb;
+    rowa = Bt + (int64_t)nca * K;
+    rowb = Bt + (int64_t)ncb * K;
   }
 }
 
@@ -177,13 +195,10 @@ __global__ void __launch_bounds__(kSddmmWarps * 32)
   sddmm_range<V, VEC>(M, K, W, row_ptr, col_idx, A, Bt, out, out4, s_begin, s_end, nnz);
 }
 
-// Batched launch over up to kSddmmMaxBatch problems of one configuration.  The work of a
-// problem is its slice count times its number of 64-wide K chunks (slice counts from each
-// problem's row_ptr[W], read on the device and prefix-summed per CTA in shared memory); the
-// total work is split evenly over the persistent warps, a warp's share of a problem being
-// the slices whose work offsets fall in the warp's range, so problems with different K are
-// balanced and every slice is computed exactly once.  A warp's run may cross into the next
-// problem.
+// Batched launch over up to kSddmmMaxBatch problems of one configuration.  Each problem's
+// slices (count from its row_ptr[W], read on the device and prefix-summed per CTA in shared
+// memory) are cut into chunks of kSliceChunk slices; the chunks of all problems are dealt
+// round-robin to the persistent warps.
 struct SddmmDesc {
   int64_t M, K, W;
   const int32_t* row_ptr;
@@ -194,6 +209,7 @@ struct SddmmDesc {
   int64_t out4;
 };
 constexpr int kSddmmMaxBatch = 128;
+constexpr int kSliceChunk = 8;  // slices per work chunk of the batched kernel
 struct SddmmBatch {
   int count;
   SddmmDesc d[kSddmmMaxBatch];
@@ -202,17 +218,15 @@ struct SddmmBatch {
 template <int V, bool VEC>
 __global__ void __launch_bounds__(kSddmmWarps * 32)
     sddmm_batched_kernel(const __grid_constant__ SddmmBatch b) {
-  __shared__ int64_t pre[kSddmmMaxBatch + 1];  // work prefix (slices * chunks)
+  __shared__ int64_t pre[kSddmmMaxBatch + 1];  // prefix of slice-chunk counts
   __shared__ int64_t nnzs[kSddmmMaxBatch];
-  __shared__ int32_t nks[kSddmmMaxBatch];      // 64-wide K chunks per slice (>= 1)
   const int lane = lane_id();
   if (threadIdx.x < 32) {
     int64_t carry = 0;
     for (int base = 0; base < b.count; base += 32) {
       const int p = base + lane;
       const int64_t nz = p < b.count ? (int64_t)b.d[p].row_ptr[b.d[p].W] : 0;
-      const int64_t nk = p < b.count ? (b.d[p].K > 64 ? ceil_div64(b.d[p].K, 64) : 1) : 1;
-      const int64_t v = ceil_div64(nz, 16) * nk;
+      const int64_t v = ceil_div64(ceil_div64(nz, 16), kSliceChunk);  // chunks of slices
       int64_t incl = v;
 #pragma unroll
       for (int o = 1; o < 32; o <<= 1) {
@@ -222,36 +236,24 @@ __global__ void __launch_bounds__(kSddmmWarps * 32)
       if (p < b.count) {
         pre[p] = carry + incl - v;
         nnzs[p] = nz;
-        nks[p] = (int32_t)nk;
       }
       carry += __shfl_sync(0xffffffffu, incl, 31);
     }
     if (lane == 0) pre[b.count] = carry;
   }
   __syncthreads();
-  const int64_t total = pre[b.count];
+  // Work is dealt in rounds of chunks of kSliceChunk slices: chunk c of the global chunk
+  // sequence goes to warp c % n_warps, so at any time the warps work on neighbouring chunks
+  // (one or two problems resident in L2), instead of every warp touching its own problem.
+  const int64_t n_chunks = pre[b.count];
   const int64_t n_warps = (int64_t)gridDim.x * kSddmmWarps;
   const int64_t gw = (int64_t)blockIdx.x * kSddmmWarps + (threadIdx.x >> 5);
-  const int64_t per = ceil_div64(total, n_warps);
-  const int64_t wb = gw * per;
-  const int64_t we = (wb + per < total) ? wb + per : total;
-  if (wb >= we) return;
   int p = 0;
-  {
-    int lo = 0, hi = b.count - 1;  // last problem with pre[p] <= wb
-    while (lo < hi) {
-      const int mid = (lo + hi + 1) >> 1;
-      if (pre[mid] <= wb) lo = mid; else hi = mid - 1;
-    }
-    p = lo;
-  }
-  for (; p < b.count && pre[p] < we; ++p) {
-    // this warp's slices of problem p: those whose work offset s*nk lies in [wb, we)
-    const int64_t nk = nks[p];
-    const int64_t lo = wb > pre[p] ? wb - pre[p] : 0;
-    const int64_t hi = (we < pre[p + 1] ? we : pre[p + 1]) - pre[p];
-    const int64_t s0 = ceil_div64(lo, nk), s1 = ceil_div64(hi, nk);
-    if (s0 >= s1) continue;
+  for (int64_t c = gw; c < n_chunks; c += n_warps) {
+    while (pre[p + 1] <= c) ++p;
+    const int64_t s0 = (c - pre[p]) * kSliceChunk;
+    const int64_t slices = ceil_div64(nnzs[p], 16);
+    const int64_t s1 = s0 + kSliceChunk < slices ? s0 + kSliceChunk : slices;
     const SddmmDesc& d = b.d[p];
     sddmm_range<V, VEC>(d.M, d.K, d.W, d.row_ptr, d.col_idx, d.A, d.Bt, d.out, d.out4 != 0, s0, s1,
                         nnzs[p]);

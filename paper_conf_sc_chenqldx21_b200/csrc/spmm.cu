@@ -171,16 +171,16 @@ __device__ __forceinline__ void spmm_body(int64_t M, int64_t N, int64_t W, int64
       }
       __syncthreads();
     }
-    if (part != 0) return;
   }
-  if (!active) return;
+  // (no early return: the batched kernel calls this body in a loop with barriers)
+  const bool store = part == 0 && active;
 
   // Epilogue: thread holds rows 2t, 2t+1 x columns [ncol0 + 64c, +8).
 #pragma unroll
   for (int rr = 0; rr < 2; ++rr) {
     const int r = 2 * t + rr;
     const int64_t i = w * V + r;
-    if (r >= V || i >= M) continue;
+    if (!store || r >= V || i >= M) continue;
 #pragma unroll
     for (int c = 0; c < NC; ++c) {
       const int64_t n = ncol0 + 64 * c;
@@ -231,15 +231,16 @@ struct SpmmBatch {
 template <int V, int NC, bool VEC, int SPLIT, int UNROLL>
 __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32)
     spmm_batched_kernel(const __grid_constant__ SpmmBatch b) {
-  const int64_t bid = blockIdx.x;
-  int lo = 0, hi = b.count - 1;
-  while (lo < hi) {
-    const int mid = (lo + hi + 1) >> 1;
-    if (b.first_block[mid] <= bid) lo = mid; else hi = mid - 1;
+  // grid-stride over the blocks of all problems (launched with one CTA per block, so usually
+  // one iteration); the first problem by binary search, then a forward linear advance
+  const int64_t total = b.first_block[b.count];
+  int p = first_problem(b.first_block, b.count, (int64_t)blockIdx.x);
+  for (int64_t bid = blockIdx.x; bid < total; bid += gridDim.x) {
+    while (b.first_block[p + 1] <= bid) ++p;
+    const SpmmDesc& d = b.d[p];
+    spmm_body<V, NC, VEC, SPLIT, UNROLL>(d.M, d.N, d.W, d.n_wgroups, bid - b.first_block[p],
+                                         d.row_ptr, d.col_idx, d.vals, d.B, d.C);
   }
-  const SpmmDesc& d = b.d[lo];
-  spmm_body<V, NC, VEC, SPLIT, UNROLL>(d.M, d.N, d.W, d.n_wgroups, bid - b.first_block[lo],
-                                       d.row_ptr, d.col_idx, d.vals, d.B, d.C);
 }
 
 // Kernel configuration of one problem.  NC (64- or 128-column panels) follows N; SPLIT
@@ -270,13 +271,21 @@ struct SpmmKernels {
   void (*single)(int64_t, int64_t, int64_t, int64_t, const int32_t*, const int32_t*,
                  const uint16_t*, const uint16_t*, uint16_t*);
   void (*batched)(SpmmBatch);
-  int threads, units_per_cta;
+  int threads, units_per_cta, batched_ctas_per_sm;
 };
 
 template <int V, int NC, bool VEC, int SPLIT>
 static SpmmKernels kernels_of() {
+  static const int occ = [] {
+    int b = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(
+            &b, spmm_batched_kernel<V, NC, VEC, SPLIT, 1>, SpmmCta<SPLIT>::kWarps * 32, 0) !=
+            cudaSuccess || b < 1)
+      b = 1;
+    return b;
+  }();
   return {spmm_kernel<V, NC, VEC, SPLIT, 1>, spmm_batched_kernel<V, NC, VEC, SPLIT, 1>,
-          SpmmCta<SPLIT>::kWarps * 32, SpmmCta<SPLIT>::kUnits};
+          SpmmCta<SPLIT>::kWarps * 32, SpmmCta<SPLIT>::kUnits, occ};
 }
 
 template <int V, int NC, bool VEC>
@@ -334,7 +343,7 @@ cudaError_t launch_spmm(int64_t M, int64_t K, int64_t N, int V, const int32_t* r
 cudaError_t launch_spmm_batched(int64_t count, const int64_t* M, const int64_t* K, const int64_t* N,
                                 const int* V, const int32_t* const* row_ptr,
                                 const int32_t* const* col_idx, const void* const* vals,
-                                const void* const* B, void* const* C, cudaStream_t s) {
+                                const void* const* B, void* const* C, int num_sms, cudaStream_t s) {
   // group problem indices by configuration (stable: keeps the caller's order inside a group)
   std::vector<std::pair<SpmmCfg, int64_t>> order;
   order.reserve(count);
@@ -365,6 +374,8 @@ cudaError_t launch_spmm_batched(int64_t count, const int64_t* M, const int64_t* 
     }
     if (batch.count == 0) return cudaErrorInvalidConfiguration;
     batch.first_block[batch.count] = blocks;
+    // one CTA per block (measured slightly faster than a resident-sized grid-stride grid)
+    (void)num_sms;
     if (blocks > 0) k.batched<<<(unsigned)blocks, k.threads, 0, s>>>(batch);
     const cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;

@@ -18,7 +18,7 @@ cudaError_t launch_sddmm(int64_t M, int64_t N, int64_t K, int V, const int32_t* 
 cudaError_t launch_spmm_batched(int64_t count, const int64_t* M, const int64_t* K, const int64_t* N,
                                 const int* V, const int32_t* const* row_ptr,
                                 const int32_t* const* col_idx, const void* const* vals,
-                                const void* const* B, void* const* C, cudaStream_t s);
+                                const void* const* B, void* const* C, int num_sms, cudaStream_t s);
 cudaError_t launch_sddmm_batched(int64_t count, const int64_t* M, const int64_t* K, const int* V,
                                  const int32_t* const* row_ptr, const int32_t* const* col_idx,
                                  const void* const* A, const void* const* Bt, void* const* out,
@@ -26,7 +26,7 @@ cudaError_t launch_sddmm_batched(int64_t count, const int64_t* M, const int64_t*
 cudaError_t launch_encode_batched(int64_t count, const int64_t* M, const int64_t* K, const int* V,
                                   const void* const* dense, const uint8_t* const* mask,
                                   int32_t* const* row_ptr, int32_t* const* col_idx,
-                                  void* const* vals, cudaStream_t s);
+                                  void* const* vals, int num_sms, cudaStream_t s);
 }  // namespace vs
 
 namespace {
@@ -200,7 +200,8 @@ vs_status_t vs_spmm_batched(int64_t count, const vs_spmm_problem_t* problems, vs
   }
   if (M.empty()) return VS_SUCCESS;
   return from_cuda(vs::launch_spmm_batched((int64_t)M.size(), M.data(), K.data(), N.data(), V.data(),
-                                           rp.data(), ci.data(), va.data(), B.data(), C.data(), s));
+                                           rp.data(), ci.data(), va.data(), B.data(), C.data(),
+                                           info.num_sms, s));
 }
 
 vs_status_t vs_sddmm_batched(int64_t count, const vs_sddmm_problem_t* problems,
@@ -264,7 +265,7 @@ vs_status_t vs_encode_colvec_batched(int64_t count, const vs_encode_problem_t* p
   if (M.empty()) return VS_SUCCESS;
   return from_cuda(vs::launch_encode_batched((int64_t)M.size(), M.data(), K.data(), V.data(),
                                              dense.data(), mask.data(), rp.data(), ci.data(),
-                                             vals.data(), s));
+                                             vals.data(), info.num_sms, s));
 }
 
 }  // extern "C"
