@@ -180,7 +180,7 @@ def count_launches(bufs):
         q = K >> 8
         return 16 if q >= 16 else 8 if q >= 8 else 4 if q >= 4 else 2 if q >= 2 else 1
     enc = Counter(b.p.V for b in bufs)
-    sp = Counter((b.p.V, 1 if b.p.N <= 64 else 2, split(b.p.K)) for b in bufs)
+    sp = Counter((b.p.V, 1, split(b.p.K)) for b in bufs)  # 64-column panels (NC = 1)
     sd = Counter(b.p.V for b in bufs)
     per = {"encode": sum(4 * _m.ceil(n / 128) for n in enc.values()),
            "spmm": sum(_m.ceil(n / 128) for n in sp.values()),
@@ -723,10 +723,233 @@ def ctypes_int():
     return ctypes.c_int(0)
 
 
+def run_c5(args):
+    """configs[4]: M=K=16384, N=65536, V=8, S=0.9 -- SpMM sharded over N-panels of B/C (A
+    replicated) and SDDMM (mask 16384 x 65536, inner K=16384) sharded over row windows (Bt
+    replicated), no collective on the data path.  Strong scaling: the total
+    problem is fixed, each rank encodes and computes its shard.  Inputs are generated on the
+    device (seeded) and are far larger than L2, so no flush is needed."""
+    import torch
+    import paper_conf_sc_chenqldx21_b200 as vs
+    from paper_conf_sc_chenqldx21_b200 import dist as vsd
+    from synth import gen
+
+    ws, rank, local = dist_env()
+    if ws > 1:
+        import torch.distributed as dist
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    else:
+        torch.cuda.set_device(0)
+    dev = torch.device("cuda", torch.cuda.current_device())
+    vs.load()
+    peaks = load_peaks()
+    M = K = 16384
+    N, V, S = 65536, 8, 0.9
+    W = M // V
+    # SpMM shard: A replicated, this rank's N-panel of B and C
+    pb = vsd.panel_bounds(N, ws)
+    n0, n1 = pb[rank], pb[rank + 1]
+    Np = n1 - n0
+    Ad = gen.torch_colvec_dense(M, K, V, 1 - S, seed=gen.config_seed("c5_A"), device=dev)
+    Bp = gen.torch_dense_operand(K, Np, seed=gen.config_seed(f"c5_B_{n0}"), device=dev)
+    Cp = torch.empty((M, Np), dtype=torch.float16, device=dev)
+    capA = W * K
+    rpA = torch.empty(W + 1, dtype=torch.int32, device=dev)
+    ciA = torch.empty(capA, dtype=torch.int32, device=dev)
+    vaA = torch.empty(capA * V, dtype=torch.float16, device=dev)
+    # SDDMM shard: this rank's row windows of the mask [M x N], Bt [N x K] replicated
+    wb = [(W * r) // ws for r in range(ws + 1)]
+    w0, w1 = wb[rank], wb[rank + 1]
+    Ml = (w1 - w0) * V
+    g = torch.Generator(device=dev)
+    g.manual_seed(gen.config_seed(f"c5_mask_{w0}"))
+    keep = torch.rand((w1 - w0, N), generator=g, device=dev) < (1 - S)
+    maskl = keep.repeat_interleave(V, dim=0).to(torch.uint8).contiguous()
+    del keep
+    Al = gen.torch_dense_operand(Ml, K, seed=gen.config_seed(f"c5_Arows_{w0}"), device=dev)
+    Bt = gen.torch_dense_operand(N, K, seed=gen.config_seed("c5_Bt"), device=dev)
+    capM = (w1 - w0) * N // 8  # >= nnz for density 0.1 with margin (checked below)
+    rpM = torch.empty(w1 - w0 + 1, dtype=torch.int32, device=dev)
+    ciM = torch.empty(capM, dtype=torch.int32, device=dev)
+    outM = torch.empty(capM * V, dtype=torch.float16, device=dev)
+
+    def step():
+        vs.vs_encode_colvec(M, K, V, Ad, None, rpA, ciA, vaA)
+        vs.vs_spmm(M, K, Np, V, rpA, ciA, vaA, Bp, Cp)
+        vs.vs_encode_colvec(Ml, N, V, None, maskl, rpM, ciM, None)
+        vs.vs_sddmm(Ml, N, K, V, rpM, ciM, Al, Bt, outM)
+
+    stream = torch.cuda.Stream()
+    with torch.cuda.stream(stream):
+        step()
+    stream.synchronize()
+    nnzA = int(rpA[-1].item())
+    nnzM = int(rpM[-1].item())
+    assert nnzM <= capM, "mask capacity"
+    flops = 2.0 * nnzA * V * Np + 2.0 * nnzM * V * K
+    ev = {k: (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+          for k in ("encA", "spmm", "encM", "sddmm")}
+
+    def step_instr():
+        for k, fn in (("encA", lambda: vs.vs_encode_colvec(M, K, V, Ad, None, rpA, ciA, vaA)),
+                      ("spmm", lambda: vs.vs_spmm(M, K, Np, V, rpA, ciA, vaA, Bp, Cp)),
+                      ("encM", lambda: vs.vs_encode_colvec(Ml, N, V, None, maskl, rpM, ciM, None)),
+                      ("sddmm", lambda: vs.vs_sddmm(Ml, N, K, V, rpM, ciM, Al, Bt, outM))):
+            ev[k][0].record()
+            fn()
+            ev[k][1].record()
+
+    for _ in range(args.warmup):
+        with torch.cuda.stream(stream):
+            step()
+    stream.synchronize()
+    if ws > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    clocks = ClockSampler(dev.index if ws == 1 else local).start()
+    s0, e0 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with torch.cuda.stream(stream):
+        s0.record()
+        for _ in range(args.steps):
+            step()
+        e0.record()
+    e0.synchronize()
+    ms = s0.elapsed_time(e0) / args.steps
+    cls = {k: 0.0 for k in ev}
+    for _ in range(2):
+        with torch.cuda.stream(stream):
+            step_instr()
+        stream.synchronize()
+        for k, (a, b) in ev.items():
+            cls[k] += a.elapsed_time(b) / 2
+    if ws > 1:
+        torch.distributed.barrier()
+    clk = clocks.stop()
+    tot_flops = flops
+    if ws > 1:
+        t = torch.tensor([ms], device=dev, dtype=torch.float64)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        ms = float(t.item())
+        f = torch.tensor([flops], device=dev, dtype=torch.float64)
+        torch.distributed.all_reduce(f)
+        tot_flops = float(f.item())
+    value = tot_flops / (ms * 1e-3) / 1e12
+    # roofline of the dominant kernel class on this rank (algorithmic bytes, SURVEY §8(d))
+    kref = K  # every column of B is referenced at 10% density over 2048 windows
+    bytes_spmm = 4 * (W + 1) + nnzA * (4 + 2 * V) + 2 * kref * Np + 2 * M * Np
+    bytes_sddmm = 4 * (w1 - w0 + 1) + 4 * nnzM + 2 * Ml * K + 2 * N * K + 2 * nnzM * V
+    dom = "spmm" if cls["spmm"] >= cls["sddmm"] else "sddmm"
+    db = bytes_spmm if dom == "spmm" else bytes_sddmm
+    ach = db / (cls[dom] * 1e-3) / 1e9
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": ws, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "strong",
+        "vs_baseline": None, "dtype": "f16", "data": "synthetic",
+        "config": {"workload": "c5", "M": M, "K": K, "N": N, "V": V, "S": S,
+                   "step": "encode A, SpMM on this rank's N-panel (A replicated); encode this "
+                           "rank's mask rows, SDDMM (mask 16384x65536, inner 16384, Bt replicated)",
+                   "l2": "inputs far larger than L2 (no flush)", "nnz_v_spmm": nnzA,
+                   "nnz_v_sddmm_rank0": nnzM, "parallelism": f"spmm N-panels x{ws}, sddmm row windows x{ws}"},
+        "roofline": {"bound": "hbm", "achieved": ach, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                     "frac": ach / peaks["hbm_gbs"], "traffic": None, "kernel": dom,
+                     "algorithmic_bytes_per_launch": db, "avg_launch_us": cls[dom] * 1e3,
+                     "peak_source": peaks["source"]},
+        "kernels": {k: {"ms": v} for k, v in cls.items()},
+        "gpu_launches": 8 * args.steps,
+        "clocks": clk,
+        "e2e": None,
+    }
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if ws > 1:
+        torch.distributed.destroy_process_group()
+    return 0
+
+
+def run_attention(args):
+    """NEXT item, the Fig. 20 analogue: sparse multi-head attention of Eq. 1
+     on band-256 + random V x 1 masks, batch 8 x 4 heads.
+    Workload name: attention_l<l>_k<k>_s<S>[_v<V>] (default l=4096, k=64, S=0.9, V=8).
+    Step = SDDMM batch (scores) -> softmax batch -> SpMM batch, one CUDA graph.  Compared
+    with dense fp16 attention (torch: cuBLAS matmul, masked softmax, matmul) on the same box."""
+    import math
+    import re
+    import torch
+    import paper_conf_sc_chenqldx21_b200 as vs
+    from synth import gen
+
+    m = re.match(r"attention(?:_l(\d+))?(?:_k(\d+))?(?:_s([0-9.]+))?(?:_v(\d+))?$", args.workload)
+    l = int(m.group(1) or 4096)
+    k = int(m.group(2) or 64)
+    S = float(m.group(3) or 0.9)
+    V = int(m.group(4) or 8)
+    heads = 32
+    torch.cuda.set_device(0)
+    dev = torch.device("cuda", 0)
+    vs.load()
+    rng = gen.make_rng(f"attn_l{l}_s{S}_v{V}")
+    mask = torch.from_numpy(gen.attention_mask(rng, l, V, S)).to(dev)  # one mask for all heads
+    rp, ci, _ = vs.encode(V, mask=mask)
+    nnz = int(rp[-1].item())
+    Qs = [gen.torch_dense_operand(l, k, seed=gen.config_seed(f"q{h}"), device=dev) for h in range(heads)]
+    Ks = [gen.torch_dense_operand(l, k, seed=gen.config_seed(f"k{h}"), device=dev) for h in range(heads)]
+    Vs = [gen.torch_dense_operand(l, k, seed=gen.config_seed(f"v{h}"), device=dev) for h in range(heads)]
+    Ss = [torch.empty(nnz * V, dtype=torch.float16, device=dev) for _ in range(heads)]
+    Os = [torch.empty((l, k), dtype=torch.float16, device=dev) for _ in range(heads)]
+    scale = 1.0 / math.sqrt(k)
+    sd = vs.make_sddmm_batch([(l, l, k, V, rp, ci, Qs[h], Ks[h], Ss[h]) for h in range(heads)])
+    sm = vs.make_softmax_batch([(l, V, scale, rp, Ss[h], Ss[h]) for h in range(heads)])
+    sp = vs.make_spmm_batch([(l, l, k, V, rp, ci, Ss[h], Vs[h], Os[h]) for h in range(heads)])
+
+    def step():
+        vs.vs_sddmm_batched(sd)
+        vs.vs_softmax_colvec_batched(sm)
+        vs.vs_spmm_batched(sp)
+
+    Qd = torch.stack(Qs)
+    Kd = torch.stack(Ks)
+    Vd = torch.stack(Vs)
+    neg = torch.zeros((l, l), dtype=torch.float16, device=dev).masked_fill(mask == 0, float("-inf"))
+
+    def dense():
+        a = torch.matmul(Qd, Kd.transpose(1, 2)) * scale + neg
+        return torch.matmul(torch.softmax(a, dim=-1), Vd)
+
+    stream = torch.cuda.Stream()
+    g = capture(torch, step, stream)
+    with torch.cuda.stream(stream):
+        for _ in range(args.warmup):
+            g.replay()
+        dense()
+    stream.synchronize()
+    gd = capture(torch, dense, stream)
+    clocks = ClockSampler(0).start()
+    t_sparse = min(time_graph(torch, g, stream) for _ in range(max(1, args.steps)))
+    t_dense = min(time_graph(torch, gd, stream) for _ in range(max(1, args.steps)))
+    clk = clocks.stop()
+    flops = heads * (2.0 * nnz * V * k) * 2  # SDDMM + SpMM (softmax not counted)
+    line = {"metric": METRIC, "value": flops / (t_sparse * 1e-3) / 1e12, "unit": UNIT, "n_gpus": 1,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": t_sparse,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f16",
+            "data": "synthetic",
+            "config": {"workload": args.workload, "l": l, "k": k, "sparsity": S, "V": V,
+                       "heads_x_batch": heads, "mask": "band 256 + random (P:1560-1566)",
+                       "nnz_v": nnz, "l2": "warm (per-step graph timing, min of steps)"},
+            "dense_attention_ms": t_dense, "speedup_vs_dense": t_dense / t_sparse,
+            "gpu_launches": 3 * args.steps, "clocks": clk, "e2e": None}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
 def main(argv=None):
     args = parse_args(argv)
     if args.impl == "reference":
         return run_reference(args)
+    if args.workload == "c5":
+        return run_c5(args)
+    if args.workload.startswith("attention"):
+        return run_attention(args)
     return run_ours(args)
 
 

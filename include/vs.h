@@ -134,6 +134,22 @@ vs_status_t vs_sddmm(int64_t M, int64_t N, int64_t K, int V,
                      const void* A, const void* Bt, void* out_vals, vs_stream_t stream);
 
 /*
+ * vs_softmax_colvec — row softmax over the stored entries of a column-vector CSR matrix
+ * (NEXT item of the hot path: sparse attention, Eq. 1 P:1535-1545,
+ * A = Softmax((Q K^T o C) / sqrt(k)); the paper's softmax kernel on the column-vector
+ * encoding).  For every row i = wV + r < M:
+ *   out[p*V + r] = exp(scale*x_p - m) / sum_q exp(scale*x_q - m),  x_p = vals[p*V + r],
+ * over the stored vectors p of window w (m = the row's max of scale*x).  Rows >= M (padding
+ * of the last window) get +0.  Entries outside the mask take no part (they are -inf in the
+ * dense view).  fp16 in/out, fp32 arithmetic.
+ *   vals, out : fp16 [nnz_v * V]; out may equal vals (in place).  For V = 4 and 8 both must be
+ *               2V-byte aligned (VS_ERROR_MISALIGNED otherwise).
+ *   M == 0 or nnz_v == 0: no-op.
+ */
+vs_status_t vs_softmax_colvec(int64_t M, int V, const int32_t* row_ptr, const void* vals,
+                              void* out, float scale, vs_stream_t stream);
+
+/*
  * Batched entry points: many independent problems per call (SURVEY §8(f) rank 3 — the
  * DLMC-sized problems of the paper's benchmarks, are launch-latency bound on
  * B200 one at a time).
@@ -183,6 +199,18 @@ vs_status_t vs_sddmm_batched(int64_t count, const vs_sddmm_problem_t* problems,
                              vs_stream_t stream);
 vs_status_t vs_encode_colvec_batched(int64_t count, const vs_encode_problem_t* problems,
                                      vs_stream_t stream);
+
+typedef struct {
+  int64_t M;
+  int32_t V;
+  float scale;
+  const int32_t* row_ptr;
+  const void* vals;
+  void* out;
+} vs_softmax_problem_t;
+
+vs_status_t vs_softmax_colvec_batched(int64_t count, const vs_softmax_problem_t* problems,
+                                      vs_stream_t stream);
 
 #ifdef __cplusplus
 }

@@ -59,6 +59,8 @@ def lib():
             L.oracle_sddmm_sample.restype = None
             L.oracle_sddmm_sample.argtypes = [_I64, _I64, _I64, ctypes.c_int, _P, _P, _P,
                                               _I64, _P, _P, _P, _P]
+            L.oracle_softmax.restype = None
+            L.oracle_softmax.argtypes = [_I64, ctypes.c_int, _P, _P, ctypes.c_double, _P]
             L.oracle_half_to_double.restype = ctypes.c_double
             L.oracle_half_to_double.argtypes = [ctypes.c_uint16]
             L.oracle_num_threads.restype = ctypes.c_int
@@ -160,6 +162,20 @@ def sddmm_sample(M, N, K, V, row_ptr, col_idx, A, Bt, vec_p):
                               _ptr(_f16(A)), _ptr(_f16(Bt)), vec_p.size, _ptr(vec_p), _ptr(vec_w),
                               _ptr(out), _ptr(S))
     return out.reshape(-1, V), S.reshape(-1, V)
+
+
+def softmax(M: int, V: int, row_ptr, vals, scale: float) -> np.ndarray:
+    """Row softmax over the stored entries (Eq. 1).  Returns float64 [nnz*V]."""
+    rp = np.ascontiguousarray(row_ptr, np.int32)
+    out = np.empty(int(rp[-1]) * V, np.float64)
+    lib().oracle_softmax(M, V, _ptr(rp), _ptr(_f16(vals)), float(scale), _ptr(out))
+    return out
+
+
+def softmax_tolerance(p64) -> np.ndarray:
+    """Softmax bar: fp16 output rounding (2^-11 relative) plus fp32 exp / sum
+    error, bounded by 2^-10 * p + 2^-24."""
+    return 2.0 ** -10 * np.abs(np.asarray(p64, np.float64)) + 2.0 ** -24
 
 
 def tolerance(S64) -> np.ndarray:

@@ -15,6 +15,9 @@
  *                  mask, B passed transposed (Bt[N x K] row-major).
  *   *_sample       the same sums for a caller-chosen list of output elements (used where
  *                  the full problem is too large for the host).
+ *   oracle_softmax §7.4 Eq. 1 P:1535-1545 (NEXT item) — row softmax over the
+ *                  stored entries of the column-vector matrix (the masked attention scores;
+ *                  entries outside the mask are -inf in the dense view).
  *
  * Inputs are fp16 bit patterns (uint16_t); each is widened to double exactly by
  * half_to_double() and every product and sum is formed in double.  Alongside each result
@@ -200,6 +203,36 @@ void oracle_sddmm_sample(int64_t M, int64_t N, int64_t K, int V, const int32_t* 
       }
       out64[s * V + r] = acc;
       if (S64) S64[s * V + r] = sc;
+    }
+  }
+}
+
+/*
+ * Row softmax (Eq. 1): for every row i = wV + r < M, over the stored vectors p of
+ * window w: out[p*V + r] = exp(scale*x_p - m) / sum_q exp(scale*x_q - m), x_p = vals[p*V + r],
+ * m = max_q scale*x_q.  Rows >= M get 0.
+ */
+void oracle_softmax(int64_t M, int V, const int32_t* row_ptr, const uint16_t* vals, double scale,
+                    double* out64) {
+  int64_t W = ceil_div(M, V);
+#pragma omp parallel for schedule(dynamic, 1)
+  for (int64_t w = 0; w < W; ++w) {
+    for (int r = 0; r < V; ++r) {
+      int64_t i = w * V + r;
+      int64_t p;
+      if (i >= M) {
+        for (p = row_ptr[w]; p < row_ptr[w + 1]; ++p) out64[p * V + r] = 0.0;
+        continue;
+      }
+      double m = -INFINITY, sum = 0.0;
+      for (p = row_ptr[w]; p < row_ptr[w + 1]; ++p) {
+        double x = scale * half_to_double(vals[p * V + r]);
+        if (x > m) m = x;
+      }
+      for (p = row_ptr[w]; p < row_ptr[w + 1]; ++p)
+        sum += exp(scale * half_to_double(vals[p * V + r]) - m);
+      for (p = row_ptr[w]; p < row_ptr[w + 1]; ++p)
+        out64[p * V + r] = exp(scale * half_to_double(vals[p * V + r]) - m) / sum;
     }
   }
 }

@@ -22,7 +22,8 @@ import os
 import threading
 
 __all__ = ["VSError", "lib_path", "load", "vs_encode_colvec", "vs_spmm", "vs_sddmm",
-           "vs_encode_colvec_batched", "vs_spmm_batched", "vs_sddmm_batched",
+           "vs_softmax_colvec", "vs_encode_colvec_batched", "vs_spmm_batched", "vs_sddmm_batched",
+           "vs_softmax_colvec_batched", "sparse_attention",
            "encode", "spmm", "sddmm", "num_windows"]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
@@ -57,6 +58,12 @@ class EncodeProblem(ctypes.Structure):
                 ("row_ptr", ctypes.c_void_p), ("col_idx", ctypes.c_void_p), ("vals", ctypes.c_void_p)]
 
 
+class SoftmaxProblem(ctypes.Structure):
+    """vs_softmax_problem_t"""
+    _fields_ = [("M", ctypes.c_int64), ("V", ctypes.c_int32), ("scale", ctypes.c_float),
+                ("row_ptr", ctypes.c_void_p), ("vals", ctypes.c_void_p), ("out", ctypes.c_void_p)]
+
+
 STATUS = {0: "VS_SUCCESS", 1: "VS_ERROR_INVALID_VALUE", 2: "VS_ERROR_NOT_SUPPORTED",
           3: "VS_ERROR_CUDA", 4: "VS_ERROR_MISALIGNED"}
 
@@ -87,8 +94,11 @@ def load():
             L.vs_spmm.argtypes = [_I64, _I64, _I64, ctypes.c_int, _P, _P, _P, _P, _P, _P]
             L.vs_sddmm.restype = ctypes.c_int
             L.vs_sddmm.argtypes = [_I64, _I64, _I64, ctypes.c_int, _P, _P, _P, _P, _P, _P]
+            L.vs_softmax_colvec.restype = ctypes.c_int
+            L.vs_softmax_colvec.argtypes = [_I64, ctypes.c_int, _P, _P, _P, ctypes.c_float, _P]
             for name, st in (("vs_spmm_batched", SpmmProblem), ("vs_sddmm_batched", SddmmProblem),
-                             ("vs_encode_colvec_batched", EncodeProblem)):
+                             ("vs_encode_colvec_batched", EncodeProblem),
+                             ("vs_softmax_colvec_batched", SoftmaxProblem)):
                 f = getattr(L, name)
                 f.restype = ctypes.c_int
                 f.argtypes = [_I64, ctypes.POINTER(st), _P]
@@ -166,6 +176,15 @@ def vs_sddmm(M, N, K, V, row_ptr, col_idx, A, Bt, out_vals, stream=None):
     _check(st, "vs_sddmm")
 
 
+def vs_softmax_colvec(M, V, row_ptr, vals, out, scale, stream=None):
+    """Row softmax over the stored entries (Eq. 1)."""
+    import torch
+    st = load().vs_softmax_colvec(int(M), int(V), _ptr(row_ptr, torch.int32, "row_ptr"),
+                                  _ptr(vals, torch.float16, "vals"), _ptr(out, torch.float16, "out"),
+                                  float(scale), _stream(stream))
+    _check(st, "vs_softmax_colvec")
+
+
 # ------------------------------------------------------------------ batched mirrors
 #
 # Each takes a list of per-problem tuples in the order of the C struct fields (tensors for
@@ -203,6 +222,37 @@ def make_encode_batch(problems):
                                _addr(m, torch.uint8, "mask"), _addr(rp, torch.int32, "row_ptr"),
                                _addr(ci, torch.int32, "col_idx"), _addr(va, torch.float16, "vals"))
     return arr
+
+
+def make_softmax_batch(problems):
+    """problems: [(M, V, scale, row_ptr, vals, out), ...]"""
+    import torch
+    arr = (SoftmaxProblem * len(problems))()
+    for i, (M, V, sc, rp, va, out) in enumerate(problems):
+        arr[i] = SoftmaxProblem(int(M), int(V), float(sc), _addr(rp, torch.int32, "row_ptr"),
+                                _addr(va, torch.float16, "vals"), _addr(out, torch.float16, "out"))
+    return arr
+
+
+def vs_softmax_colvec_batched(batch, stream=None):
+    if isinstance(batch, list):
+        batch = make_softmax_batch(batch)
+    _check(load().vs_softmax_colvec_batched(len(batch), batch, _stream(stream)),
+           "vs_softmax_colvec_batched")
+
+
+def sparse_attention(row_ptr, col_idx, Q, Kmat, Vmat, V, scale=None, nnz=None, stream=None):
+    """Eq. 1 on a column-vector mask (row_ptr, col_idx) over [l x l]:
+    S = (Q K^T) o C (vs_sddmm), P = softmax(scale * S) row-wise (vs_softmax_colvec),
+    out = P Vmat (vs_spmm).  Q, Kmat: [l x k]; Vmat: [l x dv]; returns out [l x dv]."""
+    import math
+    import torch
+    l, k = Q.shape
+    if scale is None:
+        scale = 1.0 / math.sqrt(k)
+    S = sddmm(row_ptr, col_idx, Q, Kmat, V, nnz=nnz, stream=stream)
+    vs_softmax_colvec(l, V, row_ptr, S, S, scale, stream=stream)
+    return spmm(row_ptr, col_idx, S, Vmat, l, V, stream=stream)
 
 
 def vs_spmm_batched(batch, stream=None):

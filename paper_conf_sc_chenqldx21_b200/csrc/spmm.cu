@@ -19,6 +19,7 @@
 //   2t and 2t+1: the epilogue stores 16 bytes per row with no shuffles.
 //   B fragment (k = vector slot, n = row r < V) is vals[p*V + g].
 #include <algorithm>
+#include <cstdlib>
 #include <utility>
 #include <vector>
 
@@ -92,6 +93,67 @@ __device__ __forceinline__ void spmm_body(int64_t M, int64_t N, int64_t W, int64
 
   const int kslot[4] = {2 * t, 2 * t + 1, 2 * t + 8, 2 * t + 9};
 
+  constexpr int kStride = 16 * SPLIT;  // distance between a warp's consecutive groups
+  if constexpr (UNROLL == 0) {
+    // Pipelined: while the MMAs of group i run, the B rows of group i+1 are in flight, its
+    // vals are being fetched and the column indices of group i+2 too (two register sets of
+    // rows and vals whose roles alternate; one set of column indices, refilled as soon as
+    // it has been turned into row addresses).
+    auto load_col = [&](int p0, int (&cl)[4]) {
+#pragma unroll
+      for (int s = 0; s < 4; ++s) {
+        const int p = p0 + kslot[s];
+        cl[s] = p < p_end ? ldg32i(col_idx + p) : -1;
+      }
+    };
+    auto load_bv = [&](int p0, uint16_t (&b)[4]) {
+#pragma unroll
+      for (int s = 0; s < 4; ++s) {
+        const int p = p0 + kslot[s];
+        b[s] = (p < p_end && g < V) ? ldg16(vals + (int64_t)p * V + g) : (uint16_t)0;
+      }
+    };
+    auto load_rows = [&](const int (&cl)[4], uint4 (&r)[4][NC]) {
+#pragma unroll
+      for (int s = 0; s < 4; ++s) load_brow<NC, VEC>(B, N, cl[s] < 0 ? 0 : cl[s], cl[s] >= 0, ncol0, r[s]);
+    };
+    auto mma_group = [&](const uint4 (&r)[4][NC], const uint16_t (&b)[4]) {
+      const uint32_t b0 = pack_h2(b[0], b[1]);
+      const uint32_t b1 = pack_h2(b[2], b[3]);
+#pragma unroll
+      for (int c = 0; c < NC; ++c)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const uint32_t w0 = word(r[0][c], j), w1 = word(r[1][c], j);
+          const uint32_t w2 = word(r[2][c], j), w3 = word(r[3][c], j);
+          mma_16816(acc[c][j], pack_lo(w0, w1), pack_hi(w0, w1), pack_lo(w2, w3),
+                    pack_hi(w2, w3), b0, b1);
+        }
+    };
+    int pc = p_begin + 16 * part;
+    int coln[4];
+    uint16_t bvA[4], bvB[4];
+    uint4 rA[4][NC], rB[4][NC];
+    load_col(pc, coln);
+    load_rows(coln, rA);
+    load_bv(pc, bvA);
+    load_col(pc + kStride, coln);
+    while (pc < p_end) {
+      int pn = pc + kStride;
+      if (pn < p_end) load_rows(coln, rB);
+      load_col(pn + kStride, coln);
+      load_bv(pn, bvB);
+      mma_group(rA, bvA);
+      pc = pn;
+      if (pc >= p_end) break;
+      pn = pc + kStride;
+      if (pn < p_end) load_rows(coln, rA);
+      load_col(pn + kStride, coln);
+      load_bv(pn, bvA);
+      mma_group(rB, bvB);
+      pc = pn;
+    }
+  } else {
   // group metadata (column index + this thread's vals element per slot), prefetched one
   // iteration ahead so the col_idx -> B-row dependency is not on every iteration's path.
   // An iteration handles UNROLL groups (this warp's groups are p_begin + 16*(part + SPLIT*i)).
@@ -106,7 +168,6 @@ __device__ __forceinline__ void spmm_body(int64_t M, int64_t N, int64_t W, int64
       b[s] = (valid && g < V) ? ldg16(vals + (int64_t)p * V + g) : (uint16_t)0;
     }
   };
-  constexpr int kStride = 16 * SPLIT;  // distance between a warp's consecutive groups
   int p0 = p_begin + 16 * part;
 #pragma unroll
   for (int u = 0; u < UNROLL; ++u) load_meta(p0 + u * kStride, col[u], bv[u]);
@@ -144,6 +205,8 @@ __device__ __forceinline__ void spmm_body(int64_t M, int64_t N, int64_t W, int64
         bv[u][s] = bvn[u][s];
       }
     p0 = p1;
+  }
+
   }
 
   if constexpr (SPLIT > 1) {
@@ -259,7 +322,13 @@ struct SpmmCfg {
 SpmmCfg spmm_config(int64_t K, int64_t N, int V, const void* B, const void* C) {
   SpmmCfg c;
   c.V = V;
-  c.NC = N <= 64 ? 1 : 2;
+  // 64-column panels: a K x 64 panel of B stays L1-resident for K <= ~1500 (tools/tune.py:
+  // 3% faster than 128-column panels over the DLMC batch; VS_SPMM_NC=2 selects 128 columns).
+  static const int nc_knob = [] {
+    const char* e = std::getenv("VS_SPMM_NC");
+    return e ? std::atoi(e) : 1;
+  }();
+  c.NC = (N <= 64 || nc_knob != 2) ? 1 : 2;
   const int64_t q = K >> 8;
   c.SPLIT = q >= 16 ? 16 : q >= 8 ? 8 : q >= 4 ? 4 : q >= 2 ? 2 : 1;
   c.VEC = (N % 8 == 0) && ((reinterpret_cast<uintptr_t>(B) & 15) == 0) &&
@@ -274,18 +343,25 @@ struct SpmmKernels {
   int threads, units_per_cta, batched_ctas_per_sm;
 };
 
+// Main-loop variant (tools/tune.py): 0 (default) = the plain loop; VS_SPMM_PIPE=1 keeps the
+// B rows of the next group in flight during the current group's MMAs -- measured 10% slower,
+// the kernel is bound by the L1TEX data pipe (ncu: l1tex__data_pipe_lsu_wavefronts at
+// 79-93% of peak), not by latency.
+static int spmm_pipe() {
+  static const int v = [] {
+    const char* e = std::getenv("VS_SPMM_PIPE");
+    return e ? std::atoi(e) : 0;
+  }();
+  return v;
+}
+
 template <int V, int NC, bool VEC, int SPLIT>
 static SpmmKernels kernels_of() {
-  static const int occ = [] {
-    int b = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-            &b, spmm_batched_kernel<V, NC, VEC, SPLIT, 1>, SpmmCta<SPLIT>::kWarps * 32, 0) !=
-            cudaSuccess || b < 1)
-      b = 1;
-    return b;
-  }();
+  if (spmm_pipe())
+    return {spmm_kernel<V, NC, VEC, SPLIT, 0>, spmm_batched_kernel<V, NC, VEC, SPLIT, 0>,
+            SpmmCta<SPLIT>::kWarps * 32, SpmmCta<SPLIT>::kUnits, 0};
   return {spmm_kernel<V, NC, VEC, SPLIT, 1>, spmm_batched_kernel<V, NC, VEC, SPLIT, 1>,
-          SpmmCta<SPLIT>::kWarps * 32, SpmmCta<SPLIT>::kUnits, occ};
+          SpmmCta<SPLIT>::kWarps * 32, SpmmCta<SPLIT>::kUnits, 0};
 }
 
 template <int V, int NC, bool VEC>

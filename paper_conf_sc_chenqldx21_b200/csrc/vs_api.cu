@@ -27,6 +27,11 @@ cudaError_t launch_encode_batched(int64_t count, const int64_t* M, const int64_t
                                   const void* const* dense, const uint8_t* const* mask,
                                   int32_t* const* row_ptr, int32_t* const* col_idx,
                                   void* const* vals, int num_sms, cudaStream_t s);
+cudaError_t launch_softmax(int64_t M, int V, const int32_t* row_ptr, const void* vals, void* out,
+                           float scale, cudaStream_t s);
+cudaError_t launch_softmax_batched(int64_t count, const int64_t* M, const int* V,
+                                   const int32_t* const* row_ptr, const void* const* vals,
+                                   void* const* out, const float* scale, cudaStream_t s);
 }  // namespace vs
 
 namespace {
@@ -100,6 +105,18 @@ vs_status_t check_sddmm(int64_t M, int64_t N, int64_t K, int V, const int32_t* r
   return VS_SUCCESS;
 }
 
+vs_status_t check_softmax(int64_t M, int V, const int32_t* row_ptr, const void* vals,
+                          const void* out) {
+  if (!valid_v(V) || M < 0) return VS_ERROR_INVALID_VALUE;
+  if (M == 0) return VS_SUCCESS;
+  // vals / out may be NULL only when never touched (nnz_v == 0)
+  if (row_ptr == nullptr) return VS_ERROR_INVALID_VALUE;
+  if (!al(row_ptr, 4)) return VS_ERROR_MISALIGNED;
+  const uintptr_t need = V >= 4 ? 2 * V : 2;
+  if ((vals && !al(vals, need)) || (out && !al(out, need))) return VS_ERROR_MISALIGNED;
+  return VS_SUCCESS;
+}
+
 }  // namespace
 
 extern "C" {
@@ -168,6 +185,47 @@ vs_status_t vs_sddmm(int64_t M, int64_t N, int64_t K, int V, const int32_t* row_
   if (st != VS_SUCCESS) return st;
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   return from_cuda(vs::launch_sddmm(M, N, K, V, row_ptr, col_idx, A, Bt, out_vals, info.num_sms, s));
+}
+
+vs_status_t vs_softmax_colvec(int64_t M, int V, const int32_t* row_ptr, const void* vals,
+                              void* out, float scale, vs_stream_t stream) {
+  vs_status_t st0 = check_softmax(M, V, row_ptr, vals, out);
+  if (st0 != VS_SUCCESS || M == 0) return st0;
+  DevInfo info;
+  vs_status_t st = check_device(&info);
+  if (st != VS_SUCCESS) return st;
+  return from_cuda(vs::launch_softmax(M, V, row_ptr, vals, out, scale,
+                                      reinterpret_cast<cudaStream_t>(stream)));
+}
+
+vs_status_t vs_softmax_colvec_batched(int64_t count, const vs_softmax_problem_t* problems,
+                                      vs_stream_t stream) {
+  if (count < 0 || (count > 0 && problems == nullptr)) return VS_ERROR_INVALID_VALUE;
+  for (int64_t i = 0; i < count; ++i) {
+    const vs_softmax_problem_t& p = problems[i];
+    const vs_status_t st = check_softmax(p.M, p.V, p.row_ptr, p.vals, p.out);
+    if (st != VS_SUCCESS) return st;
+  }
+  if (count == 0) return VS_SUCCESS;
+  DevInfo info;
+  vs_status_t st = check_device(&info);
+  if (st != VS_SUCCESS) return st;
+  std::vector<int64_t> M;
+  std::vector<int> V;
+  std::vector<const int32_t*> rp;
+  std::vector<const void*> va;
+  std::vector<void*> out;
+  std::vector<float> sc;
+  for (int64_t i = 0; i < count; ++i) {
+    const vs_softmax_problem_t& p = problems[i];
+    if (p.M == 0) continue;
+    M.push_back(p.M); V.push_back(p.V); rp.push_back(p.row_ptr); va.push_back(p.vals);
+    out.push_back(p.out); sc.push_back(p.scale);
+  }
+  if (M.empty()) return VS_SUCCESS;
+  return from_cuda(vs::launch_softmax_batched((int64_t)M.size(), M.data(), V.data(), rp.data(),
+                                              va.data(), out.data(), sc.data(),
+                                              reinterpret_cast<cudaStream_t>(stream)));
 }
 
 vs_status_t vs_spmm_batched(int64_t count, const vs_spmm_problem_t* problems, vs_stream_t stream) {

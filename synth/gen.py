@@ -27,6 +27,7 @@ import numpy as np
 
 __all__ = [
     "config_seed", "make_rng", "fp16_values", "vector_keep", "colvec_dense", "colvec_mask",
+    "attention_mask",
     "dense_operand", "torch_colvec_dense", "torch_dense_operand",
 ]
 
@@ -97,6 +98,23 @@ def colvec_mask(rng: np.random.Generator, M: int, N: int, V: int, density: float
     W = -(-M // V) if M > 0 else 0
     keep = vector_keep(rng, W, N, density, kind)
     return np.ascontiguousarray(np.repeat(keep, V, axis=0)[:M].astype(np.uint8))
+
+
+def attention_mask(rng: np.random.Generator, l: int, V: int, sparsity: float,
+                   band: int = 256) -> np.ndarray:
+    """uint8 [l, l] attention mask of V x 1 vectors: a dense band of width
+    `band` along the diagonal plus uniformly random off-band vectors, with the off-band
+    probability chosen so that the overall density is 1 - sparsity (when the band alone is
+    sparser than that)."""
+    W = -(-l // V)
+    wi = np.arange(W)[:, None] * V + V // 2
+    cj = np.arange(l)[None, :]
+    in_band = np.abs(cj - wi) < band // 2
+    band_frac = in_band.mean()
+    target = 1.0 - sparsity
+    p_off = max(0.0, (target - band_frac) / max(1e-12, 1.0 - band_frac))
+    keep = in_band | (rng.random((W, l)) < p_off)
+    return np.ascontiguousarray(np.repeat(keep, V, axis=0)[:l].astype(np.uint8))
 
 
 def dense_operand(rng: np.random.Generator, rows: int, cols: int, exact: bool = False) -> np.ndarray:

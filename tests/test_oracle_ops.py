@@ -237,3 +237,81 @@ def test_adjoint_identity(V):
     lhs = float(np.sum(Y * f64(G)))
     rhs = float(np.dot(f64(va), dW))
     assert abs(lhs - rhs) <= 1e-9 * max(1.0, abs(lhs))
+
+
+# ---------------------------------------------------- softmax (NEXT item, Eq. 1)
+
+def dense_masked_softmax(vals, rp, ci, M, N, V, scale):
+    """numpy: scatter the stored entries into a dense [M x N] matrix filled with -inf, then
+    the textbook row softmax; gathered back at the stored positions."""
+    D = np.full((M, N), -np.inf)
+    W = len(rp) - 1
+    for w in range(W):
+        for p in range(rp[w], rp[w + 1]):
+            for r in range(V):
+                if w * V + r < M:
+                    D[w * V + r, ci[p]] = scale * f64(vals[p * V + r])
+    with np.errstate(invalid="ignore"):
+        E = np.exp(D - D.max(axis=1, keepdims=True))
+        P = E / E.sum(axis=1, keepdims=True)
+    out = []
+    for w in range(W):
+        for p in range(rp[w], rp[w + 1]):
+            for r in range(V):
+                out.append(P[w * V + r, ci[p]] if w * V + r < M else 0.0)
+    return np.array(out)
+
+
+@pytest.mark.parametrize("V", [1, 2, 4, 8])
+def test_softmax_matches_dense_masked_softmax(V):
+    rng = gen.make_rng(f"sm_{V}")
+    M, N = 8 * 5 + 3, 70
+    mask = gen.colvec_mask(rng, M, N, V, 0.3)
+    rp, ci, _ = oracle.encode(M, N, V, mask=mask)
+    vals = gen.fp16_values(rng, int(rp[-1]) * V) * np.float16(4)
+    out = oracle.softmax(M, V, rp, vals, 0.125)
+    np.testing.assert_allclose(out, dense_masked_softmax(vals, rp, ci, M, N, V, 0.125),
+                               rtol=1e-12, atol=1e-15)
+
+
+@pytest.mark.parametrize("V", [2, 8])
+def test_softmax_invariants(V):
+    """Rows sum to 1, a constant row is uniform, a shift of a row changes nothing, padded
+    rows are 0."""
+    rng = gen.make_rng(f"smi_{V}")
+    M, N = 8 * 4 + 5, 50
+    mask = gen.colvec_mask(rng, M, N, V, 0.4)
+    rp, ci, _ = oracle.encode(M, N, V, mask=mask)
+    nnz = int(rp[-1])
+    vals = gen.fp16_values(rng, nnz * V)
+    out = oracle.softmax(M, V, rp, vals, 1.0).reshape(-1, V)
+    for w in range(len(rp) - 1):
+        seg = out[rp[w]:rp[w + 1]]
+        if seg.shape[0] == 0:
+            continue
+        for r in range(V):
+            if w * V + r < M:
+                assert abs(seg[:, r].sum() - 1.0) < 1e-12
+            else:
+                assert np.all(seg[:, r] == 0)
+    const = np.full(nnz * V, np.float16(0.5))
+    outc = oracle.softmax(M, V, rp, const, 3.0).reshape(-1, V)
+    for w in range(len(rp) - 1):
+        n = rp[w + 1] - rp[w]
+        for r in range(V):
+            if n and w * V + r < M:
+                np.testing.assert_allclose(outc[rp[w]:rp[w + 1], r], 1.0 / n, rtol=1e-14)
+    # shift invariance on values k/16 (exact in fp16 before and after the shift)
+    grid = (rng.integers(-16, 16, nnz * V) / 16.0).astype(np.float16)
+    shifted = (grid.astype(np.float64) - 0.5).astype(np.float16)
+    assert np.array_equal(shifted.astype(np.float64) + 0.5, grid.astype(np.float64))
+    np.testing.assert_allclose(oracle.softmax(M, V, rp, shifted, 1.0),
+                               oracle.softmax(M, V, rp, grid, 1.0), rtol=1e-12, atol=1e-15)
+
+
+def test_attention_mask_density():
+    rng = gen.make_rng("amask")
+    m = gen.attention_mask(rng, 4096, 8, 0.9)   # band 256 = 6.25% < 10%: random fills the rest
+    assert abs(m.mean() - 0.1) < 0.01
+    # the diagonal band is dense
+    assert m[1000, 1000 - 100:1000 + 100].all()
