@@ -171,8 +171,7 @@ def alg_bytes(p, nnz_v, k_ref):
 
 def count_launches(bufs):
     """Kernel launches of one batched step, by the library's grouping rules (vs_api.cu):
-    encode groups by V (4 kernels per group of <= 128 problems: zero row_ptr, count, scan,
-    compact), SpMM by (V, panel width NC from N, SPLIT from K), SDDMM by V (1 kernel per
+    encode groups by V (3 kernels per group of <= 128 problems: count, scan, compact), SpMM by (V, panel width NC from N, SPLIT from K), SDDMM by V (1 kernel per
     group of <= 128)."""
     import math as _m
     from collections import Counter
@@ -182,7 +181,7 @@ def count_launches(bufs):
     enc = Counter(b.p.V for b in bufs)
     sp = Counter((b.p.V, 1, split(b.p.K)) for b in bufs)  # 64-column panels (NC = 1)
     sd = Counter(b.p.V for b in bufs)
-    per = {"encode": sum(4 * _m.ceil(n / 128) for n in enc.values()),
+    per = {"encode": sum(3 * _m.ceil(n / 128) for n in enc.values()),
            "spmm": sum(_m.ceil(n / 128) for n in sp.values()),
            "sddmm": sum(_m.ceil(n / 128) for n in sd.values())}
     return {"per_class": per, "total": sum(per.values())}

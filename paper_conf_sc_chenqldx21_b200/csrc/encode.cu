@@ -1,13 +1,12 @@
 // encode.cu — dense fp16 matrix / uint8 mask -> column-vector CSR (§4.2, Fig. 8).
 //
-// Three kernels (+ one memset node), count and compact with one CTA per row window and one
-// warp per 256-column chunk (up to 8 warps); each lane tests 8 consecutive columns with one
-// 16-byte load per row of the window.  Keep bit = any nonzero fp16 bit pattern (or mask
-// byte) over the window's V rows.
-//   1. encode_count   : each warp adds its chunk's count to row_ptr[w+1] (zeroed by the
-//      memset) with one reduction atomic: no barrier, no waiting, order-independent.
-//   2. encode_scan    : one CTA turns the counts into the inclusive prefix in place.
-//   3. encode_compact : re-reads the window (L2-resident), block-scans the lanes' keep counts
+// Three kernels, count and compact with one warp per row window (4 windows per CTA); each
+// lane tests 8 consecutive columns per 256-column step with one 16-byte load per row of the
+// window.  Keep bit = any nonzero fp16 bit pattern (or mask byte) over the window's V rows.
+//   1. encode_count   : the warp's popcount total goes to row_ptr[w+1].
+//   2. encode_scan    : one CTA turns the counts into the inclusive prefix in place and sets
+//                       row_ptr[0] = 0.
+//   3. encode_compact : re-reads the window (L2-resident), warp-scans the lanes' keep counts
 //      and writes col_idx and the V values of each kept vector (transposed from the V row
 //      loads into vector-major order) starting at row_ptr[w].
 // Columns are visited in ascending order, so col_idx ascends inside each window (Fig. 8).
@@ -19,7 +18,7 @@
 
 namespace vs {
 
-constexpr int kEncMaxThreads = 256;              // threads per CTA (one CTA per window)
+constexpr int kEncWarps = 4;                     // windows (warps) per CTA
 constexpr int kColsPerLane = 8;                  // columns per lane per step
 constexpr int kColsPerStep = kColsPerLane * 32;  // 256 columns per warp step
 
@@ -142,29 +141,29 @@ __device__ void block_scan_inplace(int32_t* a, int64_t n, int32_t* s_warp, int32
   }
 }
 
-// Phase 1: each warp counts the kept vectors of its 256-column chunks of window w and adds
-// them to row_ptr[w+1] (zeroed beforehand) with one reduction atomic -- no barrier, no
-// waiting; integer addition makes the result independent of the order.
+// Phase 1: one warp per window walks the window's 256-column chunks (the next chunk's rows
+// are loaded while the current one is counted) and writes the count into row_ptr[w+1].
 template <int V, bool VEC, bool HAS_MASK>
 __device__ __forceinline__ void count_body(int64_t M, int64_t K, int64_t w,
                                            const uint16_t* __restrict__ dense,
                                            const uint8_t* __restrict__ mask,
                                            int32_t* __restrict__ row_ptr) {
-  const int lane = lane_id(), wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  const int lane = lane_id();
   uint16_t h[V][8];
   uint32_t count = 0;
-  for (int64_t c0 = (int64_t)wid * kColsPerStep; c0 < K; c0 += (int64_t)nw * kColsPerStep) {
+#pragma unroll 2
+  for (int64_t c0 = 0; c0 < K; c0 += kColsPerStep) {
     const int64_t c = c0 + lane * kColsPerLane;
     count += __popc(window_keep8<V, VEC, HAS_MASK, false>(dense, mask, M, K, w, c, h));
   }
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) count += __shfl_xor_sync(0xffffffffu, count, o);
-  if (lane == 0 && count) atomicAdd(row_ptr + w + 1, (int32_t)count);
+  if (lane == 0) row_ptr[w + 1] = (int32_t)count;
 }
 
-// Writes col_idx and (optionally) vals of window w from row_ptr[w] on.  Per round, warp i
-// takes chunk (round * nwarps + i); a block-wide exclusive scan of the warps' keep counts
-// gives each warp its slot range, so col_idx stays ascending.
+// Writes col_idx and (optionally) vals of window w from row_ptr[w] on.  One warp per window
+// walks its 256-column chunks in order; a warp-wide exclusive scan of the lanes' keep counts
+// gives every kept column its slot, so col_idx stays ascending.
 template <int V, bool VEC, bool HAS_MASK, bool WRITE_VALS, bool VEC_VALS>
 __device__ __forceinline__ void compact_body(int64_t M, int64_t K, int64_t w,
                                              const uint16_t* __restrict__ dense,
@@ -172,12 +171,12 @@ __device__ __forceinline__ void compact_body(int64_t M, int64_t K, int64_t w,
                                              const int32_t* __restrict__ row_ptr,
                                              int32_t* __restrict__ col_idx,
                                              uint16_t* __restrict__ vals) {
-  __shared__ uint32_t warp_cnt[kEncMaxThreads / 32];
-  const int lane = lane_id(), wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  const int lane = lane_id();
   int64_t base = row_ptr[w];
   uint16_t h[V][8];
-  for (int64_t r0 = 0; r0 < K; r0 += (int64_t)nw * kColsPerStep) {
-    const int64_t c = r0 + (int64_t)wid * kColsPerStep + lane * kColsPerLane;
+#pragma unroll 2
+  for (int64_t c0 = 0; c0 < K; c0 += kColsPerStep) {
+    const int64_t c = c0 + lane * kColsPerLane;
     const uint32_t keep = window_keep8<V, VEC, HAS_MASK, WRITE_VALS>(dense, mask, M, K, w, c, h);
     const uint32_t n = __popc(keep);
     uint32_t incl = n;
@@ -186,15 +185,7 @@ __device__ __forceinline__ void compact_body(int64_t M, int64_t K, int64_t w,
       const uint32_t t = __shfl_up_sync(0xffffffffu, incl, o);
       if (lane >= o) incl += t;
     }
-    if (lane == 31) warp_cnt[wid] = incl;
-    __syncthreads();
-    uint32_t before = 0, total = 0;
-    for (int i = 0; i < nw; ++i) {
-      const uint32_t v = warp_cnt[i];
-      before += (i < wid) ? v : 0;
-      total += v;
-    }
-    int64_t slot = base + before + (incl - n);
+    int64_t slot = base + (incl - n);
 #pragma unroll
     for (int j = 0; j < 8; ++j) {
       if (keep & (1u << j)) {
@@ -217,8 +208,7 @@ __device__ __forceinline__ void compact_body(int64_t M, int64_t K, int64_t w,
         ++slot;
       }
     }
-    base += total;
-    __syncthreads();  // warp_cnt is rewritten next round
+    base += __shfl_sync(0xffffffffu, incl, 31);
   }
 }
 
@@ -228,10 +218,11 @@ __device__ __forceinline__ void compact_body(int64_t M, int64_t K, int64_t w,
 // the compact kernel WRITE_VALS and VEC_VALS (vector stores of a whole vector).
 
 template <int V, bool VEC, bool HAS_MASK>
-__global__ void __launch_bounds__(kEncMaxThreads)
-    encode_count_kernel(int64_t M, int64_t K, const uint16_t* __restrict__ dense,
+__global__ void __launch_bounds__(kEncWarps * 32)
+    encode_count_kernel(int64_t M, int64_t K, int64_t W, const uint16_t* __restrict__ dense,
                         const uint8_t* __restrict__ mask, int32_t* __restrict__ row_ptr) {
-  count_body<V, VEC, HAS_MASK>(M, K, blockIdx.x, dense, mask, row_ptr);
+  const int64_t w = (int64_t)blockIdx.x * kEncWarps + (threadIdx.x >> 5);
+  if (w < W) count_body<V, VEC, HAS_MASK>(M, K, w, dense, mask, row_ptr);
 }
 
 // Phase 2: counts -> inclusive prefix, in place (one CTA).
@@ -241,15 +232,17 @@ __global__ void __launch_bounds__(kScanThreads) encode_scan_kernel(int32_t* __re
   __shared__ int32_t s_warp[32];
   __shared__ int32_t s_carry;
   block_scan_inplace(row_ptr + 1, W, s_warp, &s_carry);
+  if (threadIdx.x == 0) row_ptr[0] = 0;
 }
 
 template <int V, bool VEC, bool HAS_MASK, bool WRITE_VALS, bool VEC_VALS>
-__global__ void __launch_bounds__(kEncMaxThreads)
-    encode_compact_kernel(int64_t M, int64_t K, const uint16_t* __restrict__ dense,
+__global__ void __launch_bounds__(kEncWarps * 32)
+    encode_compact_kernel(int64_t M, int64_t K, int64_t W, const uint16_t* __restrict__ dense,
                           const uint8_t* __restrict__ mask, const int32_t* __restrict__ row_ptr,
                           int32_t* __restrict__ col_idx, uint16_t* __restrict__ vals) {
-  compact_body<V, VEC, HAS_MASK, WRITE_VALS, VEC_VALS>(M, K, blockIdx.x, dense, mask, row_ptr,
-                                                       col_idx, vals);
+  const int64_t w = (int64_t)blockIdx.x * kEncWarps + (threadIdx.x >> 5);
+  if (w < W)
+    compact_body<V, VEC, HAS_MASK, WRITE_VALS, VEC_VALS>(M, K, w, dense, mask, row_ptr, col_idx, vals);
 }
 
 // Batched: one grid over the windows of up to kEncMaxBatch problems of one configuration
@@ -269,27 +262,15 @@ struct EncBatch {
   EncDesc d[kEncMaxBatch];
 };
 
-// zero row_ptr[0..W] of every problem of the batch
-__global__ void zero_row_ptr_kernel(const __grid_constant__ EncBatch b) {
-  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-  for (int p = 0; p < b.count; ++p)
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i <= b.d[p].W; i += stride)
-      b.d[p].row_ptr[i] = 0;
-}
-
-// Batched kernels: grid-stride loop over the windows of all problems (launched with one CTA
-// per window, so usually one iteration); first problem by binary search, then a forward
-// linear advance.
+// Batched kernels: one CTA per kEncWarps windows of one problem; the problem of a CTA is found
+// by binary search over first_block.
 template <int V, bool VEC, bool HAS_MASK>
-__global__ void __launch_bounds__(kEncMaxThreads)
+__global__ void __launch_bounds__(kEncWarps * 32)
     encode_count_batched_kernel(const __grid_constant__ EncBatch b) {
-  const int64_t total = b.first_block[b.count];
-  int p = first_problem(b.first_block, b.count, (int64_t)blockIdx.x);
-  for (int64_t bid = blockIdx.x; bid < total; bid += gridDim.x) {
-    while (b.first_block[p + 1] <= bid) ++p;
-    const EncDesc& d = b.d[p];
-    count_body<V, VEC, HAS_MASK>(d.M, d.K, bid - b.first_block[p], d.dense, d.mask, d.row_ptr);
-  }
+  const int p = first_problem(b.first_block, b.count, (int64_t)blockIdx.x);
+  const EncDesc& d = b.d[p];
+  const int64_t w = (blockIdx.x - b.first_block[p]) * kEncWarps + (threadIdx.x >> 5);
+  if (w < d.W) count_body<V, VEC, HAS_MASK>(d.M, d.K, w, d.dense, d.mask, d.row_ptr);
 }
 
 // one CTA per problem
@@ -298,19 +279,18 @@ __global__ void __launch_bounds__(kScanThreads) encode_scan_batched_kernel(const
   __shared__ int32_t s_carry;
   const EncDesc& d = b.d[blockIdx.x];
   block_scan_inplace(d.row_ptr + 1, d.W, s_warp, &s_carry);
+  if (threadIdx.x == 0) d.row_ptr[0] = 0;
 }
 
 template <int V, bool VEC, bool HAS_MASK, bool WRITE_VALS, bool VEC_VALS>
-__global__ void __launch_bounds__(kEncMaxThreads)
+__global__ void __launch_bounds__(kEncWarps * 32)
     encode_compact_batched_kernel(const __grid_constant__ EncBatch b) {
-  const int64_t total = b.first_block[b.count];
-  int p = first_problem(b.first_block, b.count, (int64_t)blockIdx.x);
-  for (int64_t bid = blockIdx.x; bid < total; bid += gridDim.x) {
-    while (b.first_block[p + 1] <= bid) ++p;
-    const EncDesc& d = b.d[p];
-    compact_body<V, VEC, HAS_MASK, WRITE_VALS, VEC_VALS>(d.M, d.K, bid - b.first_block[p], d.dense,
-                                                         d.mask, d.row_ptr, d.col_idx, d.vals);
-  }
+  const int p = first_problem(b.first_block, b.count, (int64_t)blockIdx.x);
+  const EncDesc& d = b.d[p];
+  const int64_t w = (blockIdx.x - b.first_block[p]) * kEncWarps + (threadIdx.x >> 5);
+  if (w < d.W)
+    compact_body<V, VEC, HAS_MASK, WRITE_VALS, VEC_VALS>(d.M, d.K, w, d.dense, d.mask, d.row_ptr,
+                                                         d.col_idx, d.vals);
 }
 
 struct EncCfg {
@@ -333,15 +313,10 @@ static EncCfg enc_config(int64_t K, int V, const void* dense, const uint8_t* mas
   return c;
 }
 
-static int enc_threads(int64_t K) {  // one warp per 256-column chunk, up to 8 warps
-  const int64_t chunks = ceil_div64(K, kColsPerStep);
-  return (int)(32 * (chunks < 1 ? 1 : (chunks > kEncMaxThreads / 32 ? kEncMaxThreads / 32 : chunks)));
-}
-
 struct EncKernels {
-  void (*count_single)(int64_t, int64_t, const uint16_t*, const uint8_t*, int32_t*);
-  void (*compact_single)(int64_t, int64_t, const uint16_t*, const uint8_t*, const int32_t*, int32_t*,
-                         uint16_t*);
+  void (*count_single)(int64_t, int64_t, int64_t, const uint16_t*, const uint8_t*, int32_t*);
+  void (*compact_single)(int64_t, int64_t, int64_t, const uint16_t*, const uint8_t*, const int32_t*,
+                         int32_t*, uint16_t*);
   void (*count_batched)(EncBatch);
   void (*compact_batched)(EncBatch);
 };
@@ -386,14 +361,12 @@ cudaError_t launch_encode(int64_t M, int64_t K, int V, const void* dense, const 
   if (W > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
   const EncCfg c = enc_config(K, V, dense, mask, col_idx, vals);
   const EncKernels k = enc_kernels(c);
-  const dim3 grid((unsigned)W), block(enc_threads(K));
+  const dim3 grid((unsigned)ceil_div64(W, kEncWarps)), block(kEncWarps * 32);
   const uint16_t* d = static_cast<const uint16_t*>(dense);
-  cudaError_t e = cudaMemsetAsync(row_ptr, 0, (size_t)(W + 1) * sizeof(int32_t), s);
-  if (e != cudaSuccess) return e;
-  k.count_single<<<grid, block, 0, s>>>(M, K, d, mask, row_ptr);
+  k.count_single<<<grid, block, 0, s>>>(M, K, W, d, mask, row_ptr);
   encode_scan_kernel<<<1, kScanThreads, 0, s>>>(row_ptr, W);
   if (c.IDX)
-    k.compact_single<<<grid, block, 0, s>>>(M, K, d, mask, row_ptr, col_idx,
+    k.compact_single<<<grid, block, 0, s>>>(M, K, W, d, mask, row_ptr, col_idx,
                                             static_cast<uint16_t*>(vals));
   return cudaGetLastError();
 }
@@ -417,22 +390,20 @@ cudaError_t launch_encode_batched(int64_t count, const int64_t* M, const int64_t
     const EncKernels k = enc_kernels(c);
     batch.count = 0;
     int64_t blocks = 0;
-    int threads = 32;
+    const int threads = kEncWarps * 32;
     while (i < order.size() && order[i].first == key && batch.count < kEncMaxBatch) {
       const int64_t p = order[i].second;
       const int64_t W = ceil_div64(M[p], V[p]);
-      if (blocks + W > 0x7fffffffLL) break;
+      const int64_t nb = ceil_div64(W, kEncWarps);
+      if (blocks + nb > 0x7fffffffLL) break;
       batch.d[batch.count] = {M[p], K[p], W, static_cast<const uint16_t*>(dense[p]), mask[p],
                               row_ptr[p], col_idx[p], static_cast<uint16_t*>(vals[p])};
       batch.first_block[batch.count++] = blocks;
-      blocks += W;
-      const int th = enc_threads(K[p]);
-      threads = th > threads ? th : threads;
+      blocks += nb;
       ++i;
     }
     if (batch.count == 0) return cudaErrorInvalidConfiguration;
     batch.first_block[batch.count] = blocks;
-    zero_row_ptr_kernel<<<64, 256, 0, s>>>(batch);
     // one CTA per window (measured slightly faster than a resident-sized grid-stride grid)
     (void)num_sms;
     k.count_batched<<<(unsigned)blocks, threads, 0, s>>>(batch);

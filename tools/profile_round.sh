@@ -10,10 +10,10 @@ set -x
 TAG=${1:-r01}
 ARGS="--steps 1 --warmup 1 --no-baselines --no-cpu --no-e2e --detail gpurun_out/prof_detail.json"
 # The batched step of bench.py: the warm-up replays the step graph once; kernels named
-# *batched* / zero_row_ptr belong to it (the eager sizing pass uses the single-problem
+# *batched* belong to it (the eager sizing pass uses the single-problem
 # kernels, which the regex excludes).
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none \
-  -k regex:"batched|zero_row_ptr" -c 40 --csv --log-file gpurun_out/launches_${TAG}.csv \
+  -k regex:"batched" -c 40 --csv --log-file gpurun_out/launches_${TAG}.csv \
   python bench.py $ARGS > /dev/null 2>&1
 for K in spmm_batched sddmm_batched encode_count_batched encode_compact_batched; do
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:"$K" -c 3 \
