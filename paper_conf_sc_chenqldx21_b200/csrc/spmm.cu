@@ -285,11 +285,13 @@ struct SpmmDesc {
   uint16_t* C;
 };
 constexpr int kSpmmMaxBatch = 128;
-struct SpmmBatch {
+template <int CAP>
+struct SpmmBatchT {
   int count;
-  int64_t first_block[kSpmmMaxBatch + 1];
-  SpmmDesc d[kSpmmMaxBatch];
+  int64_t first_block[CAP + 1];  // register path: CTA blocks; cp path: units (window, panel)
+  SpmmDesc d[CAP];
 };
+using SpmmBatch = SpmmBatchT<kSpmmMaxBatch>;
 
 template <int V, int NC, bool VEC, int SPLIT, int UNROLL>
 __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32)
@@ -306,6 +308,240 @@ __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32)
   }
 }
 
+// ---------------------------------------------------- cp.async-staged kernel (default path)
+//
+// Why (measured on B200, profiles/r02_gather.md): in the register path above lane 4g+t
+// loads row slot t, chunk g, so every 8-lane phase of an LDG.128 touches 4 different
+// 128-byte lines: random 128-byte row gathers with that lane mapping top out at 9.2 TB/s,
+// against 13-15 TB/s for cp.async with 8 lanes per line feeding ldmatrix (and 20 TB/s for a
+// bare LDG.128 with 8 lanes per line, which cannot feed mma.sync fragments directly).
+//
+// Work unit = (row window, panel of 64*NC columns), owned by SPLIT warps of one CTA (SPLIT
+// from K only; fixed-order shared-memory reduction, deterministic), as in the register path.
+// Each warp streams its 16-vector groups through a D-stage ring in shared memory:
+//  * rows: cp.async.cg 16 B per lane, lanes 8q..8q+7 copy one 128-byte line (one row slot,
+//    one 64-column chunk-group), so each phase is one line; slot s of a stage keeps chunk c
+//    (of 8 per 64 columns) at position c ^ (s & 7), so the 8 rows read by one ldmatrix phase
+//    (slots i..i+7, one chunk) hit 8 distinct bank groups;
+//  * the group's vals (16 vectors x V fp16) and the column indices of group j + D ride in the
+//    same commit group as the rows of group j: the col_idx -> row-address dependency is D
+//    groups ahead of the MMAs;
+//  * slots past the window end are zero-filled by the copies (src-size 0): 0 x 0 terms;
+//  * MMA m16n8k16, A = gathered rows via ldmatrix.x4.trans (M = 16 panel columns, K = 16
+//    vector slots), B = vals (K = slots, N = V rows padded to 8), fp32 accumulate;
+//  * epilogue: stmatrix.x4.trans turns the accumulator tiles into row-major 16-byte pieces
+//    of the V x 64NC output tile (swizzled, in the drained ring), then 16-byte stores.
+// Wider panels (NC = 2, 4) amortise the per-group bookkeeping over more gathered bytes.
+template <int V, int NC, int D>
+struct CpRing {
+  static constexpr int kRowBytes = 16 * 128 * NC;  // one group: 16 slots x 64NC columns fp16
+  static constexpr int kValBytes = 16 * V * 2;
+  static constexpr int kColBytes = 16 * 4;
+  static constexpr int kRaw = D * (kRowBytes + kValBytes) + 2 * D * kColBytes;
+  static constexpr int kWarpBytes = (kRaw + 127) / 128 * 128;
+};
+
+template <int V, int NC, int SPLIT, int D>
+__device__ __forceinline__ void spmm_cp_body(int64_t M, int64_t N, int64_t W, int64_t n_wgroups,
+                                             int64_t bid, const int32_t* __restrict__ row_ptr,
+                                             const int32_t* __restrict__ col_idx,
+                                             const uint16_t* __restrict__ vals,
+                                             const uint16_t* __restrict__ B,
+                                             uint16_t* __restrict__ C, unsigned char* smem) {
+  using R = CpRing<V, NC, D>;
+  constexpr int UPC = SpmmCta<SPLIT>::kUnits;
+  constexpr int HALF = SPLIT > 1 ? SPLIT / 2 : 1;
+  constexpr int PW = 64 * NC;  // panel width
+  const int lane = lane_id();
+  const int g = lane >> 2, t = lane & 3;
+  const int wid = threadIdx.x >> 5;
+  const int part = wid % SPLIT;
+  const int64_t pn = bid / n_wgroups;
+  const int64_t w = (bid - pn * n_wgroups) * UPC + wid / SPLIT;
+  const bool active = w < W;
+  const int64_t n0 = pn * PW;  // first column of the panel
+  const int p_begin = active ? row_ptr[w] : 0;
+  const int p_end = active ? row_ptr[w + 1] : 0;
+  const uint32_t s_rows = smem_u32(smem + wid * R::kWarpBytes);
+  const uint32_t s_vals = s_rows + D * R::kRowBytes;
+  const uint32_t s_cols = s_vals + D * R::kValBytes;
+  // this warp's groups: vectors [first + 16*SPLIT*j, +16)
+  const int first = p_begin + 16 * part;
+  const int G = first < p_end ? (p_end - first + 16 * SPLIT - 1) / (16 * SPLIT) : 0;
+  const int cq = lane >> 3, cc = lane & 7;  // copy role: slots cq + 4k, chunk cc of each 64
+  const uint16_t* Bp = B + n0 + 8 * cc;
+
+  // column indices of group j -> col ring entry j % 2D, permuted so that lane L finds the
+  // slots it copies (L>>3) + {0, 4, 8, 12} in one 16-byte word
+  auto copy_cols = [&](int j) {
+    if (lane < 16) {
+      const int p = first + 16 * SPLIT * j + lane;
+      const bool ok = p < p_end;
+      cp_async_zfill<4>(s_cols + (j % (2 * D)) * R::kColBytes + ((lane & 3) * 4 + (lane >> 2)) * 4,
+                        ok ? (const void*)(col_idx + p) : (const void*)col_idx, ok ? 4u : 0u);
+    }
+  };
+  // rows + vals of group j, col indices of group j + D; always one commit group
+  auto issue = [&](int j) {
+    if (j < G) {
+      const int p0 = first + 16 * SPLIT * j;
+      const uint4 cl = lds128_u32(s_cols + (j % (2 * D)) * R::kColBytes + cq * 16);
+      const int cv[4] = {(int)cl.x, (int)cl.y, (int)cl.z, (int)cl.w};
+      const uint32_t rs = s_rows + (j % D) * R::kRowBytes;
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        const int sl = cq + 4 * k;
+        const bool okp = p0 + sl < p_end;
+        const uint16_t* src = Bp + (int64_t)cv[k] * N;
+#pragma unroll
+        for (int h = 0; h < NC; ++h) {
+          const bool ok = okp && (n0 + 64 * h + 8 * cc < N);
+          cp_async_zfill<16>(rs + sl * (128 * NC) + ((8 * h + (cc ^ (sl & 7))) * 16),
+                             ok ? (const void*)(src + 64 * h) : (const void*)B, ok ? 16u : 0u);
+        }
+      }
+      if (lane < 16) {
+        const int p = p0 + lane;
+        const bool ok = p < p_end;
+        cp_async_zfill<2 * V>(s_vals + (j % D) * R::kValBytes + lane * (2 * V),
+                              ok ? (const void*)(vals + (int64_t)p * V) : (const void*)vals,
+                              ok ? (uint32_t)(2 * V) : 0u);
+      }
+      if (j + D < G) copy_cols(j + D);
+    }
+    cp_async_commit();
+  };
+
+  float acc[NC][4][4];
+#pragma unroll
+  for (int h = 0; h < NC; ++h)
+#pragma unroll
+    for (int j = 0; j < 4; ++j)
+#pragma unroll
+      for (int e = 0; e < 4; ++e) acc[h][j][e] = 0.f;
+
+  const int mi = lane >> 3, ri = lane & 7;  // ldmatrix / stmatrix role
+  if (G > 0) {
+#pragma unroll 1
+    for (int j = 0; j < D && j < G; ++j) copy_cols(j);
+    cp_async_commit();
+    cp_async_wait<0>();
+    __syncwarp();
+#pragma unroll
+    for (int j = 0; j < D - 1; ++j) issue(j);
+    const int slot = ri + 8 * (mi >> 1);
+#pragma unroll 1
+    for (int j = 0; j < G; ++j) {
+      issue(j + D - 1);
+      cp_async_wait<D - 1>();
+      __syncwarp();
+      const uint32_t rs = s_rows + (j % D) * R::kRowBytes + slot * (128 * NC);
+      const uint32_t vs = s_vals + (j % D) * R::kValBytes;
+      uint32_t b0 = 0, b1 = 0;
+      if (g < V) {
+        b0 = pack_h2(lds16(vs + ((2 * t) * V + g) * 2), lds16(vs + ((2 * t + 1) * V + g) * 2));
+        b1 = pack_h2(lds16(vs + ((2 * t + 8) * V + g) * 2), lds16(vs + ((2 * t + 9) * V + g) * 2));
+      }
+#pragma unroll
+      for (int h = 0; h < NC; ++h)
+#pragma unroll
+        for (int jj = 0; jj < 4; ++jj) {
+          const int chunk = 2 * jj + (mi & 1);
+          uint32_t a0, a1, a2, a3;
+          ldsm_x4_trans(rs + ((8 * h + (chunk ^ ri)) * 16), a0, a1, a2, a3);
+          mma_16816(acc[h][jj], a0, a1, a2, a3, b0, b1);
+        }
+      __syncwarp();
+    }
+    cp_async_wait<0>();
+    __syncwarp();
+  }
+
+  if constexpr (SPLIT > 1) {
+    // fixed pairwise tree over the unit's parts through the parts' own (drained) rings
+    const uint32_t mine = s_rows;
+#pragma unroll
+    for (int hh = HALF; hh >= 1; hh >>= 1) {
+      if (part >= hh && part < 2 * hh) {
+#pragma unroll
+        for (int h = 0; h < NC; ++h)
+#pragma unroll
+          for (int j = 0; j < 4; ++j)
+#pragma unroll
+            for (int e = 0; e < 4; ++e)
+              asm volatile("st.shared.f32 [%0], %1;" ::"r"(mine + ((((h * 4 + j) * 4 + e) * 32) + lane) * 4),
+                           "f"(acc[h][j][e])
+                           : "memory");
+      }
+      __syncthreads();
+      if (part < hh) {
+        const uint32_t other = mine + hh * R::kWarpBytes;
+#pragma unroll
+        for (int h = 0; h < NC; ++h)
+#pragma unroll
+          for (int j = 0; j < 4; ++j)
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+              float v;
+              asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v)
+                           : "r"(other + ((((h * 4 + j) * 4 + e) * 32) + lane) * 4));
+              acc[h][j][e] += v;
+            }
+      }
+      __syncthreads();
+    }
+  }
+  if (part != 0 || !active) return;  // no barrier follows in this unit
+
+  // epilogue: accumulator tile (h, jj) holds C[r = 2t (+1)][n0 + 64h + 16jj + g (+8)];
+  // out tile: 8 rows x 8NC chunks of 16 B, chunk c of row r at (c & ~7) | ((c ^ r) & 7)
+  const uint32_t s_out = s_rows;
+#pragma unroll
+  for (int h = 0; h < NC; ++h)
+#pragma unroll
+    for (int q = 0; q < 2; ++q) {
+      const int chunk = 4 * q + mi;
+      stsm_x4_trans(s_out + ri * (128 * NC) + ((8 * h + (chunk ^ ri)) * 16),
+                    f2_to_h2(acc[h][2 * q][0], acc[h][2 * q][1]),
+                    f2_to_h2(acc[h][2 * q][2], acc[h][2 * q][3]),
+                    f2_to_h2(acc[h][2 * q + 1][0], acc[h][2 * q + 1][1]),
+                    f2_to_h2(acc[h][2 * q + 1][2], acc[h][2 * q + 1][3]));
+    }
+  __syncwarp();
+#pragma unroll
+  for (int idx = lane; idx < V * 8 * NC; idx += 32) {
+    const int r = idx / (8 * NC), ch = idx % (8 * NC);
+    const int64_t i = w * V + r;
+    const int64_t n = n0 + 8 * ch;
+    const uint4 v = lds128_u32(s_out + r * (128 * NC) + (((ch & ~7) | ((ch ^ r) & 7)) * 16));
+    if (i < M && n < N) stg128(C + i * N + n, v);
+  }
+}
+
+template <int V, int NC, int SPLIT, int D>
+__global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32)
+    spmm_cp_kernel(int64_t M, int64_t N, int64_t W, int64_t n_wgroups,
+                   const int32_t* __restrict__ row_ptr, const int32_t* __restrict__ col_idx,
+                   const uint16_t* __restrict__ vals, const uint16_t* __restrict__ B,
+                   uint16_t* __restrict__ C) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  spmm_cp_body<V, NC, SPLIT, D>(M, N, W, n_wgroups, blockIdx.x, row_ptr, col_idx, vals, B, C, smem);
+}
+
+template <int V, int NC, int SPLIT, int D>
+__global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32)
+    spmm_cp_batched_kernel(const __grid_constant__ SpmmBatch b) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  const int64_t total = b.first_block[b.count];
+  int p = first_problem(b.first_block, b.count, (int64_t)blockIdx.x);
+  for (int64_t bid = blockIdx.x; bid < total; bid += gridDim.x) {
+    while (b.first_block[p + 1] <= bid) ++p;
+    const SpmmDesc& d = b.d[p];
+    spmm_cp_body<V, NC, SPLIT, D>(d.M, d.N, d.W, d.n_wgroups, bid - b.first_block[p], d.row_ptr,
+                                  d.col_idx, d.vals, d.B, d.C, smem);
+  }
+}
+
 // Kernel configuration of one problem.  NC (64- or 128-column panels) follows N; SPLIT
 // (warps per unit, about one per 256 possible vectors of a window, up to 16) follows K only,
 // so N-panel shards of a problem run with exactly the same per-element accumulation order
@@ -314,16 +550,44 @@ __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32)
 struct SpmmCfg {
   int V, NC, SPLIT;
   bool VEC;
+  int CP;  // cp.async ring depth (0 = register path)
   bool operator<(const SpmmCfg& o) const {
-    return V != o.V ? V < o.V : NC != o.NC ? NC < o.NC : SPLIT != o.SPLIT ? SPLIT < o.SPLIT : VEC < o.VEC;
+    return V != o.V ? V < o.V : NC != o.NC ? NC < o.NC : SPLIT != o.SPLIT ? SPLIT < o.SPLIT
+                                                         : VEC != o.VEC ? VEC < o.VEC : CP < o.CP;
   }
 };
+
+// cp.async path on/off and its ring depth: VS_SPMM_CP = 0 selects the register path,
+// otherwise the number of stages D (3 or 4; default 3).  VS_SPMM_CPNC caps the panel width
+// (64 * NC columns, NC in {1, 2, 4}; default 2: tools/tune.py over the DLMC batch, batched
+// 502 us (cap 2) vs 569 us (cap 4) vs 650 us (cap 1) vs 629 us for the register path).
+static int spmm_cp_stages() {
+  static const int v = [] {
+    const char* e = std::getenv("VS_SPMM_CP");
+    const int d = e ? std::atoi(e) : 3;
+    return d <= 0 ? 0 : d <= 3 ? 3 : 4;
+  }();
+  return v;
+}
+static int spmm_cp_nc_cap() {
+  static const int v = [] {
+    const char* e = std::getenv("VS_SPMM_CPNC");
+    const int n = e ? std::atoi(e) : 2;
+    return n >= 4 ? 4 : n >= 2 ? 2 : 1;
+  }();
+  return v;
+}
+static int64_t cp_smem_bytes(int V, int NC, int SPLIT, int D) {
+  const int64_t warps = SPLIT > kSpmmWarps ? SPLIT : kSpmmWarps;
+  const int64_t raw = (int64_t)D * (16 * 128 * NC + 32 * V) + 2 * D * 64;
+  return warps * ((raw + 127) / 128 * 128);
+}
 
 SpmmCfg spmm_config(int64_t K, int64_t N, int V, const void* B, const void* C) {
   SpmmCfg c;
   c.V = V;
-  // 64-column panels: a K x 64 panel of B stays L1-resident for K <= ~1500 (tools/tune.py:
-  // 3% faster than 128-column panels over the DLMC batch; VS_SPMM_NC=2 selects 128 columns).
+  // register path: 64-column panels (a K x 64 panel of B stays L1-resident for K <= ~1500;
+  // tools/tune.py: 3% faster than 128-column panels; VS_SPMM_NC=2 selects 128 columns)
   static const int nc_knob = [] {
     const char* e = std::getenv("VS_SPMM_NC");
     return e ? std::atoi(e) : 1;
@@ -333,6 +597,15 @@ SpmmCfg spmm_config(int64_t K, int64_t N, int V, const void* B, const void* C) {
   c.SPLIT = q >= 16 ? 16 : q >= 8 ? 8 : q >= 4 ? 4 : q >= 2 ? 2 : 1;
   c.VEC = (N % 8 == 0) && ((reinterpret_cast<uintptr_t>(B) & 15) == 0) &&
           ((reinterpret_cast<uintptr_t>(C) & 15) == 0);
+  // cp.async path: 16-byte row copies and stores (VEC), vals copies of 2V >= 4 bytes; panel
+  // width follows N (it does not change any element's accumulation order)
+  c.CP = (c.VEC && V >= 2) ? spmm_cp_stages() : 0;
+  if (c.CP) {
+    int nc = N > 128 ? 4 : N > 64 ? 2 : 1;
+    if (nc > spmm_cp_nc_cap()) nc = spmm_cp_nc_cap();
+    while (nc > 1 && cp_smem_bytes(V, nc, c.SPLIT, c.CP) > 227 * 1024) nc >>= 1;
+    c.NC = nc;
+  }
   return c;
 }
 
@@ -341,7 +614,57 @@ struct SpmmKernels {
                  const uint16_t*, const uint16_t*, uint16_t*);
   void (*batched)(SpmmBatch);
   int threads, units_per_cta, batched_ctas_per_sm;
+  int smem;  // dynamic shared memory bytes (cp.async path), 0 otherwise
 };
+
+// cp path: raise the dynamic shared memory limit of the instantiation once per device
+template <int V, int NC, int SPLIT, int D>
+static SpmmKernels cp_kernels_of() {
+  constexpr int smem = SpmmCta<SPLIT>::kWarps * CpRing<V, NC, D>::kWarpBytes;
+  static_assert(smem <= 227 * 1024 || NC > 1, "cp ring does not fit");
+  static bool done[64] = {};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (smem > 48 * 1024 && !(dev >= 0 && dev < 64 && done[dev])) {
+    cudaFuncSetAttribute(spmm_cp_kernel<V, NC, SPLIT, D>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    cudaFuncSetAttribute(spmm_cp_batched_kernel<V, NC, SPLIT, D>,
+                         cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (dev >= 0 && dev < 64) done[dev] = true;
+  }
+  return {spmm_cp_kernel<V, NC, SPLIT, D>, spmm_cp_batched_kernel<V, NC, SPLIT, D>,
+          SpmmCta<SPLIT>::kWarps * 32, SpmmCta<SPLIT>::kUnits, 0, smem};
+}
+
+template <int V, int NC, int SPLIT>
+static SpmmKernels cp_pick_d(int d) {
+  if constexpr (SpmmCta<SPLIT>::kWarps * CpRing<V, NC, 3>::kWarpBytes > 227 * 1024) {
+    return cp_kernels_of<V, 1, SPLIT, 3>();  // unreachable: spmm_config shrinks NC first
+  } else if constexpr (SpmmCta<SPLIT>::kWarps * CpRing<V, NC, 4>::kWarpBytes > 227 * 1024) {
+    return cp_kernels_of<V, NC, SPLIT, 3>();
+  } else {
+    return d == 4 ? cp_kernels_of<V, NC, SPLIT, 4>() : cp_kernels_of<V, NC, SPLIT, 3>();
+  }
+}
+
+template <int V, int NC>
+static SpmmKernels cp_pick_split(int split, int d) {
+  switch (split) {
+    case 16: return cp_pick_d<V, NC, 16>(d);
+    case 8: return cp_pick_d<V, NC, 8>(d);
+    case 4: return cp_pick_d<V, NC, 4>(d);
+    case 2: return cp_pick_d<V, NC, 2>(d);
+    default: return cp_pick_d<V, NC, 1>(d);
+  }
+}
+
+template <int V>
+static SpmmKernels cp_pick(const SpmmCfg& c) {
+  switch (c.NC) {
+    case 4: return cp_pick_split<V, 4>(c.SPLIT, c.CP);
+    case 2: return cp_pick_split<V, 2>(c.SPLIT, c.CP);
+    default: return cp_pick_split<V, 1>(c.SPLIT, c.CP);
+  }
+}
 
 // Main-loop variant (tools/tune.py): 0 (default) = the plain loop; VS_SPMM_PIPE=1 keeps the
 // B rows of the next group in flight during the current group's MMAs -- measured 10% slower,
@@ -359,9 +682,9 @@ template <int V, int NC, bool VEC, int SPLIT>
 static SpmmKernels kernels_of() {
   if (spmm_pipe())
     return {spmm_kernel<V, NC, VEC, SPLIT, 0>, spmm_batched_kernel<V, NC, VEC, SPLIT, 0>,
-            SpmmCta<SPLIT>::kWarps * 32, SpmmCta<SPLIT>::kUnits, 0};
+            SpmmCta<SPLIT>::kWarps * 32, SpmmCta<SPLIT>::kUnits, 0, 0};
   return {spmm_kernel<V, NC, VEC, SPLIT, 1>, spmm_batched_kernel<V, NC, VEC, SPLIT, 1>,
-          SpmmCta<SPLIT>::kWarps * 32, SpmmCta<SPLIT>::kUnits, 0};
+          SpmmCta<SPLIT>::kWarps * 32, SpmmCta<SPLIT>::kUnits, 0, 0};
 }
 
 template <int V, int NC, bool VEC>
@@ -382,6 +705,13 @@ static SpmmKernels pick_v(const SpmmCfg& c) {
 }
 
 static SpmmKernels pick(const SpmmCfg& c) {
+  if (c.CP) {
+    switch (c.V) {
+      case 2: return cp_pick<2>(c);
+      case 4: return cp_pick<4>(c);
+      default: return cp_pick<8>(c);
+    }
+  }
   switch (c.V) {
     case 1: return pick_v<1>(c);
     case 2: return pick_v<2>(c);
@@ -408,10 +738,11 @@ cudaError_t launch_spmm(int64_t M, int64_t K, int64_t N, int V, const int32_t* r
   int64_t W, nwg;
   const int64_t grid = spmm_blocks(k, c, M, N, V, &W, &nwg);
   if (grid > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
-  k.single<<<(unsigned)grid, k.threads, 0, s>>>(M, N, W, nwg, row_ptr, col_idx,
-                                                static_cast<const uint16_t*>(vals),
-                                                static_cast<const uint16_t*>(B),
-                                                static_cast<uint16_t*>(C));
+  if (grid == 0) return cudaSuccess;
+  k.single<<<(unsigned)grid, k.threads, k.smem, s>>>(M, N, W, nwg, row_ptr, col_idx,
+                                                     static_cast<const uint16_t*>(vals),
+                                                     static_cast<const uint16_t*>(B),
+                                                     static_cast<uint16_t*>(C));
   return cudaGetLastError();
 }
 
@@ -452,7 +783,7 @@ cudaError_t launch_spmm_batched(int64_t count, const int64_t* M, const int64_t* 
     batch.first_block[batch.count] = blocks;
     // one CTA per block (measured slightly faster than a resident-sized grid-stride grid)
     (void)num_sms;
-    if (blocks > 0) k.batched<<<(unsigned)blocks, k.threads, 0, s>>>(batch);
+    if (blocks > 0) k.batched<<<(unsigned)blocks, k.threads, k.smem, s>>>(batch);
     const cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
   }

@@ -42,15 +42,20 @@ __global__ void l1_kernel(const uint4* __restrict__ p, int slice16, int passes, 
 }
 
 // gather: each group of 8 lanes reads one random 128-byte row (4 rows per LDG.128 instruction)
-__global__ void gather_kernel(const uint4* __restrict__ mat, int rows, int iters, uint4* sink) {
+// mode 1: the mma.sync fragment mapping of the register-path SpMM (lane = 4g + t reads row t,
+// chunk g): every quarter-warp phase touches 4 different rows instead of one.
+__global__ void gather_kernel(const uint4* __restrict__ mat, int rows, int iters, uint4* sink,
+                              int mode = 0) {
   const int lane = threadIdx.x & 31;
-  uint32_t x = 0x9E3779B9u * (blockIdx.x * blockDim.x + threadIdx.x / 8 + 1);
+  const int rowsel = mode ? (lane & 3) : (lane >> 3);
+  const int chunk = mode ? (lane >> 2) : (lane & 7);
+  uint32_t x = 0x9E3779B9u * (blockIdx.x * blockDim.x / 8 + (threadIdx.x >> 5) * 4 + rowsel + 1);
   uint4 acc = make_uint4(0, 0, 0, 0);
   for (int it = 0; it < iters; ++it) {
     x ^= x << 13; x ^= x >> 17; x ^= x << 5;
     const int r = x % rows;
     uint4 v;
-    asm volatile("ld.global.nc.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(mat + (int64_t)r * 8 + (lane & 7)));
+    asm volatile("ld.global.nc.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(mat + (int64_t)r * 8 + chunk));
     acc.x ^= v.x; acc.y ^= v.y; acc.z ^= v.z; acc.w ^= v.w;
   }
   if ((acc.x ^ acc.y ^ acc.z ^ acc.w) == 0x12345678) sink[threadIdx.x] = acc;
@@ -123,6 +128,13 @@ int main() {
   g.rows = (64 << 10) / 128;
   ms = time_ms([](void*) { gather_kernel<<<g.grid, 256>>>(g.p, g.rows, g.iters, g.sink); }, nullptr);
   printf("{\"test\":\"gather128_l1\",\"GBps\":%.1f}\n", (double)g.grid * 256 * 16 * g.iters / ms / 1e6);
+  // the same gathers with the lane -> (row, chunk) mapping of the mma.sync A fragment
+  g.rows = (16 << 20) / 128;
+  ms = time_ms([](void*) { gather_kernel<<<g.grid, 256>>>(g.p, g.rows, g.iters, g.sink, 1); }, nullptr);
+  printf("{\"test\":\"gather128_l2_fragmap\",\"GBps\":%.1f}\n", (double)g.grid * 256 * 16 * g.iters / ms / 1e6);
+  g.rows = (64 << 10) / 128;
+  ms = time_ms([](void*) { gather_kernel<<<g.grid, 256>>>(g.p, g.rows, g.iters, g.sink, 1); }, nullptr);
+  printf("{\"test\":\"gather128_l1_fragmap\",\"GBps\":%.1f}\n", (double)g.grid * 256 * 16 * g.iters / ms / 1e6);
   // mma.sync m16n8k16 throughput
   g.iters = 4096; g.grid = sms * 4;
   ms = time_ms([](void*) { mma_kernel<<<g.grid, 512>>>(g.iters, g.fs); }, nullptr);
