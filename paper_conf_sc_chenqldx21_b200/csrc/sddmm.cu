@@ -3,12 +3,11 @@
 //   out_vals[p*V + r] = sum_k A[wV+r][k] * Bt[col_idx[p]][k]   (p in window w)
 //
 // Work decomposition (B200 re-design; the paper launches ceil(M/V) x ceil(N/32) CTAs over
-// the DENSE N, many of them idle): a persistent grid of warps splits the
-// stored vectors 0..nnz_v-1 (nnz_v = row_ptr[W], read on the device, so no host sync) into
-// 16-vector slices; every warp owns a contiguous run of slices, finds the window of its
-// first vector once by a warp-cooperative search of row_ptr and then walks forward.  A
-// slice that straddles windows is finished window by window (rows of other windows are
-// computed and dropped).
+// the DENSE N, many of them idle): a persistent grid of warps; the 16-vector
+// chunks of every row window are owned by q warps of the launch (warp j takes chunks j,
+// j + q, ...), q chosen on the device from nnz_v = row_ptr[W] (no host sync) so that every
+// warp gets about the same number of chunks.  Chunks never straddle windows, so the A rows
+// of a window are loaded once per warp.
 //
 // MMA mapping (operand switch as in P:1059-1063): M = 16 vectors of the slice, N = V rows of
 // the window (padded to 8), K = the inner dimension.  Both operands are K-contiguous rows
@@ -18,6 +17,7 @@
 // partial sum stays inside one MMA accumulator, so the paper's cross-octet shuffle+FADD
 // reduction (17-30% of instructions) disappears.
 #include <algorithm>
+#include <cstdlib>
 #include <utility>
 #include <vector>
 
@@ -52,38 +52,16 @@ __device__ __forceinline__ uint32_t wordj(const uint4& v, int j) {
   return j == 0 ? v.x : (j == 1 ? v.y : (j == 2 ? v.z : v.w));
 }
 
-// Largest w in [0, W) with row_ptr[w] <= v (the window owning vector v; empty windows
-// before it are skipped).  Warp-cooperative 32-ary search; all lanes get the result.
-__device__ __forceinline__ int64_t find_window(const int32_t* __restrict__ row_ptr, int64_t W,
-                                               int64_t v) {
-  int64_t lo = 0, hi = W;  // answer in [lo, hi)
-  const int lane = lane_id();
-  while (hi - lo > 1) {
-    const int64_t span = hi - lo;
-    const int64_t step = (span + 31) / 32;
-    const int64_t probe = lo + (int64_t)lane * step;
-    const bool le = (probe < hi) && (row_ptr[probe] <= v);
-    const unsigned ballot = __ballot_sync(0xffffffffu, le);
-    // lanes 0..(n-1) satisfy le (row_ptr non-decreasing); lane 0 always (row_ptr[lo] <= v)
-    const int last = 31 - __clz(ballot);
-    const int64_t nlo = lo + (int64_t)last * step;
-    const int64_t nhi = (last == 31) ? hi : (lo + (int64_t)(last + 1) * step);
-    lo = nlo;
-    hi = nhi < hi ? nhi : hi;
-  }
-  return lo;
-}
-
-// Stores the two vectors (M rows g, g+8) of a 16-vector slice held in acc, restricted to the
-// vectors [lo, hi) of window w.
+// Stores the two vectors (M rows g, g+8) of a 16-vector chunk held in acc, restricted to
+// the vectors below `hi`.
 template <int V>
-__device__ __forceinline__ void store_slice(const float (&acc)[4], int64_t v0, int64_t lo,
-                                            int64_t hi, int64_t w, int64_t M, int g, int t,
+__device__ __forceinline__ void store_chunk(const float (&acc)[4], int64_t v0, int64_t hi,
+                                            int64_t w, int64_t M, int g, int t,
                                             uint16_t* __restrict__ out, bool out4) {
 #pragma unroll
   for (int q = 0; q < 2; ++q) {
     const int64_t v = v0 + g + 8 * q;
-    if (v < lo || v >= hi) continue;
+    if (v >= hi) continue;
     const int r = 2 * t;
     const float f0 = (w * V + r < M) ? acc[2 * q] : 0.f;
     const float f1 = (w * V + r + 1 < M) ? acc[2 * q + 1] : 0.f;
@@ -97,108 +75,102 @@ __device__ __forceinline__ void store_slice(const float (&acc)[4], int64_t v0, i
   }
 }
 
-// One warp computes the 16-vector slices [s_begin, s_end) of one problem (nnz stored
-// vectors in total); s_begin < s_end.  The work is one stream of 64-wide K chunks (slice by
-// slice; a slice that straddles windows is finished window by window, re-reading its rows),
-// software-pipelined one chunk ahead: while the MMAs of a chunk run, the gathered Bt rows of
-// the next chunk -- possibly the first chunk of the next segment or slice -- are in flight,
-// and the column indices of the next slice are fetched one slice ahead.  The first loads are
-// issued before the window search, which does not affect them.  (Processing 2 or 4 slices of
-// one window together to share the A fragment measured no faster, tools/tune.py.)
-template <int V, bool VEC>
-__device__ __forceinline__ void sddmm_range(int64_t M, int64_t K, int64_t W,
-                                            const int32_t* __restrict__ row_ptr,
-                                            const int32_t* __restrict__ col_idx,
-                                            const uint16_t* __restrict__ A,
-                                            const uint16_t* __restrict__ Bt,
-                                            uint16_t* __restrict__ out, bool out4, int64_t s_begin,
-                                            int64_t s_end, int64_t nnz) {
+// One warp computes the 16-vector chunks j0, j0 + q, j0 + 2q, ... of window w.
+// Dependency chain: row_ptr[w], row_ptr[w+1] -> col_idx of the first chunk -> the gathered
+// Bt rows; then ONE round trip per chunk and K block of 64*KC: the Bt rows (and, when the
+// block is not the whole K, the window's A rows) of all KC 64-wide chunks are loaded
+// together, then the KC x 4 MMAs run; the column indices of the warp's next chunk are
+// fetched one chunk ahead.  Latency is hidden across warps (no register double buffer:
+// measured slower, 628 vs 554 us over the DLMC batch, because of the occupancy it costs).
+// (The previous design -- contiguous 16-vector slices straddling windows, one 64-wide chunk
+// in flight -- paid a round trip per chunk on the A row and per window of a straddling
+// slice: 7 us for a 98%-sparse 512 x 512 mask at K = 256; this one takes 3.3 us.)
+template <int V, bool VEC, int KC, bool ARES>
+__device__ __forceinline__ void sddmm_window(int64_t M, int64_t K,
+                                             const int32_t* __restrict__ row_ptr,
+                                             const int32_t* __restrict__ col_idx,
+                                             const uint16_t* __restrict__ A,
+                                             const uint16_t* __restrict__ Bt,
+                                             uint16_t* __restrict__ out, bool out4, int64_t w,
+                                             int64_t j0, int64_t q) {
+  (void)ARES;
   const int lane = lane_id();
   const int g = lane >> 2, t = lane & 3;
   const int64_t kt = 8 * t;
-  int64_t v0 = s_begin * 16;
-  int64_t v_hi = (v0 + 16 < nnz) ? v0 + 16 : nnz;
-  bool oka = v0 + g < v_hi, okb = v0 + g + 8 < v_hi;
-  const uint16_t* rowa = Bt + (int64_t)(oka ? ldg32i(col_idx + v0 + g) : 0) * K;
-  const uint16_t* rowb = Bt + (int64_t)(okb ? ldg32i(col_idx + v0 + g + 8) : 0) * K;
-  uint4 a0, a1, b0, b1;  // Bt chunk [k0, k0 + 64) of vectors g and g+8 (the next one to use)
-  load_seg2<VEC>(rowa, K, kt, oka, a0, a1);
-  load_seg2<VEC>(rowb, K, kt, okb, b0, b1);
-  int64_t w = find_window(row_ptr, W, v0);
-  int64_t w_end_p = row_ptr[w + 1];
-
-  for (int64_t s = s_begin; s < s_end; ++s) {
-    // next slice's column indices, one slice ahead
-    const bool has_next = s + 1 < s_end;
-    const int64_t nv0 = v0 + 16;
-    const int64_t nv_hi = (nv0 + 16 < nnz) ? nv0 + 16 : nnz;
-    const bool noka = has_next && nv0 + g < nv_hi, nokb = has_next && nv0 + g + 8 < nv_hi;
-    const int nca = noka ? ldg32i(col_idx + nv0 + g) : 0;
-    const int ncb = nokb ? ldg32i(col_idx + nv0 + g + 8) : 0;
-
-    int64_t v_cur = v0;
-    while (v_cur < v_hi) {
-      while (w_end_p <= v_cur) {  // advance to the window owning v_cur
-        ++w;
-        w_end_p = row_ptr[w + 1];
+  const int64_t pb = row_ptr[w], pe = row_ptr[w + 1];
+  int64_t v0 = pb + 16 * j0;
+  if (v0 >= pe) return;
+  const int64_t arow = w * V + g;
+  const bool ok_row = (g < V) && (arow < M);
+  const uint16_t* rowA = A + arow * K;
+  const bool one_block = K <= 64 * KC;
+  int ca = (v0 + g < pe) ? ldg32i(col_idx + v0 + g) : 0;
+  int cb = (v0 + g + 8 < pe) ? ldg32i(col_idx + v0 + g + 8) : 0;
+  uint4 xx0[KC], xx1[KC];  // A rows of the window, K block
+  if (one_block) {
+#pragma unroll
+    for (int c = 0; c < KC; ++c) load_seg2<VEC>(rowA, K, 64 * c + kt, ok_row, xx0[c], xx1[c]);
+  }
+  for (; v0 < pe; v0 += 16 * q) {
+    const bool oka = v0 + g < pe, okb = v0 + g + 8 < pe;
+    const int64_t nv0 = v0 + 16 * q;
+    const int nca = (nv0 + g < pe) ? ldg32i(col_idx + nv0 + g) : 0;
+    const int ncb = (nv0 + g + 8 < pe) ? ldg32i(col_idx + nv0 + g + 8) : 0;
+    const uint16_t* rowa = Bt + (int64_t)ca * K;
+    const uint16_t* rowb = Bt + (int64_t)cb * K;
+    float acc[4] = {0.f, 0.f, 0.f, 0.f};
+    for (int64_t kb = 0; kb < K; kb += 64 * KC) {
+      uint4 xa0[KC], xa1[KC], xb0[KC], xb1[KC];
+#pragma unroll
+      for (int c = 0; c < KC; ++c) {
+        const int64_t k = kb + 64 * c + kt;
+        load_seg2<VEC>(rowa, K, k, oka, xa0[c], xa1[c]);
+        load_seg2<VEC>(rowb, K, k, okb, xb0[c], xb1[c]);
+        if (!one_block) load_seg2<VEC>(rowA, K, k, ok_row, xx0[c], xx1[c]);
       }
-      const int64_t seg_hi = w_end_p < v_hi ? w_end_p : v_hi;  // vectors [v_cur, seg_hi) in w
-      const bool last_seg = seg_hi == v_hi;
-      const int64_t arow = w * V + g;
-      const bool ok_row = (g < V) && (arow < M);
-      const uint16_t* rowA = A + arow * K;
-      float acc[4] = {0.f, 0.f, 0.f, 0.f};
-      for (int64_t k0 = 0; k0 < K; k0 += 64) {
-        uint4 x0, x1;  // A row g of the window, same K permutation
-        load_seg2<VEC>(rowA, K, k0 + kt, ok_row, x0, x1);
-        const uint4 ca0 = a0, ca1 = a1, cb0 = b0, cb1 = b1;
-        if (k0 + 64 < K) {  // next chunk of the same rows
-          load_seg2<VEC>(rowa, K, k0 + 64 + kt, oka, a0, a1);
-          load_seg2<VEC>(rowb, K, k0 + 64 + kt, okb, b0, b1);
-        } else if (!last_seg) {  // the same rows again, for the slice's next window
-          load_seg2<VEC>(rowa, K, kt, oka, a0, a1);
-          load_seg2<VEC>(rowb, K, kt, okb, b0, b1);
-        } else if (has_next) {  // first chunk of the next slice
-          load_seg2<VEC>(Bt + (int64_t)nca * K, K, kt, noka, a0, a1);
-          load_seg2<VEC>(Bt + (int64_t)ncb * K, K, kt, nokb, b0, b1);
-        }
+#pragma unroll
+      for (int c = 0; c < KC; ++c)
 #pragma unroll
         for (int j = 0; j < 4; ++j)
-          mma_16816(acc, wordj(ca0, j), wordj(cb0, j), wordj(ca1, j), wordj(cb1, j),
-                    wordj(x0, j), wordj(x1, j));
-      }
-      store_slice<V>(acc, v0, v_cur, seg_hi, w, M, g, t, out, out4);
-      v_cur = seg_hi;
+          mma_16816(acc, wordj(xa0[c], j), wordj(xb0[c], j), wordj(xa1[c], j), wordj(xb1[c], j),
+                    wordj(xx0[c], j), wordj(xx1[c], j));
     }
-    v0 = nv0;
-    v_hi = nv_hi;
-    oka = noka;
-    okb = nokb;
-    rowa = Bt + (int64_t)nca * K;
-    rowb = Bt + (int64_t)ncb * K;
+    store_chunk<V>(acc, v0, pe, w, M, g, t, out, out4);
+    ca = nca;
+    cb = ncb;
   }
 }
 
-template <int V, bool VEC>
-__global__ void __launch_bounds__(kSddmmWarps * 32)
+// Work items of one problem: W windows x q warps per window (warp j of window w takes the
+// window's 16-vector chunks j, j + q, ...); q = the number of warps per window that gives
+// every warp of the launch about the same number of chunks.
+__device__ __forceinline__ int64_t sddmm_q(int64_t chunks, int64_t W, int64_t per_warp) {
+  const int64_t q = ceil_div64(chunks, W * per_warp);
+  return q < 1 ? 1 : (q > 64 ? 64 : q);
+}
+
+template <int V, bool VEC, int KC, bool ARES>
+__global__ void __launch_bounds__(kSddmmWarps * 32, 4)
     sddmm_kernel(int64_t M, int64_t K, int64_t W, const int32_t* __restrict__ row_ptr,
                  const int32_t* __restrict__ col_idx, const uint16_t* __restrict__ A,
                  const uint16_t* __restrict__ Bt, uint16_t* __restrict__ out, bool out4) {
   const int64_t nnz = row_ptr[W];
-  const int64_t n_slices = ceil_div64(nnz, 16);
   const int64_t n_warps = (int64_t)gridDim.x * kSddmmWarps;
   const int64_t gw = (int64_t)blockIdx.x * kSddmmWarps + (threadIdx.x >> 5);
-  const int64_t per = ceil_div64(n_slices, n_warps);
-  const int64_t s_begin = gw * per;
-  const int64_t s_end = (s_begin + per < n_slices) ? s_begin + per : n_slices;
-  if (s_begin >= s_end) return;
-  sddmm_range<V, VEC>(M, K, W, row_ptr, col_idx, A, Bt, out, out4, s_begin, s_end, nnz);
+  const int64_t chunks = ceil_div64(nnz, 16) + W;  // upper bound of sum_w ceil(nnz_w / 16)
+  const int64_t q = sddmm_q(chunks, W, ceil_div64(chunks, n_warps));
+  const int64_t items = W * q;
+  for (int64_t it = gw; it < items; it += n_warps) {
+    const int64_t w = it / q;
+    sddmm_window<V, VEC, KC, ARES>(M, K, row_ptr, col_idx, A, Bt, out, out4, w, it - w * q, q);
+  }
 }
 
-// Batched launch over up to kSddmmMaxBatch problems of one configuration.  Each problem's
-// slices (count from its row_ptr[W], read on the device and prefix-summed per CTA in shared
-// memory) are cut into chunks of kSliceChunk slices; the chunks of all problems are dealt
-// round-robin to the persistent warps.
+// Batched launch over up to kSddmmMaxBatch problems of one configuration: every problem
+// gets W_p x q_p work items (q_p from its nnz, read on the device, so every warp gets about
+// the same number of chunks); the items of all problems are dealt round-robin to the
+// persistent warps in problem order, so at any time the warps work on one or two problems
+// (L2 locality).
 struct SddmmDesc {
   int64_t M, K, W;
   const int32_t* row_ptr;
@@ -209,54 +181,67 @@ struct SddmmDesc {
   int64_t out4;
 };
 constexpr int kSddmmMaxBatch = 128;
-constexpr int kSliceChunk = 8;  // slices per work chunk of the batched kernel
 struct SddmmBatch {
   int count;
   SddmmDesc d[kSddmmMaxBatch];
 };
 
-template <int V, bool VEC>
-__global__ void __launch_bounds__(kSddmmWarps * 32)
+template <int V, bool VEC, int KC, bool ARES>
+__global__ void __launch_bounds__(kSddmmWarps * 32, 4)
     sddmm_batched_kernel(const __grid_constant__ SddmmBatch b) {
-  __shared__ int64_t pre[kSddmmMaxBatch + 1];  // prefix of slice-chunk counts
-  __shared__ int64_t nnzs[kSddmmMaxBatch];
+  __shared__ int64_t pre[kSddmmMaxBatch + 1];  // prefix of work items
+  __shared__ int64_t qs[kSddmmMaxBatch];
   const int lane = lane_id();
+  const int64_t n_warps = (int64_t)gridDim.x * kSddmmWarps;
   if (threadIdx.x < 32) {
+    // pass 1: total chunks -> chunks per warp
+    int64_t tot = 0;
+    for (int base = 0; base < b.count; base += 32) {
+      const int p = base + lane;
+      int64_t ch = 0;
+      if (p < b.count) ch = ceil_div64((int64_t)b.d[p].row_ptr[b.d[p].W], 16) + b.d[p].W;
+#pragma unroll
+      for (int o = 16; o >= 1; o >>= 1) ch += __shfl_xor_sync(0xffffffffu, ch, o);
+      tot += ch;
+    }
+    const int64_t per_warp = ceil_div64(tot, n_warps) > 0 ? ceil_div64(tot, n_warps) : 1;
+    // pass 2: items per problem, exclusive prefix
     int64_t carry = 0;
     for (int base = 0; base < b.count; base += 32) {
       const int p = base + lane;
-      const int64_t nz = p < b.count ? (int64_t)b.d[p].row_ptr[b.d[p].W] : 0;
-      const int64_t v = ceil_div64(ceil_div64(nz, 16), kSliceChunk);  // chunks of slices
-      int64_t incl = v;
+      int64_t items = 0, q = 1;
+      if (p < b.count) {
+        const int64_t W = b.d[p].W;
+        const int64_t ch = ceil_div64((int64_t)b.d[p].row_ptr[W], 16) + W;
+        q = sddmm_q(ch, W, per_warp);
+        items = W * q;
+      }
+      int64_t incl = items;
 #pragma unroll
       for (int o = 1; o < 32; o <<= 1) {
         const int64_t x = __shfl_up_sync(0xffffffffu, incl, o);
         if (lane >= o) incl += x;
       }
       if (p < b.count) {
-        pre[p] = carry + incl - v;
-        nnzs[p] = nz;
+        pre[p] = carry + incl - items;
+        qs[p] = q;
       }
       carry += __shfl_sync(0xffffffffu, incl, 31);
     }
     if (lane == 0) pre[b.count] = carry;
   }
   __syncthreads();
-  // Work is dealt in rounds of chunks of kSliceChunk slices: chunk c of the global chunk
-  // sequence goes to warp c % n_warps, so at any time the warps work on neighbouring chunks
-  // (one or two problems resident in L2), instead of every warp touching its own problem.
-  const int64_t n_chunks = pre[b.count];
-  const int64_t n_warps = (int64_t)gridDim.x * kSddmmWarps;
+  const int64_t n_items = pre[b.count];
   const int64_t gw = (int64_t)blockIdx.x * kSddmmWarps + (threadIdx.x >> 5);
   int p = 0;
-  for (int64_t c = gw; c < n_chunks; c += n_warps) {
-    while (pre[p + 1] <= c) ++p;
-    const int64_t s0 = (c - pre[p]) * kSliceChunk;
-    const int64_t slices = ceil_div64(nnzs[p], 16);
-    const int64_t s1 = s0 + kSliceChunk < slices ? s0 + kSliceChunk : slices;
+  for (int64_t it = gw; it < n_items; it += n_warps) {
+    while (pre[p + 1] <= it) ++p;
     const SddmmDesc& d = b.d[p];
-    sddmm_range<V, VEC>(d.M, d.K, d.W, d.row_ptr, d.col_idx, d.A, d.Bt, d.out, d.out4 != 0, s0, s1,
-                        nnzs[p]);
+    const int64_t q = qs[p];
+    const int64_t loc = it - pre[p];
+    const int64_t w = loc / q;
+    sddmm_window<V, VEC, KC, ARES>(d.M, d.K, d.row_ptr, d.col_idx, d.A, d.Bt, d.out, d.out4 != 0, w,
+                             loc - w * q, q);
   }
 }
 
@@ -270,15 +255,41 @@ static int ctas_per_sm(Kern k) {
   return b;
 }
 
-template <int V, bool VEC>
+// Kernel variant of a problem: K block 64 * KC (KC = 2 for K > 64: measured faster than
+// KC = 4 over the DLMC set, tools/tune.py; VS_SDDMM_KC caps it) and whether the A row of a
+// window stays in registers (ARES; unused by the current body, always 0).  Encoded as
+// KC * 2 + ARES.
+static int sddmm_variant(int64_t K, bool vec) {
+  static const int cap = [] {
+    const char* e = std::getenv("VS_SDDMM_KC");
+    const int c = e ? std::atoi(e) : 2;
+    return c >= 2 ? 2 : 1;
+  }();
+  int kc = (!vec || K <= 64) ? 1 : 2;
+  if (kc > cap) kc = cap;
+  return kc * 2;
+}
+
+template <int V, bool VEC, int KC, bool ARES>
 static int sddmm_ctas_per_sm() {
-  static const int n = ctas_per_sm(sddmm_kernel<V, VEC>);
+  static const int n = ctas_per_sm(sddmm_kernel<V, VEC, KC, ARES>);
   return n;
 }
-template <int V, bool VEC>
+template <int V, bool VEC, int KC, bool ARES>
 static int sddmm_batched_ctas_per_sm() {
-  static const int n = ctas_per_sm(sddmm_batched_kernel<V, VEC>);
+  static const int n = ctas_per_sm(sddmm_batched_kernel<V, VEC, KC, ARES>);
   return n;
+}
+
+template <int V, bool VEC, int KC, bool ARES>
+static void launch_sddmm_one(int64_t M, int64_t K, const int32_t* row_ptr, const int32_t* col_idx,
+                             const uint16_t* A, const uint16_t* Bt, uint16_t* out, int num_sms,
+                             cudaStream_t s) {
+  const int64_t W = ceil_div64(M, V);
+  const bool out4 = (reinterpret_cast<uintptr_t>(out) & 3) == 0;
+  dim3 grid((unsigned)(num_sms * sddmm_ctas_per_sm<V, VEC, KC, ARES>()));
+  sddmm_kernel<V, VEC, KC, ARES><<<grid, kSddmmWarps * 32, 0, s>>>(M, K, W, row_ptr, col_idx, A,
+                                                                   Bt, out, out4);
 }
 
 template <int V>
@@ -286,23 +297,33 @@ static cudaError_t launch_sddmm_v(int64_t M, int64_t N, int64_t K, const int32_t
                                   const int32_t* col_idx, const uint16_t* A, const uint16_t* Bt,
                                   uint16_t* out, bool vec, int num_sms, cudaStream_t s) {
   (void)N;
-  const int64_t W = ceil_div64(M, V);
-  dim3 block(kSddmmWarps * 32);
-  const bool out4 = (reinterpret_cast<uintptr_t>(out) & 3) == 0;
-  if (vec) {
-    dim3 grid((unsigned)(num_sms * sddmm_ctas_per_sm<V, true>()));
-    sddmm_kernel<V, true><<<grid, block, 0, s>>>(M, K, W, row_ptr, col_idx, A, Bt, out, out4);
-  } else {
-    dim3 grid((unsigned)(num_sms * sddmm_ctas_per_sm<V, false>()));
-    sddmm_kernel<V, false><<<grid, block, 0, s>>>(M, K, W, row_ptr, col_idx, A, Bt, out, out4);
+  switch ((vec ? 8 : 0) + sddmm_variant(K, vec)) {
+    case 8 + 2: launch_sddmm_one<V, true, 1, false>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s); break;
+    case 8 + 3: launch_sddmm_one<V, true, 1, true>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s); break;
+    case 8 + 4: launch_sddmm_one<V, true, 2, false>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s); break;
+    case 8 + 5: launch_sddmm_one<V, true, 2, true>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s); break;
+    case 3: launch_sddmm_one<V, false, 1, true>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s); break;
+    default: launch_sddmm_one<V, false, 1, false>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s); break;
   }
   return cudaGetLastError();
 }
 
-template <int V, bool VEC>
+template <int V, bool VEC, int KC, bool ARES>
 static void launch_sddmm_batch(const SddmmBatch& b, int num_sms, cudaStream_t s) {
-  dim3 grid((unsigned)(num_sms * sddmm_batched_ctas_per_sm<V, VEC>()));
-  sddmm_batched_kernel<V, VEC><<<grid, kSddmmWarps * 32, 0, s>>>(b);
+  dim3 grid((unsigned)(num_sms * sddmm_batched_ctas_per_sm<V, VEC, KC, ARES>()));
+  sddmm_batched_kernel<V, VEC, KC, ARES><<<grid, kSddmmWarps * 32, 0, s>>>(b);
+}
+
+template <int V>
+static void launch_sddmm_batch_v(const SddmmBatch& b, int code, int num_sms, cudaStream_t s) {
+  switch (code) {
+    case 8 + 2: return launch_sddmm_batch<V, true, 1, false>(b, num_sms, s);
+    case 8 + 3: return launch_sddmm_batch<V, true, 1, true>(b, num_sms, s);
+    case 8 + 4: return launch_sddmm_batch<V, true, 2, false>(b, num_sms, s);
+    case 8 + 5: return launch_sddmm_batch<V, true, 2, true>(b, num_sms, s);
+    case 3: return launch_sddmm_batch<V, false, 1, true>(b, num_sms, s);
+    default: return launch_sddmm_batch<V, false, 1, false>(b, num_sms, s);
+  }
 }
 
 cudaError_t launch_sddmm_batched(int64_t count, const int64_t* M, const int64_t* K, const int* V,
@@ -314,7 +335,8 @@ cudaError_t launch_sddmm_batched(int64_t count, const int64_t* M, const int64_t*
   for (int64_t i = 0; i < count; ++i) {
     const bool vec = (K[i] % 8 == 0) && ((reinterpret_cast<uintptr_t>(A[i]) & 15) == 0) &&
                      ((reinterpret_cast<uintptr_t>(Bt[i]) & 15) == 0);
-    order.push_back({V[i] * 2 + (vec ? 1 : 0), i});
+    // key: V, vector path, kernel variant
+    order.push_back({V[i] * 16 + (vec ? 8 : 0) + sddmm_variant(K[i], vec), i});
   }
   std::stable_sort(order.begin(), order.end(),
                    [](const auto& a, const auto& b) { return a.first < b.first; });
@@ -331,12 +353,12 @@ cudaError_t launch_sddmm_batched(int64_t count, const int64_t* M, const int64_t*
            static_cast<uint16_t*>(out[p]), (reinterpret_cast<uintptr_t>(out[p]) & 3) == 0 ? 1 : 0};
       ++i;
     }
-    const bool vec = key & 1;
-    switch (key >> 1) {
-      case 1: vec ? launch_sddmm_batch<1, true>(batch, num_sms, s) : launch_sddmm_batch<1, false>(batch, num_sms, s); break;
-      case 2: vec ? launch_sddmm_batch<2, true>(batch, num_sms, s) : launch_sddmm_batch<2, false>(batch, num_sms, s); break;
-      case 4: vec ? launch_sddmm_batch<4, true>(batch, num_sms, s) : launch_sddmm_batch<4, false>(batch, num_sms, s); break;
-      default: vec ? launch_sddmm_batch<8, true>(batch, num_sms, s) : launch_sddmm_batch<8, false>(batch, num_sms, s); break;
+    const int code = key & 15;
+    switch (key >> 4) {
+      case 1: launch_sddmm_batch_v<1>(batch, code, num_sms, s); break;
+      case 2: launch_sddmm_batch_v<2>(batch, code, num_sms, s); break;
+      case 4: launch_sddmm_batch_v<4>(batch, code, num_sms, s); break;
+      default: launch_sddmm_batch_v<8>(batch, code, num_sms, s); break;
     }
     const cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
