@@ -170,21 +170,33 @@ def alg_bytes(p, nnz_v, k_ref):
 
 
 def count_launches(bufs):
-    """Kernel launches of one batched step, by the library's grouping rules (vs_api.cu):
-    encode groups by V (3 kernels per group of <= 128 problems: count, scan, compact), SpMM by (V, panel width NC from N, SPLIT from K), SDDMM by V (1 kernel per
-    group of <= 128)."""
+    """Kernel launches of one batched step, by the library's grouping rules: encode groups by
+    V (3 kernels per group of <= 128 problems: count, scan, compact); SpMM (cp.async path,
+    spmm.cu spmm_config) by (V, panel width NC = 1 for N <= 64 else 2, SPLIT from K); SDDMM
+    (sddmm.cu sddmm_variant) by (V, K block KC = 1 for an inner dimension <= 64 else 2)."""
     import math as _m
     from collections import Counter
     def split(K):
         q = K >> 8
         return 16 if q >= 16 else 8 if q >= 8 else 4 if q >= 4 else 2 if q >= 2 else 1
     enc = Counter(b.p.V for b in bufs)
-    sp = Counter((b.p.V, 1, split(b.p.K)) for b in bufs)  # 64-column panels (NC = 1)
-    sd = Counter(b.p.V for b in bufs)
+    sp = Counter((b.p.V, 1 if b.p.N <= 64 else 2, split(b.p.K)) for b in bufs)
+    sd = Counter((b.p.V, 1 if b.p.N <= 64 else 2) for b in bufs)
     per = {"encode": sum(3 * _m.ceil(n / 128) for n in enc.values()),
            "spmm": sum(_m.ceil(n / 128) for n in sp.values()),
            "sddmm": sum(_m.ceil(n / 128) for n in sd.values())}
     return {"per_class": per, "total": sum(per.values())}
+
+
+# Measured on-chip ceiling of the gather both kernels are made of (tools/gather_bench.cu,
+# profiles/r02_gather.md): random 128-byte rows, LDG.128 with 8 lanes per line, 64 warps/SM.
+GATHER_PEAK_GBS = 20494.0
+
+
+def gathered_bytes(p, nnz_v):
+    """Bytes of the gathered dense operand that reach the SMs (rows of B panels in SpMM,
+    rows of Bt in SDDMM): 2 * nnz_v * N per op (V flop per gathered byte)."""
+    return {"encode": 0.0, "spmm": 2.0 * nnz_v * p.N, "sddmm": 2.0 * nnz_v * p.N}
 
 
 # --------------------------------------------------------------- reference (oracle) arm
@@ -504,6 +516,14 @@ def run_ours(args):
     roofline_tensor = {"bound": "tensor", "achieved": tensor_tf, "peak": peaks["bf16_tflops"],
                        "unit": "TFLOP/s", "frac": tensor_tf / peaks["bf16_tflops"],
                        "kernel": dominant}
+    gath = sum(gathered_bytes(b.p, b.nnz_v)[dominant] for b in bufs)
+    gath_gbs = gath / (cls_ms[dominant] * 1e-3) / 1e9 if cls_ms[dominant] else 0.0
+    roofline_gather = {"bound": "l2_gather", "achieved": gath_gbs, "peak": GATHER_PEAK_GBS,
+                       "unit": "GB/s", "frac": gath_gbs / GATHER_PEAK_GBS, "kernel": dominant,
+                       "peak_source": "measured: tools/gather_bench.cu ldg_line (profiles/r02_gather.md)",
+                       "note": "the working set of the DLMC problems is L2-resident after the first "
+                               "touch; the kernels are bound by the random-row gather into the SMs, "
+                               "not by HBM (DESIGN.md 9)"}
 
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": ws, "steps": args.steps,
@@ -522,6 +542,7 @@ def run_ours(args):
                                       f"{len(branches)} concurrent graph branches"},
         "roofline": roofline,
         "roofline_tensor": roofline_tensor,
+        "roofline_gather": roofline_gather,
         "kernels": {k: {"ms_per_step": v, "share": (v / instr_total if instr_total else None),
                         "launches_per_step": launches_per_step["per_class"][k],
                         "tflops": (flops_cls[k] / (v * 1e-3) / 1e12 if v and flops_cls[k] else None),
@@ -854,6 +875,16 @@ def run_c5(args):
                      "frac": ach / peaks["hbm_gbs"], "traffic": None, "kernel": dom,
                      "algorithmic_bytes_per_launch": db, "avg_launch_us": cls[dom] * 1e3,
                      "peak_source": peaks["source"]},
+        "roofline_tensor": {"bound": "tensor", "achieved": (flops_dom := (2.0 * nnzA * V * Np if dom == "spmm"
+                                                                          else 2.0 * nnzM * V * K)) / (cls[dom] * 1e-3) / 1e12,
+                            "peak": peaks["bf16_tflops_sustained"], "unit": "TFLOP/s",
+                            "frac": flops_dom / (cls[dom] * 1e-3) / 1e12 / peaks["bf16_tflops_sustained"],
+                            "kernel": dom, "peak_source": "sustained dense bf16 (MEASURED_PEAKS.json)"},
+        "roofline_gather": {"bound": "l2_gather",
+                            "achieved": (gb := (2.0 * nnzA * Np if dom == "spmm" else 2.0 * nnzM * K)) / (cls[dom] * 1e-3) / 1e9,
+                            "peak": GATHER_PEAK_GBS, "unit": "GB/s",
+                            "frac": gb / (cls[dom] * 1e-3) / 1e9 / GATHER_PEAK_GBS, "kernel": dom,
+                            "peak_source": "measured: tools/gather_bench.cu ldg_line (profiles/r02_gather.md)"},
         "kernels": {k: {"ms": v} for k, v in cls.items()},
         "gpu_launches": 8 * args.steps,
         "clocks": clk,

@@ -134,7 +134,8 @@ def test_spmm_tiny_sweep(vs, V, density):
 
 @pytest.mark.parametrize("V", [1, 2, 4, 8])
 @pytest.mark.parametrize("M,K,N", [(256, 256, 64), (300, 257, 200), (129, 1000, 136),
-                                   (64, 64, 130), (512, 512, 256), (100, 300, 1000)])
+                                   (64, 64, 130), (512, 512, 256), (100, 300, 1000),
+                                   (64, 2100, 72), (33, 4200, 64)])  # SPLIT = 8, 16
 @pytest.mark.parametrize("density", [0.1, 0.5])
 def test_spmm_multitile(vs, V, M, K, N, density):
     rng = gen.make_rng(f"gspmm_mt_{V}_{M}_{K}_{N}_{density}")

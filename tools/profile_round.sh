@@ -13,13 +13,13 @@ ARGS="--steps 1 --warmup 1 --no-baselines --no-cpu --no-e2e --detail gpurun_out/
 # *batched* belong to it (the eager sizing pass uses the single-problem
 # kernels, which the regex excludes).
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none \
-  -k regex:"batched" -c 40 --csv --log-file gpurun_out/launches_${TAG}.csv \
+  -k regex:"batched" -c 60 --csv --log-file gpurun_out/launches_${TAG}.csv \
   python bench.py $ARGS > /dev/null 2>&1
-for K in spmm_batched sddmm_batched encode_count_batched encode_compact_batched; do
+for K in spmm_cp_batched sddmm_batched encode_count_batched encode_compact_batched; do
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:"$K" -c 3 \
     -o /tmp/full_${TAG}_${K} python bench.py $ARGS > /tmp/ncu_${K}.log 2>&1
   python tools/ncu_summary.py full /tmp/full_${TAG}_${K}.ncu-rep > gpurun_out/full_${TAG}_${K}.md
   python tools/ncu_summary.py traffic /tmp/full_${TAG}_${K}.ncu-rep > gpurun_out/traffic_${TAG}_${K}.json
 done
-cp /tmp/full_${TAG}_spmm_batched.ncu-rep gpurun_out/ 2>/dev/null
+ls -la /tmp/*.ncu-rep
 du -sh gpurun_out
