@@ -396,6 +396,7 @@ cudaError_t launch_encode_batched(int64_t count, const int64_t* M, const int64_t
       const int64_t W = ceil_div64(M[p], V[p]);
       const int64_t nb = ceil_div64(W, kEncWarps);
       if (blocks + nb > 0x7fffffffLL) break;
+
       batch.d[batch.count] = {M[p], K[p], W, static_cast<const uint16_t*>(dense[p]), mask[p],
                               row_ptr[p], col_idx[p], static_cast<uint16_t*>(vals[p])};
       batch.first_block[batch.count++] = blocks;

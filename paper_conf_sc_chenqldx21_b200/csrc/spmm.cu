@@ -518,8 +518,21 @@ __device__ __forceinline__ void spmm_cp_body(int64_t M, int64_t N, int64_t W, in
   }
 }
 
+// VS_SPMM_CP_WARPS: resident warps per SM the register allocation is sized for (build-time
+// knob for tools/tune.py variants; 0 = no cap).  24 (80 registers, with D = 2 stages so the
+// rings of 24 warps fit in shared memory): batched DLMC SpMM 443 us, against 621 us
+// uncapped (~140 registers, 16 warps/SM) and 469 us at 32 warps.
+#ifndef VS_SPMM_CP_WARPS
+#define VS_SPMM_CP_WARPS 24
+#endif
+template <int SPLIT>
+struct CpMinBlocks {
+  static constexpr int v = VS_SPMM_CP_WARPS / SpmmCta<SPLIT>::kWarps > 0
+                               ? VS_SPMM_CP_WARPS / SpmmCta<SPLIT>::kWarps : 1;
+};
+
 template <int V, int NC, int SPLIT, int D>
-__global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32)
+__global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32, CpMinBlocks<SPLIT>::v)
     spmm_cp_kernel(int64_t M, int64_t N, int64_t W, int64_t n_wgroups,
                    const int32_t* __restrict__ row_ptr, const int32_t* __restrict__ col_idx,
                    const uint16_t* __restrict__ vals, const uint16_t* __restrict__ B,
@@ -529,7 +542,7 @@ __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32)
 }
 
 template <int V, int NC, int SPLIT, int D>
-__global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32)
+__global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32, CpMinBlocks<SPLIT>::v)
     spmm_cp_batched_kernel(const __grid_constant__ SpmmBatch b) {
   extern __shared__ __align__(128) unsigned char smem[];
   const int64_t total = b.first_block[b.count];
@@ -558,14 +571,14 @@ struct SpmmCfg {
 };
 
 // cp.async path on/off and its ring depth: VS_SPMM_CP = 0 selects the register path,
-// otherwise the number of stages D (3 or 4; default 3).  VS_SPMM_CPNC caps the panel width
+// otherwise the number of stages D (2 or 3; default 2, see VS_SPMM_CP_WARPS; 4 was slower).  VS_SPMM_CPNC caps the panel width
 // (64 * NC columns, NC in {1, 2, 4}; default 2: tools/tune.py over the DLMC batch, batched
 // 502 us (cap 2) vs 569 us (cap 4) vs 650 us (cap 1) vs 629 us for the register path).
 static int spmm_cp_stages() {
   static const int v = [] {
     const char* e = std::getenv("VS_SPMM_CP");
-    const int d = e ? std::atoi(e) : 3;
-    return d <= 0 ? 0 : d <= 3 ? 3 : 4;
+    const int d = e ? std::atoi(e) : 2;
+    return d <= 0 ? 0 : d <= 2 ? 2 : 3;
   }();
   return v;
 }
@@ -637,12 +650,12 @@ static SpmmKernels cp_kernels_of() {
 
 template <int V, int NC, int SPLIT>
 static SpmmKernels cp_pick_d(int d) {
-  if constexpr (SpmmCta<SPLIT>::kWarps * CpRing<V, NC, 3>::kWarpBytes > 227 * 1024) {
-    return cp_kernels_of<V, 1, SPLIT, 3>();  // unreachable: spmm_config shrinks NC first
-  } else if constexpr (SpmmCta<SPLIT>::kWarps * CpRing<V, NC, 4>::kWarpBytes > 227 * 1024) {
-    return cp_kernels_of<V, NC, SPLIT, 3>();
+  if constexpr (SpmmCta<SPLIT>::kWarps * CpRing<V, NC, 2>::kWarpBytes > 227 * 1024) {
+    return cp_kernels_of<V, 1, SPLIT, 2>();  // unreachable: spmm_config shrinks NC first
+  } else if constexpr (SpmmCta<SPLIT>::kWarps * CpRing<V, NC, 3>::kWarpBytes > 227 * 1024) {
+    return cp_kernels_of<V, NC, SPLIT, 2>();
   } else {
-    return d == 4 ? cp_kernels_of<V, NC, SPLIT, 4>() : cp_kernels_of<V, NC, SPLIT, 3>();
+    return d == 2 ? cp_kernels_of<V, NC, SPLIT, 2>() : cp_kernels_of<V, NC, SPLIT, 3>();
   }
 }
 
