@@ -326,10 +326,64 @@ static void launch_sddmm_batch_v(const SddmmBatch& b, int code, int num_sms, cud
   }
 }
 
-cudaError_t launch_sddmm_batched(int64_t count, const int64_t* M, const int64_t* K, const int* V,
-                                 const int32_t* const* row_ptr, const int32_t* const* col_idx,
-                                 const void* const* A, const void* const* Bt, void* const* out,
-                                 int num_sms, cudaStream_t s) {
+bool sddmm_tc_eligible(int64_t K, const void* A, const void* Bt, const void* out);
+cudaError_t launch_sddmm_tc_batched(int64_t count, const int64_t* M, const int64_t* N, const int64_t* K, const int* V,
+                                    const int32_t* const* row_ptr, const int32_t* const* col_idx,
+                                    const void* const* A, const void* const* Bt, void* const* out,
+                                    int num_sms, cudaStream_t s);
+
+// tcgen05 path (sddmm_tc.cu): VS_SDDMM_TC=1 sends problems with K % 8 == 0, K > 0 and
+// 16-byte aligned A, Bt and out_vals to the tensor-core kernel, single and batched calls
+// alike (so both give the same bits).  Default off: measured 1.8-2.5x slower than the
+// mma.sync kernels below over the DLMC set (profiles/r01b_tcgen05.md) --
+// the cp.async shared-memory staging that tcgen05 operands need caps the row gather at
+// ~60 B/clk/SM, below the register path.  Read at every call (tests switch it per call).
+static bool sddmm_tc_on() {
+  const char* e = std::getenv("VS_SDDMM_TC");
+  return e != nullptr && std::atoi(e) != 0;
+}
+
+static cudaError_t launch_sddmm_mma_batched(int64_t count, const int64_t* M, const int64_t* K,
+                                            const int* V, const int32_t* const* row_ptr,
+                                            const int32_t* const* col_idx, const void* const* A,
+                                            const void* const* Bt, void* const* out, int num_sms,
+                                            cudaStream_t s);
+
+cudaError_t launch_sddmm_batched(int64_t count, const int64_t* M, const int64_t* N, const int64_t* K,
+                                 const int* V, const int32_t* const* row_ptr,
+                                 const int32_t* const* col_idx, const void* const* A,
+                                 const void* const* Bt, void* const* out, int num_sms,
+                                 cudaStream_t s) {
+  if (!sddmm_tc_on())
+    return launch_sddmm_mma_batched(count, M, K, V, row_ptr, col_idx, A, Bt, out, num_sms, s);
+  std::vector<int64_t> sel[2];
+  for (int64_t i = 0; i < count; ++i) sel[sddmm_tc_eligible(K[i], A[i], Bt[i], out[i]) ? 1 : 0].push_back(i);
+  for (int path = 0; path < 2; ++path) {
+    if (sel[path].empty()) continue;
+    std::vector<int64_t> m, n, k;
+    std::vector<int> v;
+    std::vector<const int32_t*> rp, ci;
+    std::vector<const void*> a, bt;
+    std::vector<void*> o;
+    for (int64_t i : sel[path]) {
+      m.push_back(M[i]); n.push_back(N[i]); k.push_back(K[i]); v.push_back(V[i]); rp.push_back(row_ptr[i]);
+      ci.push_back(col_idx[i]); a.push_back(A[i]); bt.push_back(Bt[i]); o.push_back(out[i]);
+    }
+    const cudaError_t e =
+        path ? launch_sddmm_tc_batched((int64_t)m.size(), m.data(), n.data(), k.data(), v.data(),
+                                       rp.data(), ci.data(), a.data(), bt.data(), o.data(), num_sms, s)
+             : launch_sddmm_mma_batched((int64_t)m.size(), m.data(), k.data(), v.data(), rp.data(),
+                                        ci.data(), a.data(), bt.data(), o.data(), num_sms, s);
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
+}
+
+static cudaError_t launch_sddmm_mma_batched(int64_t count, const int64_t* M, const int64_t* K,
+                                            const int* V, const int32_t* const* row_ptr,
+                                            const int32_t* const* col_idx, const void* const* A,
+                                            const void* const* Bt, void* const* out, int num_sms,
+                                            cudaStream_t s) {
   // group by (V, vector path); keep the caller's order inside a group
   std::vector<std::pair<int, int64_t>> order;
   for (int64_t i = 0; i < count; ++i) {
@@ -369,6 +423,8 @@ cudaError_t launch_sddmm_batched(int64_t count, const int64_t* M, const int64_t*
 cudaError_t launch_sddmm(int64_t M, int64_t N, int64_t K, int V, const int32_t* row_ptr,
                          const int32_t* col_idx, const void* A, const void* Bt, void* out,
                          int num_sms, cudaStream_t s) {
+  if (sddmm_tc_on() && sddmm_tc_eligible(K, A, Bt, out))
+    return launch_sddmm_tc_batched(1, &M, &N, &K, &V, &row_ptr, &col_idx, &A, &Bt, &out, num_sms, s);
   const uint16_t* a = static_cast<const uint16_t*>(A);
   const uint16_t* b = static_cast<const uint16_t*>(Bt);
   uint16_t* o = static_cast<uint16_t*>(out);

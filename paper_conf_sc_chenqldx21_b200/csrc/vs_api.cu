@@ -19,10 +19,11 @@ cudaError_t launch_spmm_batched(int64_t count, const int64_t* M, const int64_t* 
                                 const int* V, const int32_t* const* row_ptr,
                                 const int32_t* const* col_idx, const void* const* vals,
                                 const void* const* B, void* const* C, int num_sms, cudaStream_t s);
-cudaError_t launch_sddmm_batched(int64_t count, const int64_t* M, const int64_t* K, const int* V,
-                                 const int32_t* const* row_ptr, const int32_t* const* col_idx,
-                                 const void* const* A, const void* const* Bt, void* const* out,
-                                 int num_sms, cudaStream_t s);
+cudaError_t launch_sddmm_batched(int64_t count, const int64_t* M, const int64_t* N, const int64_t* K,
+                                 const int* V, const int32_t* const* row_ptr,
+                                 const int32_t* const* col_idx, const void* const* A,
+                                 const void* const* Bt, void* const* out, int num_sms,
+                                 cudaStream_t s);
 cudaError_t launch_encode_batched(int64_t count, const int64_t* M, const int64_t* K, const int* V,
                                   const void* const* dense, const uint8_t* const* mask,
                                   int32_t* const* row_ptr, int32_t* const* col_idx,
@@ -275,7 +276,7 @@ vs_status_t vs_sddmm_batched(int64_t count, const vs_sddmm_problem_t* problems,
   vs_status_t st = check_device(&info);
   if (st != VS_SUCCESS) return st;
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
-  std::vector<int64_t> M, K;
+  std::vector<int64_t> M, N, K;
   std::vector<int> V;
   std::vector<const int32_t*> rp, ci;
   std::vector<const void*> A, Bt;
@@ -283,11 +284,11 @@ vs_status_t vs_sddmm_batched(int64_t count, const vs_sddmm_problem_t* problems,
   for (int64_t i = 0; i < count; ++i) {
     const vs_sddmm_problem_t& p = problems[i];
     if (p.M == 0 || p.N == 0) continue;
-    M.push_back(p.M); K.push_back(p.K); V.push_back(p.V); rp.push_back(p.row_ptr);
+    M.push_back(p.M); N.push_back(p.N); K.push_back(p.K); V.push_back(p.V); rp.push_back(p.row_ptr);
     ci.push_back(p.col_idx); A.push_back(p.A); Bt.push_back(p.Bt); out.push_back(p.out_vals);
   }
   if (M.empty()) return VS_SUCCESS;
-  return from_cuda(vs::launch_sddmm_batched((int64_t)M.size(), M.data(), K.data(), V.data(), rp.data(),
+  return from_cuda(vs::launch_sddmm_batched((int64_t)M.size(), M.data(), N.data(), K.data(), V.data(), rp.data(),
                                             ci.data(), A.data(), Bt.data(), out.data(),
                                             info.num_sms, s));
 }

@@ -24,6 +24,20 @@ def vs():
     return m
 
 
+@pytest.fixture(params=["mma", "tc"])
+def sddmm_path(request):
+    """Runs an SDDMM test on both kernels: the mma.sync path (default) and the tcgen05/TMEM
+    path (VS_SDDMM_TC=1, read by libvs at every call)."""
+    import os
+    old = os.environ.get("VS_SDDMM_TC")
+    os.environ["VS_SDDMM_TC"] = "1" if request.param == "tc" else "0"
+    yield request.param
+    if old is None:
+        os.environ.pop("VS_SDDMM_TC", None)
+    else:
+        os.environ["VS_SDDMM_TC"] = old
+
+
 def dev(x):
     return torch.from_numpy(np.ascontiguousarray(x)).cuda()
 
@@ -222,7 +236,7 @@ def run_sddmm(vs, mask, A, Bt, V):
 
 @pytest.mark.parametrize("V", [1, 2, 4, 8])
 @pytest.mark.parametrize("density", [0.0, 0.3, 1.0])
-def test_sddmm_tiny_sweep(vs, V, density):
+def test_sddmm_tiny_sweep(vs, sddmm_path, V, density):
     for M, N, K in itertools.product([1, 3, 8, 9, 16], [1, 5, 16, 17], [1, 8, 16, 24, 72]):
         rng = gen.make_rng(f"gsddmm_{V}_{density}_{M}_{N}_{K}")
         mask = gen.colvec_mask(rng, M, N, V, density)
@@ -236,7 +250,7 @@ def test_sddmm_tiny_sweep(vs, V, density):
 @pytest.mark.parametrize("M,N,K", [(256, 64, 256), (300, 257, 200), (129, 1000, 64),
                                    (64, 64, 1000), (512, 512, 128), (100, 300, 13)])
 @pytest.mark.parametrize("density", [0.1, 0.5])
-def test_sddmm_multitile(vs, V, M, N, K, density):
+def test_sddmm_multitile(vs, sddmm_path, V, M, N, K, density):
     rng = gen.make_rng(f"gsddmm_mt_{V}_{M}_{N}_{K}_{density}")
     mask = gen.colvec_mask(rng, M, N, V, density)
     A = gen.dense_operand(rng, M, K)
@@ -247,7 +261,7 @@ def test_sddmm_multitile(vs, V, M, N, K, density):
 
 @pytest.mark.parametrize("V", [1, 2, 4, 8])
 @pytest.mark.parametrize("K", [64, 200, 384])
-def test_sddmm_integer_exact_bitwise(vs, V, K):
+def test_sddmm_integer_exact_bitwise(vs, sddmm_path, V, K):
     rng = gen.make_rng(f"gsddmm_int_{V}_{K}")
     M, N = 61, 90
     mask = gen.colvec_mask(rng, M, N, V, 0.4)
@@ -258,7 +272,7 @@ def test_sddmm_integer_exact_bitwise(vs, V, K):
 
 
 @pytest.mark.parametrize("V", [1, 2, 4, 8])
-def test_sddmm_all_ones_mask_equals_gemm(vs, V):
+def test_sddmm_all_ones_mask_equals_gemm(vs, sddmm_path, V):
     rng = gen.make_rng(f"gsddmm_ones_{V}")
     M, N, K = 64, 96, 128
     mask = np.ones((M, N), np.uint8)
@@ -271,7 +285,7 @@ def test_sddmm_all_ones_mask_equals_gemm(vs, V):
 
 
 @pytest.mark.parametrize("V", [1, 4, 8])
-def test_sddmm_identity_A_bitwise(vs, V):
+def test_sddmm_identity_A_bitwise(vs, sddmm_path, V):
     rng = gen.make_rng(f"gsddmm_eye_{V}")
     M = K = 64
     N = 77
@@ -281,7 +295,7 @@ def test_sddmm_identity_A_bitwise(vs, V):
     assert np.array_equal(out.astype(np.float64), o64)
 
 
-def test_sddmm_degenerate(vs):
+def test_sddmm_degenerate(vs, sddmm_path):
     mask = np.zeros((16, 10), np.uint8)
     rp, ci, _ = vs.encode(4, mask=dev(mask))
     vs.vs_sddmm(16, 10, 32, 4, rp, ci, dev(np.zeros((16, 32), np.float16)),
@@ -294,7 +308,7 @@ def test_sddmm_degenerate(vs):
     assert torch.count_nonzero(out).item() == 0
 
 
-def test_sddmm_padded_rows_are_zero(vs):
+def test_sddmm_padded_rows_are_zero(vs, sddmm_path):
     rng = gen.make_rng("gsddmm_pad")
     M, N, K, V = 13, 40, 64, 8   # last window has 5 padded rows
     mask = gen.colvec_mask(rng, M, N, V, 0.5)
