@@ -14,6 +14,8 @@
 #include <utility>
 #include <vector>
 
+#include <cstdlib>
+
 #include "common.cuh"
 
 namespace vs {
@@ -372,6 +374,16 @@ cudaError_t launch_encode(int64_t M, int64_t K, int V, const void* dense, const 
 }
 
 // Problems with W == 0 are handled by the caller.
+// Input bytes per batched launch triple (count, scan, compact): VS_ENC_CHUNK_MB (0 = no
+// limit, the default).  L2-sized chunks let the compact pass re-read its inputs from L2, but
+// measured slower (tools/tune.py, DLMC batch: no limit 247 us, 96 MB 309 us, 48 MB 424 us,
+// 24 MB 517 us): fewer, wider launches win.
+static int64_t enc_chunk_bytes() {
+  const char* e = std::getenv("VS_ENC_CHUNK_MB");
+  const int64_t mb = e ? std::atoll(e) : 0;
+  return mb * (1LL << 20);
+}
+
 cudaError_t launch_encode_batched(int64_t count, const int64_t* M, const int64_t* K, const int* V,
                                   const void* const* dense, const uint8_t* const* mask,
                                   int32_t* const* row_ptr, int32_t* const* col_idx,
@@ -391,11 +403,16 @@ cudaError_t launch_encode_batched(int64_t count, const int64_t* M, const int64_t
     batch.count = 0;
     int64_t blocks = 0;
     const int threads = kEncWarps * 32;
+    int64_t bytes = 0;
     while (i < order.size() && order[i].first == key && batch.count < kEncMaxBatch) {
       const int64_t p = order[i].second;
       const int64_t W = ceil_div64(M[p], V[p]);
       const int64_t nb = ceil_div64(W, kEncWarps);
       if (blocks + nb > 0x7fffffffLL) break;
+      // L2-sized chunks: the compact pass re-reads the inputs the count pass just read
+      const int64_t pb = M[p] * K[p] * ((dense[p] ? 2 : 0) + (mask[p] ? 1 : 0));
+      if (batch.count > 0 && enc_chunk_bytes() > 0 && bytes + pb > enc_chunk_bytes()) break;
+      bytes += pb;
 
       batch.d[batch.count] = {M[p], K[p], W, static_cast<const uint16_t*>(dense[p]), mask[p],
                               row_ptr[p], col_idx[p], static_cast<uint16_t*>(vals[p])};

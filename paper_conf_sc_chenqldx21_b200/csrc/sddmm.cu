@@ -26,6 +26,11 @@
 namespace vs {
 
 constexpr int kSddmmWarps = 4;
+// resident CTAs per SM the register allocation is sized for (tools/tune.py over the DLMC batch:
+// 4 -> 551 us, 5 -> 516 us (12 B of spills), 6 -> 644 us, 8 -> 782 us: spills in the loop)
+#ifndef VS_SDDMM_MINB
+#define VS_SDDMM_MINB 5
+#endif
 
 template <bool VEC>
 __device__ __forceinline__ void load_seg2(const uint16_t* __restrict__ row, int64_t K, int64_t k,
@@ -150,7 +155,7 @@ __device__ __forceinline__ int64_t sddmm_q(int64_t chunks, int64_t W, int64_t pe
 }
 
 template <int V, bool VEC, int KC, bool ARES>
-__global__ void __launch_bounds__(kSddmmWarps * 32, 4)
+__global__ void __launch_bounds__(kSddmmWarps * 32, VS_SDDMM_MINB)
     sddmm_kernel(int64_t M, int64_t K, int64_t W, const int32_t* __restrict__ row_ptr,
                  const int32_t* __restrict__ col_idx, const uint16_t* __restrict__ A,
                  const uint16_t* __restrict__ Bt, uint16_t* __restrict__ out, bool out4) {
@@ -187,7 +192,7 @@ struct SddmmBatch {
 };
 
 template <int V, bool VEC, int KC, bool ARES>
-__global__ void __launch_bounds__(kSddmmWarps * 32, 4)
+__global__ void __launch_bounds__(kSddmmWarps * 32, VS_SDDMM_MINB)
     sddmm_batched_kernel(const __grid_constant__ SddmmBatch b) {
   __shared__ int64_t pre[kSddmmMaxBatch + 1];  // prefix of work items
   __shared__ int64_t qs[kSddmmMaxBatch];
