@@ -99,6 +99,38 @@ vs_status_t vs_encode_colvec(int64_t M, int64_t K, int V,
                              int64_t* nnz_vec_host, vs_stream_t stream);
 
 /*
+ * vs_transpose_colvec — column-vector encoding (grain V) of A^T [K x M] from the encoding
+ * of A [M x K].  The training-side operand: with Y = W X (SpMM), the
+ * backward pass needs dX = W^T dY, "W^T ... encode[d] with our column-vector sparse
+ * encoding" (§8 Case 1; the transposed operand of the Discussion).
+ *
+ *   Window kw of A^T covers columns kw*V .. kw*V+V-1 of A; vector (kw, m) holds
+ *   A[m][kw*V + j], j < V (j with kw*V + j >= K is padding, +0.0).  It is kept iff one of
+ *   its V fp16 bit patterns is nonzero (vals != NULL; the keep rule of vs_encode_colvec, so
+ *   the result is bit-identical to encoding the dense transpose), or iff the A vector it
+ *   comes from is stored (vals == NULL: pattern-only transpose of a mask, no valsT).  For
+ *   patterns of square V x V blocks each block gives exactly V vectors.
+ *
+ *   row_ptr[W+1], col_idx[nnz_v], vals[nnz_v*V] (or NULL): A, W = ceil(M/V); col_idx must
+ *     not repeat inside a window (the encoder's output satisfies this).
+ *   rowT_ptr : int32 [ceil(K/V) + 1] output, always written.
+ *   colT_idx : int32 [nnzT] output (ascending m inside each window), or NULL = count mode.
+ *   valsT    : fp16 [nnzT * V] output (requires vals), or NULL.
+ *   workspace: device buffer of vs_transpose_colvec_workspace(M, K, V) bytes (int32
+ *              aligned), scratch for the call.
+ *   nnzT_host: if non-NULL, the call synchronises `stream` and stores rowT_ptr[ceil(K/V)].
+ *   Count mode (colT_idx == NULL) writes rowT_ptr only; full mode needs colT_idx / valsT
+ *   capacities >= nnzT (from a count-mode call, or the bound ceil(K/V) * M).
+ *   Deterministic: no atomics on outputs (the workspace collects per-(column group,
+ *   window) row masks with atomicOr, which is order-independent).
+ */
+int64_t vs_transpose_colvec_workspace(int64_t M, int64_t K, int V);
+vs_status_t vs_transpose_colvec(int64_t M, int64_t K, int V,
+                                const int32_t* row_ptr, const int32_t* col_idx, const void* vals,
+                                int32_t* rowT_ptr, int32_t* colT_idx, void* valsT,
+                                void* workspace, int64_t* nnzT_host, vs_stream_t stream);
+
+/*
  * vs_spmm — C[M x N] = A[M x K] * B[K x N], A sparse in column-vector CSR.
  * Problem statement §4.1 P:571-588 (B, C row-major; A in CSR); kernel §5.3-5.4
  * P:846-921 (each output tile V x TileN).

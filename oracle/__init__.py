@@ -114,6 +114,25 @@ def decode(M: int, K: int, V: int, row_ptr, col_idx, vals) -> np.ndarray:
     return out.view(np.float16)
 
 
+def transpose(M: int, K: int, V: int, row_ptr, col_idx, vals=None):
+    """Column-vector encoding (grain V) of A^T [K x M] from the encoding of A [M x K]: by
+    definition, the encoding of the dense transpose (Discussion: C^T "under
+    column-vector sparse encoding"; §8 Case 1: "encode both W and W^T with our
+    column-vector sparse encoding").  With vals None the transpose is of the pattern: every
+    stored vector's rows (< M) count as nonzero.  Returns (rowT, colT, valsT or None)."""
+    if vals is not None:
+        dense = decode(M, K, V, row_ptr, col_idx, vals)
+        return encode(K, M, V, dense=np.ascontiguousarray(dense.T))
+    mask = np.zeros((M, K), dtype=np.uint8)
+    W = len(row_ptr) - 1
+    for w in range(W):
+        for p in range(int(row_ptr[w]), int(row_ptr[w + 1])):
+            for r in range(V):
+                if w * V + r < M:
+                    mask[w * V + r, int(col_idx[p])] = 1
+    return encode(K, M, V, mask=np.ascontiguousarray(mask.T))
+
+
 def spmm(M: int, K: int, N: int, V: int, row_ptr, col_idx, vals, B):
     """Returns (C64 [M,N] float64, S64 [M,N] float64 = sum |a*b|)."""
     B16 = _f16(B)

@@ -94,6 +94,11 @@ def load():
             L.vs_spmm.argtypes = [_I64, _I64, _I64, ctypes.c_int, _P, _P, _P, _P, _P, _P]
             L.vs_sddmm.restype = ctypes.c_int
             L.vs_sddmm.argtypes = [_I64, _I64, _I64, ctypes.c_int, _P, _P, _P, _P, _P, _P]
+            L.vs_transpose_colvec_workspace.restype = _I64
+            L.vs_transpose_colvec_workspace.argtypes = [_I64, _I64, ctypes.c_int]
+            L.vs_transpose_colvec.restype = ctypes.c_int
+            L.vs_transpose_colvec.argtypes = [_I64, _I64, ctypes.c_int, _P, _P, _P, _P, _P, _P, _P,
+                                              ctypes.POINTER(ctypes.c_int64), _P]
             L.vs_softmax_colvec.restype = ctypes.c_int
             L.vs_softmax_colvec.argtypes = [_I64, ctypes.c_int, _P, _P, _P, ctypes.c_float, _P]
             for name, st in (("vs_spmm_batched", SpmmProblem), ("vs_sddmm_batched", SddmmProblem),
@@ -174,6 +179,26 @@ def vs_sddmm(M, N, K, V, row_ptr, col_idx, A, Bt, out_vals, stream=None):
                          _ptr(Bt, torch.float16, "Bt"), _ptr(out_vals, torch.float16, "out_vals"),
                          _stream(stream))
     _check(st, "vs_sddmm")
+
+
+def vs_transpose_colvec_workspace(M, K, V) -> int:
+    return int(load().vs_transpose_colvec_workspace(int(M), int(K), int(V)))
+
+
+def vs_transpose_colvec(M, K, V, row_ptr, col_idx, vals, rowT_ptr, colT_idx=None, valsT=None,
+                        workspace=None, want_nnz=False, stream=None):
+    """Mirror of vs_transpose_colvec.  Count mode when colT_idx
+    is None.  Returns nnzT when ``want_nnz`` (the call then synchronises), else None."""
+    import torch
+    nnz = ctypes.c_int64(-1)
+    st = load().vs_transpose_colvec(
+        int(M), int(K), int(V), _ptr(row_ptr, torch.int32, "row_ptr"),
+        _ptr(col_idx, torch.int32, "col_idx"), _ptr(vals, torch.float16, "vals"),
+        _ptr(rowT_ptr, torch.int32, "rowT_ptr"), _ptr(colT_idx, torch.int32, "colT_idx"),
+        _ptr(valsT, torch.float16, "valsT"), _ptr(workspace, None, "workspace"),
+        ctypes.byref(nnz) if want_nnz else None, _stream(stream))
+    _check(st, "vs_transpose_colvec")
+    return int(nnz.value) if want_nnz else None
 
 
 def vs_softmax_colvec(M, V, row_ptr, vals, out, scale, stream=None):
@@ -298,6 +323,24 @@ def encode(V, dense=None, mask=None, capacity=None, stream=None):
                      col_idx if capacity > 0 else None, vals if capacity > 0 else None,
                      stream=stream)
     return row_ptr, col_idx, vals
+
+
+def transpose(row_ptr, col_idx, vals, M, K, V, stream=None):
+    """Column-vector encoding of A^T [K x M] from that of A [M x K] (vals None: pattern
+    only).  Returns (rowT_ptr, colT_idx, valsT); one count-mode call sizes the outputs."""
+    import torch
+    dev = row_ptr.device
+    KT = num_windows(K, V)
+    rowT = torch.empty(KT + 1, dtype=torch.int32, device=dev)
+    ws = torch.empty(max(vs_transpose_colvec_workspace(M, K, V), 4), dtype=torch.uint8, device=dev)
+    n = vs_transpose_colvec(M, K, V, row_ptr, col_idx, vals, rowT, workspace=ws, want_nnz=True,
+                            stream=stream)
+    colT = torch.empty(max(n, 1), dtype=torch.int32, device=dev)
+    valsT = torch.empty(max(n, 1) * V, dtype=torch.float16, device=dev) if vals is not None else None
+    if n > 0:  # (n == 0: rowT is complete and there is nothing else to write)
+        vs_transpose_colvec(M, K, V, row_ptr, col_idx, vals, rowT, colT, valsT, workspace=ws,
+                            stream=stream)
+    return rowT, colT[:n], (valsT[:n * V] if valsT is not None else None)
 
 
 def spmm(row_ptr, col_idx, vals, B, M, V, out=None, stream=None):

@@ -33,6 +33,10 @@ cudaError_t launch_softmax(int64_t M, int V, const int32_t* row_ptr, const void*
 cudaError_t launch_softmax_batched(int64_t count, const int64_t* M, const int* V,
                                    const int32_t* const* row_ptr, const void* const* vals,
                                    void* const* out, const float* scale, cudaStream_t s);
+int64_t transpose_workspace_bytes(int64_t M, int64_t K, int V);
+cudaError_t launch_transpose(int64_t M, int64_t K, int V, const int32_t* row_ptr,
+                             const int32_t* col_idx, const void* vals, int32_t* rowT, int32_t* colT,
+                             void* valsT, void* workspace, int num_sms, cudaStream_t s);
 }  // namespace vs
 
 namespace {
@@ -186,6 +190,40 @@ vs_status_t vs_sddmm(int64_t M, int64_t N, int64_t K, int V, const int32_t* row_
   if (st != VS_SUCCESS) return st;
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   return from_cuda(vs::launch_sddmm(M, N, K, V, row_ptr, col_idx, A, Bt, out_vals, info.num_sms, s));
+}
+
+int64_t vs_transpose_colvec_workspace(int64_t M, int64_t K, int V) {
+  if (!valid_v(V) || M < 0 || K < 0) return 0;
+  return vs::transpose_workspace_bytes(M, K, V);
+}
+
+vs_status_t vs_transpose_colvec(int64_t M, int64_t K, int V, const int32_t* row_ptr,
+                                const int32_t* col_idx, const void* vals, int32_t* rowT_ptr,
+                                int32_t* colT_idx, void* valsT, void* workspace,
+                                int64_t* nnzT_host, vs_stream_t stream) {
+  if (!valid_v(V) || M < 0 || K < 0 || rowT_ptr == nullptr) return VS_ERROR_INVALID_VALUE;
+  if (valsT != nullptr && (vals == nullptr || colT_idx == nullptr)) return VS_ERROR_INVALID_VALUE;
+  const int64_t W = (M + V - 1) / V;
+  if (W > 0 && K > 0 && (row_ptr == nullptr || workspace == nullptr)) return VS_ERROR_INVALID_VALUE;
+  if (M >= (int64_t(1) << 23)) return VS_ERROR_NOT_SUPPORTED;  // packed 23-bit prefixes
+  if (!al(rowT_ptr, 4) || (row_ptr && !al(row_ptr, 4)) || (col_idx && !al(col_idx, 4)) ||
+      (colT_idx && !al(colT_idx, 4)) || (workspace && !al(workspace, 4)))
+    return VS_ERROR_MISALIGNED;
+  if ((vals && !al(vals, 2)) || (valsT && !al(valsT, 2))) return VS_ERROR_MISALIGNED;
+  DevInfo info;
+  vs_status_t st = check_device(&info);
+  if (st != VS_SUCCESS) return st;
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  st = from_cuda(vs::launch_transpose(M, K, V, row_ptr, col_idx, vals, rowT_ptr, colT_idx, valsT,
+                                      workspace, info.num_sms, s));
+  if (st != VS_SUCCESS || nnzT_host == nullptr) return st;
+  int32_t n = 0;
+  const int64_t KT = (K + V - 1) / V;
+  if (cudaMemcpyAsync(&n, rowT_ptr + KT, 4, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+      cudaStreamSynchronize(s) != cudaSuccess)
+    return VS_ERROR_CUDA;
+  *nnzT_host = n;
+  return VS_SUCCESS;
 }
 
 vs_status_t vs_softmax_colvec(int64_t M, int V, const int32_t* row_ptr, const void* vals,

@@ -92,6 +92,19 @@ def colvec_dense(rng: np.random.Generator, M: int, K: int, V: int, density: floa
     return np.ascontiguousarray(full.astype(np.float16))
 
 
+def block_dense(rng: np.random.Generator, M: int, K: int, V: int, density: float,
+                exact: bool = False) -> np.ndarray:
+    """fp16 [M, K] made of square V x V nonzero blocks (each kept with probability
+    ``density``): the pattern under which both W and W^T are column-vector encodings
+    (§8 Case 1)."""
+    W = -(-M // V) if M > 0 else 0
+    KB = -(-K // V) if K > 0 else 0
+    keep = rng.random((W, KB)) < density
+    full = np.repeat(np.repeat(keep, V, axis=0), V, axis=1)[:M, :K]
+    vals = fp16_values(rng, (M, K), exact=exact)
+    return np.ascontiguousarray(np.where(full, vals, np.float16(0.0)).astype(np.float16))
+
+
 def colvec_mask(rng: np.random.Generator, M: int, N: int, V: int, density: float,
                 kind: str = "bern") -> np.ndarray:
     """uint8 [M, N] binary mask made of V x 1 column vectors (the SDDMM mask D)."""
