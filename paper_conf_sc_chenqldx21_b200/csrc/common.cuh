@@ -147,6 +147,11 @@ __device__ __forceinline__ void cp_async_zfill(uint32_t dst, const void* src, ui
                  : "memory");
   }
 }
+// 16-byte cp.async that allocates in L1 (.ca): gathered rows re-read by other CTAs of the SM
+__device__ __forceinline__ void cp_async_ca16_zfill(uint32_t dst, const void* src, uint32_t src_size) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(src_size)
+               : "memory");
+}
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
 template <int N>
 __device__ __forceinline__ void cp_async_wait() {

@@ -332,6 +332,11 @@ __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32)
 //  * epilogue: stmatrix.x4.trans turns the accumulator tiles into row-major 16-byte pieces
 //    of the V x 64NC output tile (swizzled, in the drained ring), then 16-byte stores.
 // Wider panels (NC = 2, 4) amortise the per-group bookkeeping over more gathered bytes.
+// VS_SPMM_CA: gathered B rows copied with cp.async.ca (L1-allocating) instead of .cg
+// (measured 1.18x slower over the batched DLMC SpMM: the rings leave little L1)
+#ifndef VS_SPMM_CA
+#define VS_SPMM_CA 0
+#endif
 template <int V, int NC, int D>
 struct CpRing {
   static constexpr int kRowBytes = 16 * 128 * NC;  // one group: 16 slots x 64NC columns fp16
@@ -396,8 +401,13 @@ __device__ __forceinline__ void spmm_cp_body(int64_t M, int64_t N, int64_t W, in
 #pragma unroll
         for (int h = 0; h < NC; ++h) {
           const bool ok = okp && (n0 + 64 * h + 8 * cc < N);
+#if VS_SPMM_CA
+          cp_async_ca16_zfill(rs + sl * (128 * NC) + ((8 * h + (cc ^ (sl & 7))) * 16),
+                              ok ? (const void*)(src + 64 * h) : (const void*)B, ok ? 16u : 0u);
+#else
           cp_async_zfill<16>(rs + sl * (128 * NC) + ((8 * h + (cc ^ (sl & 7))) * 16),
                              ok ? (const void*)(src + 64 * h) : (const void*)B, ok ? 16u : 0u);
+#endif
         }
       }
       if (lane < 16) {
