@@ -49,6 +49,9 @@ def parse_args(argv=None):
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--workload", default=DEFAULT_WORKLOAD)
+    ap.add_argument("--schedule", choices=["chains", "phases"], default="chains",
+                    help="batched step as one chain per V group on concurrent branches, or as "
+                         "three phases (encode, then SpMM || SDDMM)")
     ap.add_argument("--no-baselines", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
@@ -397,6 +400,42 @@ def run_ours(args):
         if post:
             post()
 
+    # the same batched calls scheduled as one chain per V group (encode -> SpMM || SDDMM of
+    # that group), the chains on concurrent graph branches: a group's SpMM/SDDMM overlap the
+    # other groups' encode and fill each other's tails.  Same kernels, same work, same bits.
+    groups = {}
+    for b in bufs:
+        groups.setdefault(b.p.V, []).append(b)
+    chain_arrs = []
+    for V in sorted(groups):
+        gb = groups[V]
+        chain_arrs.append((
+            vs.make_encode_batch([(b.p.M, b.p.K, b.p.V, b.Wd, None, b.row_ptr, b.col_idx, b.vals) for b in gb]),
+            vs.make_spmm_batch([(b.p.M, b.p.K, b.p.N, b.p.V, b.row_ptr, b.col_idx, b.vals, b.X, b.Y) for b in gb]),
+            vs.make_sddmm_batch([(b.p.M, b.p.K, b.p.N, b.p.V, b.row_ptr, b.col_idx, b.G, b.X, b.dW) for b in gb])))
+    chain_streams = [(torch.cuda.Stream(), torch.cuda.Stream()) for _ in chain_arrs]
+
+    def step_chains(pre=None, post=None):
+        cur = torch.cuda.current_stream()
+        if pre:
+            pre()
+        for (enc_a, sp_a, sd_a), (s_main, s_side) in zip(chain_arrs, chain_streams):
+            s_main.wait_stream(cur)
+            with torch.cuda.stream(s_main):
+                vs.vs_encode_colvec_batched(enc_a)
+                s_side.wait_stream(s_main)
+                vs.vs_spmm_batched(sp_a)
+            with torch.cuda.stream(s_side):
+                vs.vs_sddmm_batched(sd_a)
+        for s_main, s_side in chain_streams:
+            cur.wait_stream(s_main)
+            cur.wait_stream(s_side)
+        if post:
+            post()
+
+    step_main, step_alt = ((step_chains, step_batched) if args.schedule == "chains"
+                           else (step_batched, step_chains))
+
     # per-problem calls (single entry points) on 8 concurrent graph branches: comparison only
     branches = [torch.cuda.Stream() for _ in range(max(1, args.streams))]
 
@@ -426,7 +465,8 @@ def run_ours(args):
             e0.record()
             ev.append((name, s0, e0))
 
-    g_step = capture(torch, step_batched, stream)
+    g_step = capture(torch, step_main, stream)
+    g_alt = capture(torch, step_alt, stream)
     g_pp = capture(torch, step_per_problem, stream)
     g_instr = capture(torch, step_instr, stream)
     flush = torch.empty(512 * 1024 * 1024 // 4, dtype=torch.int32, device=dev)
@@ -435,6 +475,7 @@ def run_ours(args):
         with torch.cuda.stream(stream):
             flush.fill_(i)
             g_step.replay()
+            g_alt.replay()
             g_pp.replay()
             g_instr.replay()
     stream.synchronize()
@@ -459,6 +500,11 @@ def run_ours(args):
             ends[i].record()
     torch.cuda.synchronize()
     step_ms = [s0.elapsed_time(e0) for s0, e0 in zip(starts, ends)]
+    alt_ms = []
+    for i in range(args.steps):
+        with torch.cuda.stream(stream):
+            flush.fill_(i + 3)
+        alt_ms.append(time_graph(torch, g_alt, stream))
     pp_ms = []
     for i in range(args.steps):
         with torch.cuda.stream(stream):
@@ -534,9 +580,14 @@ def run_ours(args):
                              "x S{.5,.7,.9,.98} x N{64,128,256}" if args.workload == "dlmc_layer" else args.workload,
                    "step": "per problem: encode W -> SpMM Y=WX -> SDDMM dW=(G X^T) o pattern(W)",
                    "flops_per_step": flops_step, "l2": "flushed between timed steps (512 MiB write, untimed)",
-                   "launch": "batched C ABI (vs_*_batched), step replayed as one CUDA graph; "
-                             "SDDMM batch on a forked branch concurrent with the SpMM batch",
+                   "launch": "batched C ABI (vs_*_batched), step replayed as one CUDA graph; " + (
+                             "one chain per V group (encode -> SpMM || SDDMM), chains on concurrent "
+                             "graph branches" if args.schedule == "chains" else
+                             "encode batch, then SpMM batch || SDDMM batch"),
                    "accumulate": "fp32"},
+        "alt_schedule": {"schedule": "phases" if args.schedule == "chains" else "chains",
+                         "ms_per_step": sum(alt_ms) / args.steps,
+                         "value": ws * flops_step / (sum(alt_ms) / args.steps * 1e-3) / 1e12},
         "per_problem_calls": {"ms_per_step": ms_pp, "value": ws * flops_step / (ms_pp * 1e-3) / 1e12,
                               "note": "same step through the single-problem entry points, "
                                       f"{len(branches)} concurrent graph branches"},
@@ -568,7 +619,7 @@ def run_ours(args):
             for b in bufs:
                 b.h_Y.copy_(b.Y, non_blocking=True)
                 b.h_dW.copy_(b.dW[:b.nnz_v * b.p.V], non_blocking=True)
-        g_e2e = capture(torch, lambda: step_batched(h2d, d2h), stream)
+        g_e2e = capture(torch, lambda: step_main(h2d, d2h), stream)
         with torch.cuda.stream(stream):
             g_e2e.replay()
         stream.synchronize()
