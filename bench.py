@@ -1023,6 +1023,125 @@ def run_attention(args):
     return 0
 
 
+def run_train(args):
+    """NEXT items: one training step of sparse layers with square V x V block
+    patterns (§8 Case 1): per layer, W^T's values refreshed from W's on the
+    device (vs_transpose_colvec_values; the pattern of W^T is built once by
+    vs_transpose_colvec, W's values change every step), Y = W X (vs_spmm), dX = W^T dY
+    (vs_spmm on the transposed encoding), dW = (dY X^T) o pattern(W) (vs_sddmm).  Workload
+    name: train[_s<S>] (default S = 0.9); layers = the DLMC (M, K) shapes x V in {2, 4, 8},
+    batch N = 256.  Compared with the dense fp16 step (torch.matmul: W X, W^T dY, dY X^T)."""
+    import re
+    import torch
+    import paper_conf_sc_chenqldx21_b200 as vs
+    from synth import gen
+    from synth.workloads import DLMC_MK
+
+    m = re.match(r"train(?:_s([0-9.]+))?$", args.workload)
+    S = float(m.group(1) or 0.9)
+    N = 256
+    torch.cuda.set_device(0)
+    dev = torch.device("cuda", 0)
+    vs.load()
+    layers = []
+    for (M, K) in DLMC_MK:
+        for V in (2, 4, 8):
+            rng = gen.make_rng(f"train_{M}_{K}_{V}_{S}")
+            Wd = torch.from_numpy(gen.block_dense(rng, M, K, V, 1 - S)).to(dev)
+            X = torch.from_numpy(gen.dense_operand(rng, K, N)).to(dev)
+            dY = torch.from_numpy(gen.dense_operand(rng, M, N)).to(dev)
+            rp, ci, va = vs.encode(V, dense=Wd)
+            nnz = int(rp[-1].item())
+            rT, cT, vT = vs.transpose(rp, ci[:nnz], va[:nnz * V], M, K, V)
+            nT = int(rT[-1].item())
+            ws = torch.empty(max(vs.vs_transpose_colvec_workspace(M, K, V), 4), dtype=torch.uint8, device=dev)
+            layers.append(dict(M=M, K=K, V=V, Wd=Wd, X=X, dY=dY, rp=rp, ci=ci[:nnz], va=va[:nnz * V],
+                               rT=rT, cT=torch.empty(max(nT, 1), dtype=torch.int32, device=dev),
+                               vT=torch.empty(max(nT, 1) * V, dtype=torch.float16, device=dev),
+                               ws=ws, nnz=nnz, nT=nT,
+                               Y=torch.empty((M, N), dtype=torch.float16, device=dev),
+                               dX=torch.empty((K, N), dtype=torch.float16, device=dev),
+                               dW=torch.empty(max(nnz, 1) * V, dtype=torch.float16, device=dev)))
+    sp_f = vs.make_spmm_batch([(L["M"], L["K"], N, L["V"], L["rp"], L["ci"], L["va"], L["X"], L["Y"])
+                               for L in layers])
+    sp_b = vs.make_spmm_batch([(L["K"], L["M"], N, L["V"], L["rT"], L["cT"], L["vT"], L["dY"], L["dX"])
+                               for L in layers])
+    sd = vs.make_sddmm_batch([(L["M"], L["K"], N, L["V"], L["rp"], L["ci"], L["dY"], L["X"], L["dW"])
+                              for L in layers])
+
+    # graph branches: the per-layer transposes (small, launch-bound kernels) spread over 4
+    # branches, then dX = W^T dY; Y = W X and dW on a parallel branch (they do not need W^T)
+    tr_streams = [torch.cuda.Stream() for _ in range(4)]
+    fw = torch.cuda.Stream()
+
+    def step():
+        cur = torch.cuda.current_stream()
+        fw.wait_stream(cur)
+        with torch.cuda.stream(fw):
+            vs.vs_spmm_batched(sp_f)
+            vs.vs_sddmm_batched(sd)
+        for i, L in enumerate(layers):
+            st = tr_streams[i % len(tr_streams)]
+            if i < len(tr_streams):
+                st.wait_stream(cur)
+            with torch.cuda.stream(st):
+                vs.vs_transpose_colvec_values(L["M"], L["K"], L["V"], L["rp"], L["ci"], L["va"],
+                                              L["rT"], L["vT"], L["ws"])
+        for st in tr_streams:
+            cur.wait_stream(st)
+        vs.vs_spmm_batched(sp_b)
+        cur.wait_stream(fw)
+
+    def dense():
+        for L in layers:
+            torch.matmul(L["Wd"], L["X"])
+            torch.matmul(L["Wd"].t(), L["dY"])
+            torch.matmul(L["dY"], L["X"].t())
+
+    # the pattern of W^T is fixed (pruned weights): one full transpose per layer before the
+    # steps; every step refreshes W^T's values from W's (vs_transpose_colvec_values)
+    for L in layers:
+        vs.vs_transpose_colvec(L["M"], L["K"], L["V"], L["rp"], L["ci"], L["va"], L["rT"], L["cT"],
+                               L["vT"], workspace=L["ws"])
+    # parity spot check of the step's transposed operand against a dense transpose product
+    stream = torch.cuda.Stream()
+    with torch.cuda.stream(stream):
+        step()
+    stream.synchronize()
+    L0 = layers[-1]
+    ref = torch.matmul(L0["Wd"].t().float(), L0["dY"].float())
+    assert torch.allclose(L0["dX"].float(), ref, rtol=2e-2, atol=2e-2), "train: dX mismatch"
+    g = capture(torch, step, stream)
+    gd = capture(torch, dense, stream)
+    with torch.cuda.stream(stream):
+        for _ in range(max(3, args.warmup)):
+            g.replay()
+            gd.replay()
+    stream.synchronize()
+    clocks = ClockSampler(0).start()
+    t_sparse = min(time_graph(torch, g, stream) for _ in range(max(1, args.steps)))
+    t_dense = min(time_graph(torch, gd, stream) for _ in range(max(1, args.steps)))
+    clk = clocks.stop()
+    # transpose kernels per layer: rowT memset + P memset + mark + colscan + scan + zero + place
+    flops = sum(3 * 2.0 * L["nnz"] * L["V"] * N for L in layers)
+    line = {"metric": METRIC, "value": flops / (t_sparse * 1e-3) / 1e12, "unit": UNIT, "n_gpus": 1,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": t_sparse,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f16",
+            "data": "synthetic",
+            "config": {"workload": args.workload, "layers": len(layers), "batch_N": N, "sparsity": S,
+                       "pattern": "square V x V blocks (P:1633-1636)",
+                       "step": "per layer: W^T values refreshed from W's (vs_transpose_colvec_values; "
+                               "the W^T pattern is built once by vs_transpose_colvec), Y = W X, "
+                               "dX = W^T dY (vs_spmm), dW = (dY X^T) o pattern(W) (vs_sddmm)",
+                       "schedule": "transposes on 4 graph branches -> dX batch; Y and dW batches on "
+                                   "a parallel branch",
+                       "l2": "warm (per-step graph timing, min of steps)"},
+            "dense_step_ms": t_dense, "speedup_vs_dense": t_dense / t_sparse,
+            "gpu_launches": len(layers) * 2 + 3 * 3, "clocks": clk, "e2e": None}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
 def main(argv=None):
     args = parse_args(argv)
     if args.impl == "reference":
@@ -1031,6 +1150,8 @@ def main(argv=None):
         return run_c5(args)
     if args.workload.startswith("attention"):
         return run_attention(args)
+    if args.workload.startswith("train"):
+        return run_train(args)
     return run_ours(args)
 
 

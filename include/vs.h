@@ -125,6 +125,17 @@ vs_status_t vs_encode_colvec(int64_t M, int64_t K, int V,
  *   window) row masks with atomicOr, which is order-independent).
  */
 int64_t vs_transpose_colvec_workspace(int64_t M, int64_t K, int V);
+/*
+ * vs_transpose_colvec_values — refreshes valsT for new values of A with an unchanged
+ * pattern (a training step updates W's values, not its pattern): rowT_ptr / colT_idx and the
+ * workspace must come from a previous full-mode vs_transpose_colvec call on the same row_ptr
+ * / col_idx.  valsT[q*V + j] = A[colT_idx[q]][kw*V + j] from the new vals for every vector q
+ * of that pattern (elements of A that are not stored give +0.0).  Two kernels, asynchronous.
+ */
+vs_status_t vs_transpose_colvec_values(int64_t M, int64_t K, int V,
+                                       const int32_t* row_ptr, const int32_t* col_idx,
+                                       const void* vals, const int32_t* rowT_ptr, void* valsT,
+                                       const void* workspace, vs_stream_t stream);
 vs_status_t vs_transpose_colvec(int64_t M, int64_t K, int V,
                                 const int32_t* row_ptr, const int32_t* col_idx, const void* vals,
                                 int32_t* rowT_ptr, int32_t* colT_idx, void* valsT,

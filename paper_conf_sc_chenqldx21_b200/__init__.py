@@ -99,6 +99,8 @@ def load():
             L.vs_transpose_colvec.restype = ctypes.c_int
             L.vs_transpose_colvec.argtypes = [_I64, _I64, ctypes.c_int, _P, _P, _P, _P, _P, _P, _P,
                                               ctypes.POINTER(ctypes.c_int64), _P]
+            L.vs_transpose_colvec_values.restype = ctypes.c_int
+            L.vs_transpose_colvec_values.argtypes = [_I64, _I64, ctypes.c_int, _P, _P, _P, _P, _P, _P, _P]
             L.vs_softmax_colvec.restype = ctypes.c_int
             L.vs_softmax_colvec.argtypes = [_I64, ctypes.c_int, _P, _P, _P, ctypes.c_float, _P]
             for name, st in (("vs_spmm_batched", SpmmProblem), ("vs_sddmm_batched", SddmmProblem),
@@ -199,6 +201,18 @@ def vs_transpose_colvec(M, K, V, row_ptr, col_idx, vals, rowT_ptr, colT_idx=None
         ctypes.byref(nnz) if want_nnz else None, _stream(stream))
     _check(st, "vs_transpose_colvec")
     return int(nnz.value) if want_nnz else None
+
+
+def vs_transpose_colvec_values(M, K, V, row_ptr, col_idx, vals, rowT_ptr, valsT, workspace,
+                               stream=None):
+    """Mirror of vs_transpose_colvec_values: new values, same transposed pattern."""
+    import torch
+    st = load().vs_transpose_colvec_values(
+        int(M), int(K), int(V), _ptr(row_ptr, torch.int32, "row_ptr"),
+        _ptr(col_idx, torch.int32, "col_idx"), _ptr(vals, torch.float16, "vals"),
+        _ptr(rowT_ptr, torch.int32, "rowT_ptr"), _ptr(valsT, torch.float16, "valsT"),
+        _ptr(workspace, None, "workspace"), _stream(stream))
+    _check(st, "vs_transpose_colvec_values")
 
 
 def vs_softmax_colvec(M, V, row_ptr, vals, out, scale, stream=None):

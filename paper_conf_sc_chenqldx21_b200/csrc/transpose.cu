@@ -148,6 +148,31 @@ __global__ void __launch_bounds__(kTrWarps * 32)
   }
 }
 
+// values refresh of an existing transposed pattern: like tr_place_kernel, but the rows
+// placed are those present in the packed mask of P (the pattern of the previous full call)
+__global__ void __launch_bounds__(kTrWarps * 32)
+    tr_place_values_kernel(int64_t M, int V, int64_t W, const int32_t* __restrict__ row_ptr,
+                           const int32_t* __restrict__ col_idx, const uint16_t* __restrict__ vals,
+                           const int32_t* __restrict__ P, const int32_t* __restrict__ rowT,
+                           uint16_t* __restrict__ valsT) {
+  const int64_t w = (int64_t)blockIdx.x * kTrWarps + (threadIdx.x >> 5);
+  if (w >= W) return;
+  const int lane = lane_id();
+  const int64_t pb = row_ptr[w], pe = row_ptr[w + 1];
+  for (int64_t p = pb + lane; p < pe; p += 32) {
+    const int32_t k = ldg32i(col_idx + p);
+    const int64_t kw = k / V;
+    const int32_t e = P[kw * W + w];
+    const uint32_t mask = (uint32_t)e & 0xFF;
+    const int64_t base = (int64_t)rowT[kw] + (e >> 8);
+    for (int r = 0; r < V; ++r) {
+      if (!((mask >> r) & 1u)) continue;
+      const int64_t pos = base + __popc(mask & ((1u << r) - 1u));
+      valsT[pos * V + (k - kw * V)] = ldg16(vals + p * V + r);
+    }
+  }
+}
+
 // zero valsT[0 .. rowT[KT] * V) (the size is only known on the device)
 __global__ void tr_zero_kernel(const int32_t* __restrict__ rowT, int64_t KT, int V,
                                uint16_t* __restrict__ valsT) {
@@ -155,6 +180,21 @@ __global__ void tr_zero_kernel(const int32_t* __restrict__ rowT, int64_t KT, int
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
        i += (int64_t)gridDim.x * blockDim.x)
     valsT[i] = 0;
+}
+
+// values refresh: the pattern (rowT, colT) and the packed prefixes in P come from a previous
+// full call with the same workspace; only valsT is rewritten from the new vals
+cudaError_t launch_transpose_values(int64_t M, int64_t K, int V, const int32_t* row_ptr,
+                                    const int32_t* col_idx, const void* vals, const int32_t* rowT,
+                                    void* valsT, const void* workspace, int num_sms, cudaStream_t s) {
+  const int64_t W = ceil_div64(M, V), KT = ceil_div64(K, V);
+  if (W == 0 || KT == 0) return cudaSuccess;
+  tr_zero_kernel<<<num_sms * 4, 256, 0, s>>>(rowT, KT, V, static_cast<uint16_t*>(valsT));
+  // pattern bits from the stored vectors (HAS_VALS = false): every stored row < M is placed
+  tr_place_values_kernel<<<(unsigned)ceil_div64(W, kTrWarps), kTrWarps * 32, 0, s>>>(
+      M, V, W, row_ptr, col_idx, static_cast<const uint16_t*>(vals),
+      static_cast<const int32_t*>(workspace), rowT, static_cast<uint16_t*>(valsT));
+  return cudaGetLastError();
 }
 
 int64_t transpose_workspace_bytes(int64_t M, int64_t K, int V) {

@@ -37,6 +37,9 @@ int64_t transpose_workspace_bytes(int64_t M, int64_t K, int V);
 cudaError_t launch_transpose(int64_t M, int64_t K, int V, const int32_t* row_ptr,
                              const int32_t* col_idx, const void* vals, int32_t* rowT, int32_t* colT,
                              void* valsT, void* workspace, int num_sms, cudaStream_t s);
+cudaError_t launch_transpose_values(int64_t M, int64_t K, int V, const int32_t* row_ptr,
+                                    const int32_t* col_idx, const void* vals, const int32_t* rowT,
+                                    void* valsT, const void* workspace, int num_sms, cudaStream_t s);
 }  // namespace vs
 
 namespace {
@@ -224,6 +227,26 @@ vs_status_t vs_transpose_colvec(int64_t M, int64_t K, int V, const int32_t* row_
     return VS_ERROR_CUDA;
   *nnzT_host = n;
   return VS_SUCCESS;
+}
+
+vs_status_t vs_transpose_colvec_values(int64_t M, int64_t K, int V, const int32_t* row_ptr,
+                                       const int32_t* col_idx, const void* vals,
+                                       const int32_t* rowT_ptr, void* valsT, const void* workspace,
+                                       vs_stream_t stream) {
+  if (!valid_v(V) || M < 0 || K < 0 || rowT_ptr == nullptr) return VS_ERROR_INVALID_VALUE;
+  if (M == 0 || K == 0) return VS_SUCCESS;
+  if (row_ptr == nullptr || workspace == nullptr || vals == nullptr || valsT == nullptr)
+    return VS_ERROR_INVALID_VALUE;
+  if (M >= (int64_t(1) << 23)) return VS_ERROR_NOT_SUPPORTED;
+  if (!al(rowT_ptr, 4) || !al(row_ptr, 4) || (col_idx && !al(col_idx, 4)) || !al(workspace, 4) ||
+      !al(vals, 2) || !al(valsT, 2))
+    return VS_ERROR_MISALIGNED;
+  DevInfo info;
+  vs_status_t st = check_device(&info);
+  if (st != VS_SUCCESS) return st;
+  return from_cuda(vs::launch_transpose_values(M, K, V, row_ptr, col_idx, vals, rowT_ptr, valsT,
+                                               workspace, info.num_sms,
+                                               reinterpret_cast<cudaStream_t>(stream)));
 }
 
 vs_status_t vs_softmax_colvec(int64_t M, int V, const int32_t* row_ptr, const void* vals,

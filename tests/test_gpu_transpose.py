@@ -110,3 +110,30 @@ def test_backward_dx_through_spmm(vs, V, M, K, N):
     X64, S64 = oracle.spmm(K, M, N, V, oT, ocT, ovT, dY)
     err = np.abs(dX.float().cpu().numpy().astype(np.float64) - X64)
     assert np.all(err <= oracle.tolerance(S64)), f"max err {err.max()}"
+
+
+@pytest.mark.parametrize("V", [1, 2, 4, 8])
+@pytest.mark.parametrize("blocks", [False, True])
+def test_transpose_values_refresh(vs, V, blocks):
+    # a training step changes W's values, not its pattern: vs_transpose_colvec_values rewrites
+    # valsT in place and must equal the oracle transpose of the new values (no new zeros)
+    rng = gen.make_rng(f"gtr_vals_{V}_{blocks}")
+    M, K = 37 * V + 3, 29 * V + 5
+    W1 = (gen.block_dense(rng, M, K, V, 0.3) if blocks else gen.colvec_dense(rng, M, K, V, 0.3))
+    W2 = np.where(W1 != 0, gen.dense_operand(rng, M, K), np.float16(0)).astype(np.float16)
+    rp, ci, va = vs.encode(V, dense=dev(W1))
+    n = int(rp[-1].item())
+    rT, cT, vT = vs.transpose(rp, ci[:n], va[:n * V], M, K, V)
+    ws = torch.empty(max(vs.vs_transpose_colvec_workspace(M, K, V), 4), dtype=torch.uint8, device="cuda")
+    nT = int(rT[-1].item())
+    cT2 = torch.empty(max(nT, 1), dtype=torch.int32, device="cuda")
+    vT2 = torch.empty(max(nT, 1) * V, dtype=torch.float16, device="cuda")
+    vs.vs_transpose_colvec(M, K, V, rp, ci[:n], va[:n * V], rT, cT2, vT2, workspace=ws)
+    rp2, ci2, va2 = vs.encode(V, dense=dev(W2))
+    assert torch.equal(rp2, rp) and torch.equal(ci2[:n], ci[:n])
+    vs.vs_transpose_colvec_values(M, K, V, rp, ci[:n], va2[:n * V], rT, vT2, ws)
+    torch.cuda.synchronize()
+    orp, oci, ova = oracle.encode(M, K, V, dense=W2)
+    oT, ocT, ovT = oracle.transpose(M, K, V, orp, oci, ova)
+    assert np.array_equal(rT.cpu().numpy(), oT) and np.array_equal(cT2[:nT].cpu().numpy(), ocT)
+    assert np.array_equal(vT2[:nT * V].cpu().numpy().view(np.uint16), ovT.view(np.uint16))
