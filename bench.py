@@ -176,7 +176,7 @@ def count_launches(bufs):
     """Kernel launches of one batched step, by the library's grouping rules: encode groups by
     V (3 kernels per group of <= 128 problems: count, scan, compact); SpMM (cp.async path,
     spmm.cu spmm_config) by (V, panel width NC = 1 for N <= 64 else 2, SPLIT from K); SDDMM
-    (sddmm.cu sddmm_variant) by (V, K block KC = 1 for an inner dimension <= 64 else 2)."""
+    (sddmm.cu sddmm_variant) by V (one kernel serves both K-block variants)."""
     import math as _m
     from collections import Counter
     def split(K):
@@ -184,7 +184,7 @@ def count_launches(bufs):
         return 16 if q >= 16 else 8 if q >= 8 else 4 if q >= 4 else 2 if q >= 2 else 1
     enc = Counter(b.p.V for b in bufs)
     sp = Counter((b.p.V, 1 if b.p.N <= 64 else 2, split(b.p.K)) for b in bufs)
-    sd = Counter((b.p.V, 1 if b.p.N <= 64 else 2) for b in bufs)
+    sd = Counter(b.p.V for b in bufs)  # one mixed-K kernel per V (sddmm_window_any)
     per = {"encode": sum(3 * _m.ceil(n / 128) for n in enc.values()),
            "spmm": sum(_m.ceil(n / 128) for n in sp.values()),
            "sddmm": sum(_m.ceil(n / 128) for n in sd.values())}

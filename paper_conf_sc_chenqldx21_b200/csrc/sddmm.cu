@@ -146,6 +146,27 @@ __device__ __forceinline__ void sddmm_window(int64_t M, int64_t K,
   }
 }
 
+// ARES slot = "mixed K blocks": one kernel serves both K <= 64 (KC = 1 body) and K > 64
+// (KC = 2 body), chosen per problem at run time, so a batch needs one launch per V instead of
+// one per (V, KC) group (no tail between the two launches).  Same bodies, same bits.
+template <int V, bool VEC, int KC, bool ARES>
+__device__ __forceinline__ void sddmm_window_any(int64_t M, int64_t K,
+                                                 const int32_t* __restrict__ row_ptr,
+                                                 const int32_t* __restrict__ col_idx,
+                                                 const uint16_t* __restrict__ A,
+                                                 const uint16_t* __restrict__ Bt,
+                                                 uint16_t* __restrict__ out, bool out4, int64_t w,
+                                                 int64_t j0, int64_t q) {
+  if constexpr (ARES && VEC) {
+    if (K <= 64)
+      sddmm_window<V, VEC, 1, false>(M, K, row_ptr, col_idx, A, Bt, out, out4, w, j0, q);
+    else
+      sddmm_window<V, VEC, 2, false>(M, K, row_ptr, col_idx, A, Bt, out, out4, w, j0, q);
+  } else {
+    sddmm_window<V, VEC, KC, ARES>(M, K, row_ptr, col_idx, A, Bt, out, out4, w, j0, q);
+  }
+}
+
 // Work items of one problem: W windows x q warps per window (warp j of window w takes the
 // window's 16-vector chunks j, j + q, ...); q = the number of warps per window that gives
 // every warp of the launch about the same number of chunks.
@@ -167,7 +188,7 @@ __global__ void __launch_bounds__(kSddmmWarps * 32, VS_SDDMM_MINB)
   const int64_t items = W * q;
   for (int64_t it = gw; it < items; it += n_warps) {
     const int64_t w = it / q;
-    sddmm_window<V, VEC, KC, ARES>(M, K, row_ptr, col_idx, A, Bt, out, out4, w, it - w * q, q);
+    sddmm_window_any<V, VEC, KC, ARES>(M, K, row_ptr, col_idx, A, Bt, out, out4, w, it - w * q, q);
   }
 }
 
@@ -245,8 +266,8 @@ __global__ void __launch_bounds__(kSddmmWarps * 32, VS_SDDMM_MINB)
     const int64_t q = qs[p];
     const int64_t loc = it - pre[p];
     const int64_t w = loc / q;
-    sddmm_window<V, VEC, KC, ARES>(d.M, d.K, d.row_ptr, d.col_idx, d.A, d.Bt, d.out, d.out4 != 0, w,
-                             loc - w * q, q);
+    sddmm_window_any<V, VEC, KC, ARES>(d.M, d.K, d.row_ptr, d.col_idx, d.A, d.Bt, d.out,
+                                       d.out4 != 0, w, loc - w * q, q);
   }
 }
 
@@ -262,7 +283,7 @@ static int ctas_per_sm(Kern k) {
 
 // Kernel variant of a problem: K block 64 * KC (KC = 2 for K > 64: measured faster than
 // KC = 4 over the DLMC set, tools/tune.py; VS_SDDMM_KC caps it) and whether the A row of a
-// window stays in registers (ARES; unused by the current body, always 0).  Encoded as
+// window stays in registers -- the ARES slot now selects the mixed-K kernel (sddmm_window_any).  Encoded as
 // KC * 2 + ARES.
 static int sddmm_variant(int64_t K, bool vec) {
   static const int cap = [] {
@@ -272,6 +293,12 @@ static int sddmm_variant(int64_t K, bool vec) {
   }();
   int kc = (!vec || K <= 64) ? 1 : 2;
   if (kc > cap) kc = cap;
+  // VS_SDDMM_MIX (default 1): vector-path problems of any K share the mixed kernel
+  static const bool mix = [] {
+    const char* e = std::getenv("VS_SDDMM_MIX");
+    return e ? std::atoi(e) != 0 : true;
+  }();
+  if (vec && mix && cap == 2) return 2 * 2 + 1;
   return kc * 2;
 }
 
