@@ -13,7 +13,7 @@ ARGS="--steps 1 --warmup 1 --no-baselines --no-cpu --no-e2e --detail gpurun_out/
 # *batched* belong to it (the eager sizing pass uses the single-problem
 # kernels, which the regex excludes).
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none \
-  -k regex:"batched" -c 66 --csv --log-file gpurun_out/launches_${TAG}.csv \
+  -k regex:"batched" -c 60 --csv --log-file gpurun_out/launches_${TAG}.csv \
   python bench.py $ARGS > /dev/null 2>&1
 for K in spmm_cp_batched sddmm_batched encode_count_batched encode_compact_batched; do
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:"$K" -c 3 \

@@ -17,7 +17,7 @@ k = d["kernels"]
 with open(os.path.join(pr, f"{tag}_launches.md"), "w") as f:
     f.write(f"# {tag} — ncu launch list of the batched bench step (dlmc_layer, 144 problems)\n\n")
     f.write("Command: tools/profile_round.sh (ncu --metrics gpu__time_duration.sum --clock-control none "
-            "-k regex:batched -c 66: two full steps). Per-launch times are cold-cache and serialised: compare shares. "
+            "-k regex:batched -c 60: two full steps of 30 launches, the chains schedule then the phases schedule). Per-launch times are cold-cache and serialised: compare shares. "
             "Live in-graph CUDA-event times of the same step (bench.py): "
             + ", ".join(f"{c} {v['ms_per_step']:.3f} ms" for c, v in k.items())
             + f" per step; step {d['ms_per_step']:.3f} ms = {d['value']:.2f} TFLOP/s.\n\n")
