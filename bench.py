@@ -192,8 +192,8 @@ def count_launches(bufs):
 
 
 # Measured on-chip ceiling of the gather both kernels are made of (tools/gather_bench.cu,
-# profiles/r02_gather.md): random 128-byte rows, LDG.128 with 8 lanes per line, 64 warps/SM.
-GATHER_PEAK_GBS = 20494.0
+# profiles/r01e_gather.md): random 128-byte rows, LDG.128 with 8 lanes per line, 64 warps/SM.
+GATHER_PEAK_GBS = 20674.0
 
 
 def gathered_bytes(p, nnz_v):
@@ -566,7 +566,7 @@ def run_ours(args):
     gath_gbs = gath / (cls_ms[dominant] * 1e-3) / 1e9 if cls_ms[dominant] else 0.0
     roofline_gather = {"bound": "l2_gather", "achieved": gath_gbs, "peak": GATHER_PEAK_GBS,
                        "unit": "GB/s", "frac": gath_gbs / GATHER_PEAK_GBS, "kernel": dominant,
-                       "peak_source": "measured: tools/gather_bench.cu ldg_line (profiles/r02_gather.md)",
+                       "peak_source": "measured: tools/gather_bench.cu ldg_line (profiles/r01e_gather.md)",
                        "note": "the working set of the DLMC problems is L2-resident after the first "
                                "touch; the kernels are bound by the random-row gather into the SMs, "
                                "not by HBM (DESIGN.md 9)"}
@@ -935,7 +935,7 @@ def run_c5(args):
                             "achieved": (gb := (2.0 * nnzA * Np if dom == "spmm" else 2.0 * nnzM * K)) / (cls[dom] * 1e-3) / 1e9,
                             "peak": GATHER_PEAK_GBS, "unit": "GB/s",
                             "frac": gb / (cls[dom] * 1e-3) / 1e9 / GATHER_PEAK_GBS, "kernel": dom,
-                            "peak_source": "measured: tools/gather_bench.cu ldg_line (profiles/r02_gather.md)"},
+                            "peak_source": "measured: tools/gather_bench.cu ldg_line (profiles/r01e_gather.md)"},
         "kernels": {k: {"ms": v} for k, v in cls.items()},
         "gpu_launches": 8 * args.steps,
         "clocks": clk,
