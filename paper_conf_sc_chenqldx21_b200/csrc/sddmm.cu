@@ -146,6 +146,54 @@ __device__ __forceinline__ void sddmm_window(int64_t M, int64_t K,
   }
 }
 
+// K <= 64 body with TWO of the warp's chunks in flight per round trip (v0 and v0 + 16q):
+// 8 LDG.128 per thread before the first MMA instead of 4, so a warp keeps twice the gather
+// bytes in flight at the same occupancy (register cost = the KC = 2 body's).  Each chunk's
+// accumulation order is the KC = 1 body's, so the bits are identical.
+template <int V>
+__device__ __forceinline__ void sddmm_window_pair(int64_t M, int64_t K,
+                                                  const int32_t* __restrict__ row_ptr,
+                                                  const int32_t* __restrict__ col_idx,
+                                                  const uint16_t* __restrict__ A,
+                                                  const uint16_t* __restrict__ Bt,
+                                                  uint16_t* __restrict__ out, bool out4, int64_t w,
+                                                  int64_t j0, int64_t q) {
+  const int lane = lane_id();
+  const int g = lane >> 2, t = lane & 3;
+  const int64_t kt = 8 * t;
+  const int64_t pb = row_ptr[w], pe = row_ptr[w + 1];
+  int64_t v0 = pb + 16 * j0;
+  if (v0 >= pe) return;
+  const int64_t arow = w * V + g;
+  const bool ok_row = (g < V) && (arow < M);
+  const int64_t sq = 16 * q;
+  auto col = [&](int64_t v) { return (v < pe) ? ldg32i(col_idx + v) : 0; };
+  int c0a = col(v0 + g), c0b = col(v0 + g + 8), c1a = col(v0 + sq + g), c1b = col(v0 + sq + g + 8);
+  uint4 xx0, xx1;
+  load_seg2<true>(A + arow * K, K, kt, ok_row, xx0, xx1);
+  for (; v0 < pe; v0 += 2 * sq) {
+    const int64_t v1 = v0 + sq, n0 = v0 + 2 * sq, n1 = n0 + sq;
+    const int n0a = col(n0 + g), n0b = col(n0 + g + 8), n1a = col(n1 + g), n1b = col(n1 + g + 8);
+    uint4 a0[2], a1[2], b0[2], b1[2];
+    load_seg2<true>(Bt + (int64_t)c0a * K, K, kt, v0 + g < pe, a0[0], a1[0]);
+    load_seg2<true>(Bt + (int64_t)c0b * K, K, kt, v0 + g + 8 < pe, b0[0], b1[0]);
+    load_seg2<true>(Bt + (int64_t)c1a * K, K, kt, v1 + g < pe, a0[1], a1[1]);
+    load_seg2<true>(Bt + (int64_t)c1b * K, K, kt, v1 + g + 8 < pe, b0[1], b1[1]);
+    float acc0[4] = {0.f, 0.f, 0.f, 0.f}, acc1[4] = {0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+    for (int j = 0; j < 4; ++j)
+      mma_16816(acc0, wordj(a0[0], j), wordj(b0[0], j), wordj(a1[0], j), wordj(b1[0], j),
+                wordj(xx0, j), wordj(xx1, j));
+#pragma unroll
+    for (int j = 0; j < 4; ++j)
+      mma_16816(acc1, wordj(a0[1], j), wordj(b0[1], j), wordj(a1[1], j), wordj(b1[1], j),
+                wordj(xx0, j), wordj(xx1, j));
+    store_chunk<V>(acc0, v0, pe, w, M, g, t, out, out4);
+    if (v1 < pe) store_chunk<V>(acc1, v1, pe, w, M, g, t, out, out4);
+    c0a = n0a; c0b = n0b; c1a = n1a; c1b = n1b;
+  }
+}
+
 // ARES slot = "mixed K blocks": one kernel serves both K <= 64 (KC = 1 body) and K > 64
 // (KC = 2 body), chosen per problem at run time, so a batch needs one launch per V instead of
 // one per (V, KC) group (no tail between the two launches).  Same bodies, same bits.
@@ -156,9 +204,11 @@ __device__ __forceinline__ void sddmm_window_any(int64_t M, int64_t K,
                                                  const uint16_t* __restrict__ A,
                                                  const uint16_t* __restrict__ Bt,
                                                  uint16_t* __restrict__ out, bool out4, int64_t w,
-                                                 int64_t j0, int64_t q) {
+                                                 int64_t j0, int64_t q, bool pair) {
   if constexpr (ARES && VEC) {
-    if (K <= 64)
+    if (K <= 64 && pair)
+      sddmm_window_pair<V>(M, K, row_ptr, col_idx, A, Bt, out, out4, w, j0, q);
+    else if (K <= 64)
       sddmm_window<V, VEC, 1, false>(M, K, row_ptr, col_idx, A, Bt, out, out4, w, j0, q);
     else
       sddmm_window<V, VEC, 2, false>(M, K, row_ptr, col_idx, A, Bt, out, out4, w, j0, q);
@@ -179,7 +229,8 @@ template <int V, bool VEC, int KC, bool ARES>
 __global__ void __launch_bounds__(kSddmmWarps * 32, VS_SDDMM_MINB)
     sddmm_kernel(int64_t M, int64_t K, int64_t W, const int32_t* __restrict__ row_ptr,
                  const int32_t* __restrict__ col_idx, const uint16_t* __restrict__ A,
-                 const uint16_t* __restrict__ Bt, uint16_t* __restrict__ out, bool out4) {
+                 const uint16_t* __restrict__ Bt, uint16_t* __restrict__ out, bool out4,
+                 bool pair) {
   const int64_t nnz = row_ptr[W];
   const int64_t n_warps = (int64_t)gridDim.x * kSddmmWarps;
   const int64_t gw = (int64_t)blockIdx.x * kSddmmWarps + (threadIdx.x >> 5);
@@ -188,7 +239,8 @@ __global__ void __launch_bounds__(kSddmmWarps * 32, VS_SDDMM_MINB)
   const int64_t items = W * q;
   for (int64_t it = gw; it < items; it += n_warps) {
     const int64_t w = it / q;
-    sddmm_window_any<V, VEC, KC, ARES>(M, K, row_ptr, col_idx, A, Bt, out, out4, w, it - w * q, q);
+    sddmm_window_any<V, VEC, KC, ARES>(M, K, row_ptr, col_idx, A, Bt, out, out4, w, it - w * q, q,
+                                       pair);
   }
 }
 
@@ -209,6 +261,7 @@ struct SddmmDesc {
 constexpr int kSddmmMaxBatch = 128;
 struct SddmmBatch {
   int count;
+  int pair;  // K <= 64 problems take two chunks per round trip (sddmm_window_pair)
   SddmmDesc d[kSddmmMaxBatch];
 };
 
@@ -267,7 +320,7 @@ __global__ void __launch_bounds__(kSddmmWarps * 32, VS_SDDMM_MINB)
     const int64_t loc = it - pre[p];
     const int64_t w = loc / q;
     sddmm_window_any<V, VEC, KC, ARES>(d.M, d.K, d.row_ptr, d.col_idx, d.A, d.Bt, d.out,
-                                       d.out4 != 0, w, loc - w * q, q);
+                                       d.out4 != 0, w, loc - w * q, q, b.pair != 0);
   }
 }
 
@@ -302,6 +355,16 @@ static int sddmm_variant(int64_t K, bool vec) {
   return kc * 2;
 }
 
+// VS_SDDMM_PAIR (default 1): K <= 64 problems of the mixed-K kernel keep two chunks in flight
+// per warp (sddmm_window_pair); 0 selects the one-chunk body.  Same bits either way.
+static bool sddmm_pair_on() {
+  static const bool on = [] {
+    const char* e = std::getenv("VS_SDDMM_PAIR");
+    return e ? std::atoi(e) != 0 : true;
+  }();
+  return on;
+}
+
 template <int V, bool VEC, int KC, bool ARES>
 static int sddmm_ctas_per_sm() {
   static const int n = ctas_per_sm(sddmm_kernel<V, VEC, KC, ARES>);
@@ -321,7 +384,7 @@ static void launch_sddmm_one(int64_t M, int64_t K, const int32_t* row_ptr, const
   const bool out4 = (reinterpret_cast<uintptr_t>(out) & 3) == 0;
   dim3 grid((unsigned)(num_sms * sddmm_ctas_per_sm<V, VEC, KC, ARES>()));
   sddmm_kernel<V, VEC, KC, ARES><<<grid, kSddmmWarps * 32, 0, s>>>(M, K, W, row_ptr, col_idx, A,
-                                                                   Bt, out, out4);
+                                                                   Bt, out, out4, sddmm_pair_on());
 }
 
 template <int V>
@@ -435,6 +498,7 @@ static cudaError_t launch_sddmm_mma_batched(int64_t count, const int64_t* M, con
   std::stable_sort(order.begin(), order.end(),
                    [](const auto& a, const auto& b) { return a.first < b.first; });
   SddmmBatch batch;
+  batch.pair = sddmm_pair_on() ? 1 : 0;
   size_t i = 0;
   while (i < order.size()) {
     const int key = order[i].first;
