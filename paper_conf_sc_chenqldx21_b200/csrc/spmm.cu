@@ -52,6 +52,17 @@ __device__ __forceinline__ uint32_t word(const uint4& v, int j) {
   return j == 0 ? v.x : (j == 1 ? v.y : (j == 2 ? v.z : v.w));
 }
 
+// Programmatic dependent launch between the launches of ONE batched call (independent
+// problems, disjoint outputs): every block lets the next launch of the batch start as soon as
+// it is running (the next kernel fills the SMs this one's last wave leaves idle), and waits
+// for the previous launch of the batch to complete before it exits, so a launch completes only
+// after all earlier launches of the batch did and whatever follows on the stream sees every
+// result.  Both are no-ops for a launch made without the PDL attribute (the batch's first).
+__device__ __forceinline__ void pdl_launch_dependents() {
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+__device__ __forceinline__ void pdl_wait_prior() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+
 // SPLIT warps cooperate on one (window, panel) unit: warp part q takes the 16-vector groups
 // q, q + SPLIT, ... and the partial accumulators are summed through shared memory by a
 // fixed pairwise tree (deterministic).  A CTA has max(4, SPLIT) warps = max(1, 4/SPLIT) units.
@@ -298,6 +309,7 @@ __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32)
     spmm_batched_kernel(const __grid_constant__ SpmmBatch b) {
   // grid-stride over the blocks of all problems (launched with one CTA per block, so usually
   // one iteration); the first problem by binary search, then a forward linear advance
+  pdl_launch_dependents();
   const int64_t total = b.first_block[b.count];
   int p = first_problem(b.first_block, b.count, (int64_t)blockIdx.x);
   for (int64_t bid = blockIdx.x; bid < total; bid += gridDim.x) {
@@ -306,6 +318,7 @@ __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32)
     spmm_body<V, NC, VEC, SPLIT, UNROLL>(d.M, d.N, d.W, d.n_wgroups, bid - b.first_block[p],
                                          d.row_ptr, d.col_idx, d.vals, d.B, d.C);
   }
+  pdl_wait_prior();
 }
 
 // ---------------------------------------------------- cp.async-staged kernel (default path)
@@ -555,6 +568,7 @@ template <int V, int NC, int SPLIT, int D>
 __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32, CpMinBlocks<SPLIT>::v)
     spmm_cp_batched_kernel(const __grid_constant__ SpmmBatch b) {
   extern __shared__ __align__(128) unsigned char smem[];
+  pdl_launch_dependents();
   const int64_t total = b.first_block[b.count];
   int p = first_problem(b.first_block, b.count, (int64_t)blockIdx.x);
   for (int64_t bid = blockIdx.x; bid < total; bid += gridDim.x) {
@@ -563,6 +577,7 @@ __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32, CpMinBlocks<SPLIT
     spmm_cp_body<V, NC, SPLIT, D>(d.M, d.N, d.W, d.n_wgroups, bid - b.first_block[p], d.row_ptr,
                                   d.col_idx, d.vals, d.B, d.C, smem);
   }
+  pdl_wait_prior();
 }
 
 // Kernel configuration of one problem.  NC (64- or 128-column panels) follows N; SPLIT
@@ -769,6 +784,16 @@ cudaError_t launch_spmm(int64_t M, int64_t K, int64_t N, int V, const int32_t* r
   return cudaGetLastError();
 }
 
+// VS_SPMM_PDL (default 1): the launches of one batched call after the first use programmatic
+// dependent launch (pdl_*); 0 launches them plainly.  Same kernels, same bits.
+static bool spmm_pdl_on() {
+  static const bool on = [] {
+    const char* e = std::getenv("VS_SPMM_PDL");
+    return e ? std::atoi(e) != 0 : true;
+  }();
+  return on;
+}
+
 // problems with K == 0 are handled by the caller (zero fill); M == 0 or N == 0 skipped.
 cudaError_t launch_spmm_batched(int64_t count, const int64_t* M, const int64_t* K, const int64_t* N,
                                 const int* V, const int32_t* const* row_ptr,
@@ -783,6 +808,7 @@ cudaError_t launch_spmm_batched(int64_t count, const int64_t* M, const int64_t* 
                    [](const auto& a, const auto& b) { return a.first < b.first; });
   SpmmBatch batch;
   size_t i = 0;
+  int launched = 0;
   while (i < order.size()) {
     const SpmmCfg c = order[i].first;
     const SpmmKernels k = pick(c);
@@ -806,7 +832,26 @@ cudaError_t launch_spmm_batched(int64_t count, const int64_t* M, const int64_t* 
     batch.first_block[batch.count] = blocks;
     // one CTA per block (measured slightly faster than a resident-sized grid-stride grid)
     (void)num_sms;
-    if (blocks > 0) k.batched<<<(unsigned)blocks, k.threads, k.smem, s>>>(batch);
+    if (blocks > 0) {
+      if (launched > 0 && spmm_pdl_on()) {
+        // later launches of the batch overlap the tail of the previous one (see pdl_*)
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3((unsigned)blocks);
+        cfg.blockDim = dim3((unsigned)k.threads);
+        cfg.dynamicSmemBytes = (size_t)k.smem;
+        cfg.stream = s;
+        cudaLaunchAttribute attr[1];
+        attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        attr[0].val.programmaticStreamSerializationAllowed = 1;
+        cfg.attrs = attr;
+        cfg.numAttrs = 1;
+        const cudaError_t le = cudaLaunchKernelEx(&cfg, k.batched, batch);
+        if (le != cudaSuccess) return le;
+      } else {
+        k.batched<<<(unsigned)blocks, k.threads, k.smem, s>>>(batch);
+      }
+      ++launched;
+    }
     const cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
   }
