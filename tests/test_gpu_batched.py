@@ -115,3 +115,31 @@ def test_batched_rejects_bad_entry_before_launch(vs):
     x = torch.zeros(8, dtype=torch.int32, device="cuda")
     with pytest.raises(vs.VSError):
         vs.vs_spmm_batched([(8, 8, 8, 3, x, x, None, None, None)])
+
+
+def test_batched_spmm_stream_order_across_configs(vs):
+    """One batched SpMM call spanning six kernel configurations (V, panel width, SPLIT):
+    the launches after the first use programmatic dependent launch (DESIGN 7.2), so a copy
+    enqueued right after the call on the same stream — no synchronisation in between — must
+    still see every problem's final C, equal bit for bit to the single calls."""
+    probs = []
+    for i, (K, N) in enumerate([(4096, 256), (1024, 256), (256, 256), (4096, 64), (1024, 64), (256, 64)]):
+        M, V = 2048 - 8 * i, 4
+        rng = gen.make_rng(f"pdl_{i}")
+        probs.append((M, K, N, V, gen.colvec_dense(rng, M, K, V, 0.3), gen.dense_operand(rng, K, N)))
+    singles, batch = [], []
+    for M, K, N, V, A, B in probs:
+        rp, ci, va = vs.encode(V, dense=dev(A))
+        Bd = dev(B)
+        C1 = torch.empty((M, N), dtype=torch.float16, device="cuda")
+        vs.vs_spmm(M, K, N, V, rp, ci, va, Bd, C1)
+        singles.append(C1)
+        batch.append((M, K, N, V, rp, ci, va, Bd, torch.full((M, N), 5.0, dtype=torch.float16, device="cuda")))
+    torch.cuda.synchronize()
+    for _ in range(3):
+        for p in batch:
+            p[8].fill_(5.0)
+        vs.vs_spmm_batched(batch)
+        snap = torch.cat([p[8].flatten() for p in batch])  # same stream, no sync
+        torch.cuda.synchronize()
+        assert torch.equal(snap.view(torch.int16), torch.cat([c.flatten() for c in singles]).view(torch.int16))
