@@ -228,6 +228,33 @@ __device__ __forceinline__ void compact_body_direct(int64_t M, int64_t K, int64_
 #ifndef VS_ENC_MINB
 #define VS_ENC_MINB 6
 #endif
+// VS_ENC_PREFETCH: next-chunk row prefetch in the staged compact pass (dense input, V <= 4)
+#ifndef VS_ENC_PREFETCH
+#define VS_ENC_PREFETCH 1
+#endif
+// The 8 columns [c, c+8) of row i as one 16-byte word; zeros past M or K (K % 8 == 0).
+__device__ __forceinline__ uint4 enc_raw_row(const uint16_t* __restrict__ dense, int64_t i, int64_t M,
+                                             int64_t K, int64_t c) {
+  return (i < M && c < K) ? ldg128_na(dense + i * K + c) : make_uint4(0, 0, 0, 0);
+}
+// Halves of the V raw row words into h and the keep bits (any nonzero bit pattern).
+template <int V>
+__device__ __forceinline__ uint32_t enc_unpack_keep(const uint4 (&raw)[V], uint16_t (&h)[V][8]) {
+  uint32_t keep = 0;
+#pragma unroll
+  for (int r = 0; r < V; ++r) {
+    const uint32_t wd[4] = {raw[r].x, raw[r].y, raw[r].z, raw[r].w};
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      h[r][2 * q] = (uint16_t)(wd[q] & 0xFFFF);
+      h[r][2 * q + 1] = (uint16_t)(wd[q] >> 16);
+    }
+#pragma unroll
+    for (int j = 0; j < 8; ++j) keep |= (uint32_t)(h[r][j] != 0) << j;
+  }
+  return keep;
+}
+
 template <int V, bool VEC, bool HAS_MASK, bool WRITE_VALS, bool VEC_VALS>
 __device__ __forceinline__ void compact_body(int64_t M, int64_t K, int64_t w,
                                              const uint16_t* __restrict__ dense,
@@ -244,10 +271,30 @@ __device__ __forceinline__ void compact_body(int64_t M, int64_t K, int64_t w,
   const int lane = lane_id();
   int64_t base = row_ptr[w];
   uint16_t h[V][8];
+  // Dense 16-byte path, V <= 4: the rows of the next 256-column chunk are loaded before the
+  // current chunk is packed and stored (the shared-memory staging and __syncwarp of a chunk
+  // otherwise keep the next chunk's loads from issuing early).  Same output.
+  constexpr bool PF = VS_ENC_PREFETCH && VEC && !HAS_MASK && V <= 4;
+  uint4 nxt[PF ? V : 1];
+  if constexpr (PF) {
+#pragma unroll
+    for (int r = 0; r < V; ++r) nxt[r] = enc_raw_row(dense, w * V + r, M, K, (int64_t)lane * kColsPerLane);
+  }
 #pragma unroll 2
   for (int64_t c0 = 0; c0 < K; c0 += kColsPerStep) {
     const int64_t c = c0 + lane * kColsPerLane;
-    const uint32_t keep = window_keep8<V, VEC, HAS_MASK, WRITE_VALS>(dense, mask, M, K, w, c, h);
+    uint32_t keep;
+    if constexpr (PF) {
+      uint4 cur[V];
+#pragma unroll
+      for (int r = 0; r < V; ++r) {
+        cur[r] = nxt[r];
+        nxt[r] = enc_raw_row(dense, w * V + r, M, K, c + kColsPerStep);
+      }
+      keep = enc_unpack_keep<V>(cur, h);
+    } else {
+      keep = window_keep8<V, VEC, HAS_MASK, WRITE_VALS>(dense, mask, M, K, w, c, h);
+    }
     const uint32_t n = __popc(keep);
     uint32_t incl = n;
 #pragma unroll
