@@ -49,6 +49,8 @@ def parse_args(argv=None):
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--workload", default=DEFAULT_WORKLOAD)
+    ap.add_argument("--priority", choices=["none", "first", "sddmm", "encode"], default="sddmm",
+                    help="high stream priority for part of the chain schedule (see step_chains)")
     ap.add_argument("--schedule", choices=["chains", "phases"], default="chains",
                     help="batched step as one chain per V group on concurrent branches, or as "
                          "three phases (encode, then SpMM || SDDMM)")
@@ -413,7 +415,14 @@ def run_ours(args):
             vs.make_encode_batch([(b.p.M, b.p.K, b.p.V, b.Wd, None, b.row_ptr, b.col_idx, b.vals) for b in gb]),
             vs.make_spmm_batch([(b.p.M, b.p.K, b.p.N, b.p.V, b.row_ptr, b.col_idx, b.vals, b.X, b.Y) for b in gb]),
             vs.make_sddmm_batch([(b.p.M, b.p.K, b.p.N, b.p.V, b.row_ptr, b.col_idx, b.G, b.X, b.dW) for b in gb])))
-    chain_streams = [(torch.cuda.Stream(), torch.cuda.Stream()) for _ in chain_arrs]
+    # --priority: which chain streams get the high stream priority (captured into the graph's
+    # kernel nodes): "first" = the V = 2 chain (its SDDMM is the longest), "sddmm" = every
+    # SDDMM branch (default: 0.916 -> 0.902 ms per step, profiles/r01g_priority.md), "encode" =
+    # every encode -> SpMM branch, "none" = all default.
+    def _prio(i, side):
+        hi = {"first": i == 0, "sddmm": side, "encode": not side}.get(args.priority, False)
+        return torch.cuda.Stream(priority=-1) if hi else torch.cuda.Stream()
+    chain_streams = [(_prio(i, False), _prio(i, True)) for i in range(len(chain_arrs))]
 
     def step_chains(pre=None, post=None):
         cur = torch.cuda.current_stream()
@@ -582,7 +591,9 @@ def run_ours(args):
                    "flops_per_step": flops_step, "l2": "flushed between timed steps (512 MiB write, untimed)",
                    "launch": "batched C ABI (vs_*_batched), step replayed as one CUDA graph; " + (
                              "one chain per V group (encode -> SpMM || SDDMM), chains on concurrent "
-                             "graph branches" if args.schedule == "chains" else
+                             "graph branches" + (f", high stream priority: {args.priority}"
+                                                 if args.priority != "none" else "")
+                             if args.schedule == "chains" else
                              "encode batch, then SpMM batch || SDDMM batch"),
                    "accumulate": "fp32"},
         "alt_schedule": {"schedule": "phases" if args.schedule == "chains" else "chains",
