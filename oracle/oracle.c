@@ -229,6 +229,11 @@ void oracle_softmax(int64_t M, int V, const int32_t* row_ptr, const uint16_t* va
         double x = scale * half_to_double(vals[p * V + r]);
         if (x > m) m = x;
       }
+      if (m == -INFINITY) { /* every stored score is -inf: the row attends to nothing, 0
+                               (reading R23; the plain formula gives 0/0) */
+        for (p = row_ptr[w]; p < row_ptr[w + 1]; ++p) out64[p * V + r] = 0.0;
+        continue;
+      }
       for (p = row_ptr[w]; p < row_ptr[w + 1]; ++p)
         sum += exp(scale * half_to_double(vals[p * V + r]) - m);
       for (p = row_ptr[w]; p < row_ptr[w + 1]; ++p)

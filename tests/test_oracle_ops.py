@@ -309,6 +309,31 @@ def test_softmax_invariants(V):
                                oracle.softmax(M, V, rp, grid, 1.0), rtol=1e-12, atol=1e-15)
 
 
+@pytest.mark.parametrize("V", [1, 4, 8])
+def test_softmax_minus_inf_scores(V):
+    """-inf scores (entries masked by the caller): where a row has a finite score the result
+    equals the dense masked softmax (exp(-inf) = 0); a row whose stored scores are all -inf
+    outputs 0 (reading R23 -- the plain formula is 0/0)."""
+    rng = gen.make_rng(f"sminf_{V}")
+    M, N = 8 * 6 + 3, 64
+    mask = gen.colvec_mask(rng, M, N, V, 0.4)
+    rp, ci, _ = oracle.encode(M, N, V, mask=mask)
+    nnz = int(rp[-1])
+    vals = gen.fp16_values(rng, nnz * V).copy()
+    vals[rng.random(nnz * V) < 0.3] = -np.inf
+    v2 = vals.reshape(-1, V)
+    w_all = 2                                # window 2: every row fully -inf
+    v2[rp[w_all]:rp[w_all + 1], :] = -np.inf
+    out = oracle.softmax(M, V, rp, vals, 0.5)
+    o2 = out.reshape(-1, V)
+    assert np.all(o2[rp[w_all]:rp[w_all + 1]] == 0)
+    assert np.all(out[np.isneginf(vals.astype(np.float64))] == 0)
+    ref = dense_masked_softmax(vals, rp, ci, M, N, V, 0.5)
+    finite = ~np.isnan(ref)                  # numpy's 0/0 rows are the R23 rows
+    np.testing.assert_allclose(out[finite], ref[finite], rtol=1e-12, atol=1e-15)
+    assert np.all(out[~finite] == 0)
+
+
 def test_attention_mask_density():
     rng = gen.make_rng("amask")
     m = gen.attention_mask(rng, 4096, 8, 0.9)   # band 256 = 6.25% < 10%: random fills the rest
