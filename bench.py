@@ -59,7 +59,8 @@ def parse_args(argv=None):
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--reps", type=int, default=20, help="launches per per-cell micro timing")
     ap.add_argument("--detail", default=os.path.join(ROOT, "gpurun_out", "bench_detail.json"))
-    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--cpu-seconds", type=float, default=8.0,
+                    help="CPU work per thread setting of the cpu_baseline leg (x3 runs)")
     ap.add_argument("--streams", type=int, default=8,
                     help="concurrent graph branches across independent problems")
     return ap.parse_args(argv)
@@ -221,29 +222,91 @@ def layer_inputs(p):
     return _INPUT_CACHE[p.id]
 
 
-def oracle_sample_run(problems, seconds):
-    """Runs the fp64 oracle (encode + SpMM + SDDMM) over problems in order until ~seconds of
-    CPU work; returns (flops, elapsed, n_problems)."""
+def oracle_sample_run(problems, seconds, threads=0, reps=1):
+    """Runs the fp64 oracle (encode + SpMM + SDDMM of each layer problem, timed inside
+    oracle.c with the monotonic clock, oracle.time_layer) over problems in order until
+    ~seconds of CPU work; per problem the median of `reps` runs counts.
+    Returns (flops, elapsed, n_problems)."""
     import oracle
     flops, t_used, n = 0.0, 0.0, 0
     for p in problems:
         Wd, X, G = layer_inputs(p)
-        t0 = time.perf_counter()
-        rp, ci, va = oracle.encode(p.M, p.K, p.V, dense=Wd)
-        oracle.spmm(p.M, p.K, p.N, p.V, rp, ci, va, X)
-        oracle.sddmm(p.M, p.K, p.N, p.V, rp, ci, G, X)
-        t_used += time.perf_counter() - t0
-        f1, f2 = problem_flops(int(rp[-1]), p)
+        secs, nnz = oracle.time_layer(p.M, p.K, p.N, p.V, Wd, X, G, threads=threads, reps=reps)
+        t_used += statistics.median(secs)
+        f1, f2 = problem_flops(nnz, p)
         flops += f1 + f2
         n += 1
-        if t_used >= seconds:
+        if t_used * reps >= seconds:
             break
     return flops, t_used, n
+
+
+def cpu_baseline_protocol(problems, seconds):
+    """the oracle as it stands, all cores and one thread, median of 3 runs
+    per problem (monotonic clock inside oracle.c), over a bounded interleaved sample of the
+    workload (about `seconds` of CPU work per thread setting)."""
+    import oracle
+    cores = oracle.num_threads()
+    f_all, t_all, n_all = oracle_sample_run(problems, seconds, threads=0, reps=3)
+    # one thread on the same first problems (it takes ~cores x longer: fewer problems fit)
+    f_one, t_one, n_one = oracle_sample_run(problems, seconds, threads=1, reps=3)
+    return {"value": f_all / t_all / 1e12, "unit": UNIT, "cores": cores, "kind": "oracle",
+            "sample": f"first {n_all} problems of the interleaved workload order (encode+SpMM+SDDMM, "
+                      f"fp64 C oracle, median of 3 runs each, {t_all:.1f} s per run set)",
+            "one_thread": {"value": f_one / t_one / 1e12, "unit": UNIT, "cores": 1,
+                           "sample": f"first {n_one} problems, median of 3 runs each"},
+            "timer": "clock_gettime(CLOCK_MONOTONIC) inside oracle.c (oracle_time_layer)"}
 
 
 def sample_order(problems):
     """Deterministic interleaving so a bounded sample spans shapes, V and S."""
     return problems[::7] + [p for i, p in enumerate(problems) if i % 7]
+
+
+def parity_gate(bufs, every=7, n_spmm=512, n_sddmm=256, replay=None):
+    """Oracle gate on the outputs of the TIMED launch configuration:
+    for every `every`-th problem of the batch, the GPU encoding (row_ptr, col_idx, vals) must
+    equal the oracle encoder bit for bit, and sampled SpMM outputs Y[i][j] / SDDMM vectors dW[p]
+    must be within 2e-3*sum|ab| + 2^-24 of the fp64 oracle.  Raises on any failure, so bench.py
+    never prints a value for a step whose results are wrong."""
+    import numpy as np
+    import oracle
+    worst, checked, ns, nd = 0.0, 0, 0, 0
+    for j, b in enumerate(bufs):
+        if j % every:
+            continue
+        p = b.p
+        Wd, X, G = layer_inputs(p)
+        rp = b.row_ptr.cpu().numpy()
+        nnz = int(rp[-1])
+        ci = b.col_idx[:nnz].cpu().numpy()
+        va = b.vals[:nnz * p.V].cpu().numpy()
+        orp, oci, ova = oracle.encode(p.M, p.K, p.V, dense=Wd)
+        if not (np.array_equal(rp, orp) and np.array_equal(ci, oci)
+                and np.array_equal(va.view(np.uint16), ova.view(np.uint16))):
+            raise AssertionError(f"parity gate: encoding of {p.id} differs from the oracle")
+        rng = np.random.default_rng(j)
+        rows = rng.integers(0, p.M, n_spmm)
+        cols = rng.integers(0, p.N, n_spmm)
+        o, sc = oracle.spmm_sample(p.M, p.K, p.N, p.V, orp, oci, ova, X, rows, cols)
+        Y = b.Y.cpu().numpy()
+        e = np.abs(Y[rows, cols].astype(np.float64) - o) / oracle.tolerance(sc)
+        if nnz:
+            ps = rng.integers(0, nnz, n_sddmm)
+            od, sd = oracle.sddmm_sample(p.M, p.K, p.N, p.V, orp, oci, G, X, ps)
+            dW = b.dW[:nnz * p.V].cpu().numpy().reshape(-1, p.V)
+            e2 = np.abs(dW[ps].astype(np.float64) - od) / oracle.tolerance(sd)
+            e = np.concatenate([e.ravel(), e2.ravel()])
+            nd += ps.size
+        ns += rows.size
+        worst = max(worst, float(e.max()) if e.size else 0.0)
+        if worst > 1.0:
+            raise AssertionError(f"parity gate: {p.id} outside the tolerance (ratio {worst:.3g})")
+        checked += 1
+    return {"problems_checked": checked, "of": len(bufs), "every": every,
+            "encode": "bit-exact vs oracle.encode", "spmm_samples": ns, "sddmm_vectors": nd,
+            "worst_err_over_tol": worst, "tolerance": "2e-3*sum|ab| + 2^-24",
+            "outputs_of": "the timed graph (one extra replay after the timed region)"}
 
 
 def run_reference(args):
@@ -533,6 +596,12 @@ def run_ours(args):
     torch.cuda.synchronize()
     clk = clocks.stop()
 
+    # oracle gate on the timed launch configuration's outputs (raises on failure)
+    with torch.cuda.stream(stream):
+        g_step.replay()
+    stream.synchronize()
+    gate = parity_gate(bufs)
+
     total_ms = sum(step_ms)
     if ws > 1:
         t = torch.tensor([total_ms], device=dev, dtype=torch.float64)
@@ -612,6 +681,7 @@ def run_ours(args):
                     for k, v in cls_ms.items()},
         "gpu_launches": launches_per_step["total"] * args.steps,
         "clocks": clk,
+        "parity_gate": gate,
     }
 
     detail = {"problems": [], "step_ms": step_ms}
@@ -661,12 +731,7 @@ def run_ours(args):
 
     # ---------------- CPU oracle baseline ----------------
     if not args.no_cpu and rank == 0 and ws == 1:
-        import oracle
-        f, t, n = oracle_sample_run(sample_order(problems), args.cpu_seconds)
-        line["cpu_baseline"] = {"value": f / t / 1e12, "unit": UNIT, "cores": oracle.num_threads(),
-                                "kind": "oracle",
-                                "sample": f"{n} of {nb} problems (encode+SpMM+SDDMM, fp64 C oracle, "
-                                          f"{t:.1f} s), interleaved order"}
+        line["cpu_baseline"] = cpu_baseline_protocol(sample_order(problems), args.cpu_seconds)
     if rank == 0:
         os.makedirs(os.path.dirname(args.detail), exist_ok=True)
         json.dump(detail, open(args.detail, "w"), indent=1)
@@ -1063,13 +1128,12 @@ def run_train(args):
             dY = torch.from_numpy(gen.dense_operand(rng, M, N)).to(dev)
             rp, ci, va = vs.encode(V, dense=Wd)
             nnz = int(rp[-1].item())
-            rT, cT, vT = vs.transpose(rp, ci[:nnz], va[:nnz * V], M, K, V)
+            # W^T's pattern from W's STORED pattern (pattern-only transpose), so the per-step
+            # value refresh places every stored element of W, zero now or not (vs.h)
+            rT, cT, vT, ws = vs.transpose_pattern(rp, ci[:nnz], M, K, V)
             nT = int(rT[-1].item())
-            ws = torch.empty(max(vs.vs_transpose_colvec_workspace(M, K, V), 4), dtype=torch.uint8, device=dev)
             layers.append(dict(M=M, K=K, V=V, Wd=Wd, X=X, dY=dY, rp=rp, ci=ci[:nnz], va=va[:nnz * V],
-                               rT=rT, cT=torch.empty(max(nT, 1), dtype=torch.int32, device=dev),
-                               vT=torch.empty(max(nT, 1) * V, dtype=torch.float16, device=dev),
-                               ws=ws, nnz=nnz, nT=nT,
+                               rT=rT, cT=cT, vT=vT, ws=ws, nnz=nnz, nT=nT,
                                Y=torch.empty((M, N), dtype=torch.float16, device=dev),
                                dX=torch.empty((K, N), dtype=torch.float16, device=dev),
                                dW=torch.empty(max(nnz, 1) * V, dtype=torch.float16, device=dev)))
@@ -1109,11 +1173,8 @@ def run_train(args):
             torch.matmul(L["Wd"].t(), L["dY"])
             torch.matmul(L["dY"], L["X"].t())
 
-    # the pattern of W^T is fixed (pruned weights): one full transpose per layer before the
-    # steps; every step refreshes W^T's values from W's (vs_transpose_colvec_values)
-    for L in layers:
-        vs.vs_transpose_colvec(L["M"], L["K"], L["V"], L["rp"], L["ci"], L["va"], L["rT"], L["cT"],
-                               L["vT"], workspace=L["ws"])
+    # the pattern of W^T is fixed (pruned weights): built once per layer before the steps
+    # (transpose_pattern); every step refreshes W^T's values from W's (vs_transpose_colvec_values)
     # parity spot check of the step's transposed operand against a dense transpose product
     stream = torch.cuda.Stream()
     with torch.cuda.stream(stream):

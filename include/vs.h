@@ -92,6 +92,8 @@ int vs_version(void);
  *     or the bound W*K).  Asynchronous unless nnz_vec_host != NULL (then it synchronises
  *     and stores nnz_v).
  *   M == 0 or K == 0 gives row_ptr = 0 everywhere and nnz_v = 0.
+ *   ceil(M/V) * K >= 2^31 (nnz_v could overflow the int32 row_ptr) -> VS_ERROR_NOT_SUPPORTED,
+ *   before anything is enqueued.
  */
 vs_status_t vs_encode_colvec(int64_t M, int64_t K, int V,
                              const void* dense, const uint8_t* mask,
@@ -117,7 +119,10 @@ vs_status_t vs_encode_colvec(int64_t M, int64_t K, int V,
  *   colT_idx : int32 [nnzT] output (ascending m inside each window), or NULL = count mode.
  *   valsT    : fp16 [nnzT * V] output (requires vals), or NULL.
  *   workspace: device buffer of vs_transpose_colvec_workspace(M, K, V) bytes (int32
- *              aligned), scratch for the call.
+ *              aligned), scratch for the call: a dense ceil(K/V) x ceil(M/V) int32 table of
+ *              per-(column group, window) row masks, i.e. O(M*K/V^2) bytes whatever nnz_v is
+ *              (4*M*K bytes at V = 1: twice the dense fp16 matrix), memset on every full and
+ *              count call.  Keep it between calls when the pattern will be refreshed.
  *   nnzT_host: if non-NULL, the call synchronises `stream` and stores rowT_ptr[ceil(K/V)].
  *   Count mode (colT_idx == NULL) writes rowT_ptr only; full mode needs colT_idx / valsT
  *   capacities >= nnzT (from a count-mode call, or the bound ceil(K/V) * M).
@@ -131,6 +136,10 @@ int64_t vs_transpose_colvec_workspace(int64_t M, int64_t K, int V);
  * workspace must come from a previous full-mode vs_transpose_colvec call on the same row_ptr
  * / col_idx.  valsT[q*V + j] = A[colT_idx[q]][kw*V + j] from the new vals for every vector q
  * of that pattern (elements of A that are not stored give +0.0).  Two kernels, asynchronous.
+ *   Build a pattern that will be refreshed with vals == NULL (pattern-only): every stored
+ *   element of A (rows < M) then has its slot in valsT.  A pattern built FROM VALUES holds
+ *   only the elements that were nonzero at build time; a stored element that was +0.0 then
+ *   and is nonzero now is not placed by the refresh (its contribution to W^T is lost).
  */
 vs_status_t vs_transpose_colvec_values(int64_t M, int64_t K, int V,
                                        const int32_t* row_ptr, const int32_t* col_idx,

@@ -63,6 +63,9 @@ def lib():
             L.oracle_softmax.argtypes = [_I64, ctypes.c_int, _P, _P, ctypes.c_double, _P]
             L.oracle_half_to_double.restype = ctypes.c_double
             L.oracle_half_to_double.argtypes = [ctypes.c_uint16]
+            L.oracle_time_layer.restype = _I64
+            L.oracle_time_layer.argtypes = [_I64, _I64, _I64, ctypes.c_int, _P, _P, _P,
+                                            ctypes.c_int, ctypes.c_int, _P]
             L.oracle_num_threads.restype = ctypes.c_int
             L.oracle_num_threads.argtypes = []
             _lib = L
@@ -181,6 +184,20 @@ def sddmm_sample(M, N, K, V, row_ptr, col_idx, A, Bt, vec_p):
                               _ptr(_f16(A)), _ptr(_f16(Bt)), vec_p.size, _ptr(vec_p), _ptr(vec_w),
                               _ptr(out), _ptr(S))
     return out.reshape(-1, V), S.reshape(-1, V)
+
+
+def time_layer(M, K, N, V, dense, X, G, threads=0, reps=3):
+    """Seconds of `reps` runs of one bench layer step (encode W -> SpMM W X -> SDDMM
+    (G X^T) o pattern(W)) with `threads` OpenMP threads (0 = all), timed inside oracle.c with
+    the monotonic clock.  Returns (list of seconds, nnz_v)."""
+    d, x, g = _f16(dense), _f16(X), _f16(G)
+    assert d.shape == (M, K) and x.shape == (K, N) and g.shape == (M, N)
+    secs = np.zeros(reps, np.float64)
+    nnz = lib().oracle_time_layer(M, K, N, V, _ptr(d), _ptr(x), _ptr(g), int(threads), int(reps),
+                                  _ptr(secs))
+    if nnz < 0:
+        raise MemoryError("oracle_time_layer: allocation failed")
+    return secs.tolist(), int(nnz)
 
 
 def softmax(M: int, V: int, row_ptr, vals, scale: float) -> np.ndarray:

@@ -28,10 +28,13 @@
  * products; numpy fp64 brute force on tiny shapes; identity and integer-exact closed forms;
  * all-ones-mask SDDMM = GEMM; the SpMM/SDDMM adjoint identity.
  */
+#define _POSIX_C_SOURCE 199309L
 #include <stdint.h>
 #include <stddef.h>
+#include <stdlib.h>
 #include <math.h>
 #include <string.h>
+#include <time.h>
 
 /* IEEE binary16 -> double, exact.  sign(1) exponent(5, bias 15) mantissa(10). */
 static double half_to_double(uint16_t h) {
@@ -249,4 +252,56 @@ int oracle_num_threads(void) {
 #else
   return 1;
 #endif
+}
+
+/*
+ * CPU-baseline timing: one layer step of the bench -- encode W, C = W X
+ * (SpMM), dW = (G X^T) o pattern(W) (SDDMM, inner dimension N) -- run `reps` times with
+ * `threads` OpenMP threads (0 = the default team), each rep timed with the monotonic clock
+ * (clock_gettime(CLOCK_MONOTONIC), the C counterpart of steady_clock).  Writes the seconds of
+ * each rep to secs[reps]; returns nnz_v (or -1 if a buffer cannot be allocated).  The timed
+ * work is exactly the functions above: nothing is tuned for the benchmark.
+ */
+static double mono_seconds(void) {
+  struct timespec ts;
+  clock_gettime(CLOCK_MONOTONIC, &ts);
+  return (double)ts.tv_sec + 1e-9 * (double)ts.tv_nsec;
+}
+
+int64_t oracle_time_layer(int64_t M, int64_t K, int64_t N, int V, const uint16_t* dense,
+                          const uint16_t* X, const uint16_t* G, int threads, int reps,
+                          double* secs) {
+#ifdef _OPENMP
+  extern void omp_set_num_threads(int);
+  extern int omp_get_max_threads(void);
+  int saved = omp_get_max_threads();
+  if (threads > 0) omp_set_num_threads(threads);
+#endif
+  int64_t W = ceil_div(M, V), nnz = 0, r;
+  int32_t* row_ptr = (int32_t*)malloc(sizeof(int32_t) * (size_t)(W + 1));
+  double* C = (double*)malloc(sizeof(double) * (size_t)(M * N));
+  double* S = (double*)malloc(sizeof(double) * (size_t)(M * N));
+  int32_t* col_idx = NULL;
+  uint16_t* vals = NULL;
+  double *o = NULL, *so = NULL;
+  for (r = 0; r < reps; ++r) {
+    double t0 = mono_seconds();
+    nnz = oracle_encode(M, K, V, dense, NULL, row_ptr, NULL, NULL);
+    if (r == 0) {
+      col_idx = (int32_t*)malloc(sizeof(int32_t) * (size_t)(nnz + 1));
+      vals = (uint16_t*)malloc(sizeof(uint16_t) * (size_t)(nnz * V + 1));
+      o = (double*)malloc(sizeof(double) * (size_t)(nnz * V + 1));
+      so = (double*)malloc(sizeof(double) * (size_t)(nnz * V + 1));
+    }
+    if (!row_ptr || !C || !S || !col_idx || !vals || !o || !so) { nnz = -1; break; }
+    oracle_encode(M, K, V, dense, NULL, row_ptr, col_idx, vals);
+    oracle_spmm(M, K, N, V, row_ptr, col_idx, vals, X, C, S);
+    oracle_sddmm(M, K, N, V, row_ptr, col_idx, G, X, o, so);
+    secs[r] = mono_seconds() - t0;
+  }
+  free(row_ptr); free(C); free(S); free(col_idx); free(vals); free(o); free(so);
+#ifdef _OPENMP
+  omp_set_num_threads(saved);
+#endif
+  return nnz;
 }

@@ -24,7 +24,7 @@ import threading
 __all__ = ["VSError", "lib_path", "load", "vs_encode_colvec", "vs_spmm", "vs_sddmm",
            "vs_softmax_colvec", "vs_encode_colvec_batched", "vs_spmm_batched", "vs_sddmm_batched",
            "vs_softmax_colvec_batched", "sparse_attention",
-           "encode", "spmm", "sddmm", "num_windows"]
+           "encode", "spmm", "sddmm", "transpose", "transpose_pattern", "num_windows"]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
 # VS_LIB_PATH overrides the library location (used to compare kernel build variants)
@@ -355,6 +355,27 @@ def transpose(row_ptr, col_idx, vals, M, K, V, stream=None):
         vs_transpose_colvec(M, K, V, row_ptr, col_idx, vals, rowT, colT, valsT, workspace=ws,
                             stream=stream)
     return rowT, colT[:n], (valsT[:n * V] if valsT is not None else None)
+
+
+def transpose_pattern(row_ptr, col_idx, M, K, V, stream=None):
+    """Pattern-only encoding of A^T for a layer whose values will be refreshed every step
+    (vs_transpose_colvec with vals = NULL: every stored element of A has a slot, so a value
+    that is +0.0 now and nonzero later is still placed; see vs.h).  Returns
+    (rowT_ptr, colT_idx, valsT buffer, workspace); fill valsT with
+    vs_transpose_colvec_values(M, K, V, row_ptr, col_idx, vals, rowT_ptr, valsT, workspace)."""
+    import torch
+    dev = row_ptr.device
+    KT = num_windows(K, V)
+    rowT = torch.empty(KT + 1, dtype=torch.int32, device=dev)
+    ws = torch.empty(max(vs_transpose_colvec_workspace(M, K, V), 4), dtype=torch.uint8, device=dev)
+    n = vs_transpose_colvec(M, K, V, row_ptr, col_idx, None, rowT, workspace=ws, want_nnz=True,
+                            stream=stream)
+    colT = torch.empty(max(n, 1), dtype=torch.int32, device=dev)
+    if n > 0:
+        vs_transpose_colvec(M, K, V, row_ptr, col_idx, None, rowT, colT, None, workspace=ws,
+                            stream=stream)
+    valsT = torch.empty(max(n, 1) * V, dtype=torch.float16, device=dev)
+    return rowT, colT[:n], valsT[:n * V], ws
 
 
 def spmm(row_ptr, col_idx, vals, B, M, V, out=None, stream=None):

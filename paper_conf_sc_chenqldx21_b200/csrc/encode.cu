@@ -514,11 +514,10 @@ cudaError_t launch_encode(int64_t M, int64_t K, int V, const void* dense, const 
 // limit, the default).  L2-sized chunks let the compact pass re-read its inputs from L2, but
 // measured slower (tools/tune.py, DLMC batch: no limit 247 us, 96 MB 309 us, 48 MB 424 us,
 // 24 MB 517 us): fewer, wider launches win.
-static int64_t enc_chunk_bytes() {
-  const char* e = std::getenv("VS_ENC_CHUNK_MB");
-  const int64_t mb = e ? std::atoll(e) : 0;
-  return mb * (1LL << 20);
-}
+#ifndef VS_ENC_CHUNK_MB
+#define VS_ENC_CHUNK_MB 0
+#endif
+static constexpr int64_t enc_chunk_bytes() { return (int64_t)VS_ENC_CHUNK_MB * (1LL << 20); }
 
 cudaError_t launch_encode_batched(int64_t count, const int64_t* M, const int64_t* K, const int* V,
                                   const void* const* dense, const uint8_t* const* mask,

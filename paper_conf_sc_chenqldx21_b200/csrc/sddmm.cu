@@ -17,7 +17,6 @@
 // partial sum stays inside one MMA accumulator, so the paper's cross-octet shuffle+FADD
 // reduction (17-30% of instructions) disappears.
 #include <algorithm>
-#include <cstdlib>
 #include <utility>
 #include <vector>
 
@@ -338,32 +337,30 @@ static int ctas_per_sm(Kern k) {
 // KC = 4 over the DLMC set, tools/tune.py; VS_SDDMM_KC caps it) and whether the A row of a
 // window stays in registers -- the ARES slot now selects the mixed-K kernel (sddmm_window_any).  Encoded as
 // KC * 2 + ARES.
+// Build-time constants (no run-time knobs in the shipped library; tools/tune.py builds
+// variants with -D): VS_SDDMM_KC caps the K block, VS_SDDMM_MIX = one mixed-K kernel per V,
+// VS_SDDMM_PAIR = two chunks in flight for K <= 64.
+#ifndef VS_SDDMM_KC
+#define VS_SDDMM_KC 2
+#endif
+#ifndef VS_SDDMM_MIX
+#define VS_SDDMM_MIX 1
+#endif
+#ifndef VS_SDDMM_PAIR
+#define VS_SDDMM_PAIR 1
+#endif
 static int sddmm_variant(int64_t K, bool vec) {
-  static const int cap = [] {
-    const char* e = std::getenv("VS_SDDMM_KC");
-    const int c = e ? std::atoi(e) : 2;
-    return c >= 2 ? 2 : 1;
-  }();
+  constexpr int cap = VS_SDDMM_KC >= 2 ? 2 : 1;
   int kc = (!vec || K <= 64) ? 1 : 2;
   if (kc > cap) kc = cap;
-  // VS_SDDMM_MIX (default 1): vector-path problems of any K share the mixed kernel
-  static const bool mix = [] {
-    const char* e = std::getenv("VS_SDDMM_MIX");
-    return e ? std::atoi(e) != 0 : true;
-  }();
-  if (vec && mix && cap == 2) return 2 * 2 + 1;
+  // vector-path problems of any K share the mixed kernel
+  if (vec && VS_SDDMM_MIX && cap == 2) return 2 * 2 + 1;
   return kc * 2;
 }
 
-// VS_SDDMM_PAIR (default 1): K <= 64 problems of the mixed-K kernel keep two chunks in flight
-// per warp (sddmm_window_pair); 0 selects the one-chunk body.  Same bits either way.
-static bool sddmm_pair_on() {
-  static const bool on = [] {
-    const char* e = std::getenv("VS_SDDMM_PAIR");
-    return e ? std::atoi(e) != 0 : true;
-  }();
-  return on;
-}
+// K <= 64 problems of the mixed-K kernel keep two chunks in flight per warp
+// (sddmm_window_pair); VS_SDDMM_PAIR=0 selects the one-chunk body.  Same bits either way.
+static constexpr bool sddmm_pair_on() { return VS_SDDMM_PAIR != 0; }
 
 template <int V, bool VEC, int KC, bool ARES>
 static int sddmm_ctas_per_sm() {
@@ -405,14 +402,13 @@ static cudaError_t launch_sddmm_v(int64_t M, int64_t N, int64_t K, const int32_t
 
 template <int V, bool VEC, int KC, bool ARES>
 static void launch_sddmm_batch(const SddmmBatch& b, int num_sms, cudaStream_t s) {
-  // VS_SDDMM_OVERSUB: grid = that many times the resident CTAs (tuning knob).  2 is 5% faster
+  // VS_SDDMM_OVERSUB (build time): grid = that many times the resident CTAs.  2 is 5% faster
   // for the SDDMM batch alone but 2% slower for the bench step, where the oversubscribed grid
   // competes with the concurrent SpMM / encode branches; default 1.
-  static const int over = [] {
-    const char* e = std::getenv("VS_SDDMM_OVERSUB");
-    const int v = e ? std::atoi(e) : 1;
-    return v < 1 ? 1 : v;
-  }();
+#ifndef VS_SDDMM_OVERSUB
+#define VS_SDDMM_OVERSUB 1
+#endif
+  constexpr int over = VS_SDDMM_OVERSUB < 1 ? 1 : VS_SDDMM_OVERSUB;
   dim3 grid((unsigned)(num_sms * sddmm_batched_ctas_per_sm<V, VEC, KC, ARES>() * over));
   sddmm_batched_kernel<V, VEC, KC, ARES><<<grid, kSddmmWarps * 32, 0, s>>>(b);
 }
@@ -429,22 +425,31 @@ static void launch_sddmm_batch_v(const SddmmBatch& b, int code, int num_sms, cud
   }
 }
 
+// tcgen05 path (sddmm_tc.cu), compiled only into a library built with -DVS_WITH_SDDMM_TC=1:
+// such a build sends problems with K % 8 == 0, K > 0 and 16-byte aligned A, Bt and out_vals
+// to the tensor-core kernel, single and batched calls alike.  Not in the shipped library:
+// measured 1.8-2.5x slower than the mma.sync kernels below over the DLMC set (DESIGN.md 7.4,
+// profiles/r01b_tcgen05.md) -- the cp.async shared-memory staging that tcgen05 operands need
+// caps the row gather at ~60 B/clk/SM, below the register path.
+#ifndef VS_WITH_SDDMM_TC
+#define VS_WITH_SDDMM_TC 0
+#endif
+static constexpr bool sddmm_tc_on() { return VS_WITH_SDDMM_TC != 0; }
+#if VS_WITH_SDDMM_TC
 bool sddmm_tc_eligible(int64_t K, const void* A, const void* Bt, const void* out);
 cudaError_t launch_sddmm_tc_batched(int64_t count, const int64_t* M, const int64_t* N, const int64_t* K, const int* V,
                                     const int32_t* const* row_ptr, const int32_t* const* col_idx,
                                     const void* const* A, const void* const* Bt, void* const* out,
                                     int num_sms, cudaStream_t s);
-
-// tcgen05 path (sddmm_tc.cu): VS_SDDMM_TC=1 sends problems with K % 8 == 0, K > 0 and
-// 16-byte aligned A, Bt and out_vals to the tensor-core kernel, single and batched calls
-// alike (so both give the same bits).  Default off: measured 1.8-2.5x slower than the
-// mma.sync kernels below over the DLMC set (profiles/r01b_tcgen05.md) --
-// the cp.async shared-memory staging that tcgen05 operands need caps the row gather at
-// ~60 B/clk/SM, below the register path.  Read at every call (tests switch it per call).
-static bool sddmm_tc_on() {
-  const char* e = std::getenv("VS_SDDMM_TC");
-  return e != nullptr && std::atoi(e) != 0;
+#else
+static bool sddmm_tc_eligible(int64_t, const void*, const void*, const void*) { return false; }
+static cudaError_t launch_sddmm_tc_batched(int64_t, const int64_t*, const int64_t*, const int64_t*,
+                                           const int*, const int32_t* const*, const int32_t* const*,
+                                           const void* const*, const void* const*, void* const*,
+                                           int, cudaStream_t) {
+  return cudaErrorNotSupported;
 }
+#endif
 
 static cudaError_t launch_sddmm_mma_batched(int64_t count, const int64_t* M, const int64_t* K,
                                             const int* V, const int32_t* const* row_ptr,

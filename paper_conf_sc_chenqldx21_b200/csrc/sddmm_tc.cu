@@ -36,6 +36,10 @@
 
 #include "common.cuh"
 
+#ifndef VS_WITH_SDDMM_TC
+#define VS_WITH_SDDMM_TC 0
+#endif
+#if VS_WITH_SDDMM_TC  // opt-in build only (see sddmm.cu)
 namespace vs {
 namespace sddmm_tc {
 
@@ -505,3 +509,4 @@ cudaError_t launch_sddmm_tc_batched(int64_t count, const int64_t* M, const int64
 }
 
 }  // namespace vs
+#endif  // VS_WITH_SDDMM_TC

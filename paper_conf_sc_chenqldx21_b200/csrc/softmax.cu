@@ -4,7 +4,8 @@
 //
 //   out[p*V + r] = exp(s*x_p - m) / sum_q exp(s*x_q - m),  x_p = vals[p*V + r],
 // over the stored vectors p of window w, for every row i = wV + r < M (m = max_p s*x_p);
-// rows >= M (padding of the last window) get 0.  fp16 in/out, fp32 arithmetic.
+// rows >= M (padding of the last window) get 0.  fp16 in/out, fp32 arithmetic.  A -inf score
+// contributes exp(-inf) = 0; a row whose stored scores are all -inf outputs 0 (DESIGN R23).
 //
 // One warp per window; lane l owns vectors rb + l, rb + l + 32, ...  Pass 1 keeps an online
 // (max, sum) per row in each lane (sum rescaled when the max grows) and combines the lanes
@@ -82,6 +83,9 @@ __device__ __forceinline__ void softmax_window(int64_t M, int64_t w, const int32
     for (int r = 0; r < V; ++r) {
       const float y = x[r] * sl;
       const float nm = fmaxf(m[r], y);
+      // a -inf score (masked out by the caller) adds nothing; while the row has seen only
+      // -inf, m stays -inf and sum 0 (no inf - inf)
+      if (nm == -INFINITY) continue;
       sum[r] = sum[r] * exp2f(m[r] - nm) + exp2f(y - nm);
       m[r] = nm;
     }
@@ -108,7 +112,7 @@ __device__ __forceinline__ void softmax_window(int64_t M, int64_t w, const int32
     load_vec<V>(vals, p, x);
     float y[V];
 #pragma unroll
-    for (int r = 0; r < V; ++r) y[r] = exp2f(x[r] * sl - m[r]) * inv[r];
+    for (int r = 0; r < V; ++r) y[r] = inv[r] == 0.f ? 0.f : exp2f(x[r] * sl - m[r]) * inv[r];
     store_vec<V>(out, p, y);
   }
 }

@@ -19,7 +19,7 @@
 //   2t and 2t+1: the epilogue stores 16 bytes per row with no shuffles.
 //   B fragment (k = vector slot, n = row r < V) is vals[p*V + g].
 #include <algorithm>
-#include <cstdlib>
+#include <mutex>
 #include <utility>
 #include <vector>
 
@@ -599,21 +599,19 @@ struct SpmmCfg {
 // otherwise the number of stages D (2 or 3; default 2, see VS_SPMM_CP_WARPS; 4 was slower).  VS_SPMM_CPNC caps the panel width
 // (64 * NC columns, NC in {1, 2, 4}; default 2: tools/tune.py over the DLMC batch, batched
 // 502 us (cap 2) vs 569 us (cap 4) vs 650 us (cap 1) vs 629 us for the register path).
-static int spmm_cp_stages() {
-  static const int v = [] {
-    const char* e = std::getenv("VS_SPMM_CP");
-    const int d = e ? std::atoi(e) : 2;
-    return d <= 0 ? 0 : d <= 2 ? 2 : 3;
-  }();
-  return v;
+// Build-time constants (the shipped library has no run-time knobs; tools/tune.py builds
+// variants with -D): VS_SPMM_CP = ring depth (0 = register path only), VS_SPMM_CPNC = panel cap.
+#ifndef VS_SPMM_CP
+#define VS_SPMM_CP 2
+#endif
+#ifndef VS_SPMM_CPNC
+#define VS_SPMM_CPNC 2
+#endif
+static constexpr int spmm_cp_stages() {
+  return VS_SPMM_CP <= 0 ? 0 : VS_SPMM_CP <= 2 ? 2 : 3;
 }
-static int spmm_cp_nc_cap() {
-  static const int v = [] {
-    const char* e = std::getenv("VS_SPMM_CPNC");
-    const int n = e ? std::atoi(e) : 2;
-    return n >= 4 ? 4 : n >= 2 ? 2 : 1;
-  }();
-  return v;
+static constexpr int spmm_cp_nc_cap() {
+  return VS_SPMM_CPNC >= 4 ? 4 : VS_SPMM_CPNC >= 2 ? 2 : 1;
 }
 static int64_t cp_smem_bytes(int V, int NC, int SPLIT, int D) {
   const int64_t warps = SPLIT > kSpmmWarps ? SPLIT : kSpmmWarps;
@@ -625,12 +623,11 @@ SpmmCfg spmm_config(int64_t K, int64_t N, int V, const void* B, const void* C) {
   SpmmCfg c;
   c.V = V;
   // register path: 64-column panels (a K x 64 panel of B stays L1-resident for K <= ~1500;
-  // tools/tune.py: 3% faster than 128-column panels; VS_SPMM_NC=2 selects 128 columns)
-  static const int nc_knob = [] {
-    const char* e = std::getenv("VS_SPMM_NC");
-    return e ? std::atoi(e) : 1;
-  }();
-  c.NC = (N <= 64 || nc_knob != 2) ? 1 : 2;
+  // tools/tune.py: 3% faster than 128-column panels; build with -DVS_SPMM_NC=2 for 128)
+#ifndef VS_SPMM_NC
+#define VS_SPMM_NC 1
+#endif
+  c.NC = (N <= 64 || VS_SPMM_NC != 2) ? 1 : 2;
   const int64_t q = K >> 8;
   c.SPLIT = q >= 16 ? 16 : q >= 8 ? 8 : q >= 4 ? 4 : q >= 2 ? 2 : 1;
   c.VEC = (N % 8 == 0) && ((reinterpret_cast<uintptr_t>(B) & 15) == 0) &&
@@ -660,14 +657,16 @@ template <int V, int NC, int SPLIT, int D>
 static SpmmKernels cp_kernels_of() {
   constexpr int smem = SpmmCta<SPLIT>::kWarps * CpRing<V, NC, D>::kWarpBytes;
   static_assert(smem <= 227 * 1024 || NC > 1, "cp ring does not fit");
-  static bool done[64] = {};
+  // once per (instantiation, device), thread-safe (std::call_once)
+  static std::once_flag once[64];
   int dev = 0;
   cudaGetDevice(&dev);
-  if (smem > 48 * 1024 && !(dev >= 0 && dev < 64 && done[dev])) {
-    cudaFuncSetAttribute(spmm_cp_kernel<V, NC, SPLIT, D>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    cudaFuncSetAttribute(spmm_cp_batched_kernel<V, NC, SPLIT, D>,
-                         cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    if (dev >= 0 && dev < 64) done[dev] = true;
+  if (smem > 48 * 1024 && dev >= 0 && dev < 64) {
+    std::call_once(once[dev], [] {
+      cudaFuncSetAttribute(spmm_cp_kernel<V, NC, SPLIT, D>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+      cudaFuncSetAttribute(spmm_cp_batched_kernel<V, NC, SPLIT, D>,
+                           cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    });
   }
   return {spmm_cp_kernel<V, NC, SPLIT, D>, spmm_cp_batched_kernel<V, NC, SPLIT, D>,
           SpmmCta<SPLIT>::kWarps * 32, SpmmCta<SPLIT>::kUnits, 0, smem};
@@ -708,13 +707,10 @@ static SpmmKernels cp_pick(const SpmmCfg& c) {
 // B rows of the next group in flight during the current group's MMAs -- measured 10% slower,
 // the kernel is bound by the L1TEX data pipe (ncu: l1tex__data_pipe_lsu_wavefronts at
 // 79-93% of peak), not by latency.
-static int spmm_pipe() {
-  static const int v = [] {
-    const char* e = std::getenv("VS_SPMM_PIPE");
-    return e ? std::atoi(e) : 0;
-  }();
-  return v;
-}
+#ifndef VS_SPMM_PIPE
+#define VS_SPMM_PIPE 0
+#endif
+static constexpr int spmm_pipe() { return VS_SPMM_PIPE; }
 
 template <int V, int NC, bool VEC, int SPLIT>
 static SpmmKernels kernels_of() {
@@ -784,15 +780,12 @@ cudaError_t launch_spmm(int64_t M, int64_t K, int64_t N, int V, const int32_t* r
   return cudaGetLastError();
 }
 
-// VS_SPMM_PDL (default 1): the launches of one batched call after the first use programmatic
+// VS_SPMM_PDL (build-time, default 1): the launches of one batched call after the first use programmatic
 // dependent launch (pdl_*); 0 launches them plainly.  Same kernels, same bits.
-static bool spmm_pdl_on() {
-  static const bool on = [] {
-    const char* e = std::getenv("VS_SPMM_PDL");
-    return e ? std::atoi(e) != 0 : true;
-  }();
-  return on;
-}
+#ifndef VS_SPMM_PDL
+#define VS_SPMM_PDL 1
+#endif
+static constexpr bool spmm_pdl_on() { return VS_SPMM_PDL != 0; }
 
 // problems with K == 0 are handled by the caller (zero fill); M == 0 or N == 0 skipped.
 cudaError_t launch_spmm_batched(int64_t count, const int64_t* M, const int64_t* K, const int64_t* N,

@@ -88,6 +88,8 @@ vs_status_t check_encode(int64_t M, int64_t K, int V, const void* dense, const u
   if (M * K > 0 && vals != nullptr && dense == nullptr) return VS_ERROR_INVALID_VALUE;
   if (!al(row_ptr, 4) || (col_idx && !al(col_idx, 4))) return VS_ERROR_MISALIGNED;
   if ((dense && !al(dense, 2)) || (vals && !al(vals, 2))) return VS_ERROR_MISALIGNED;
+  // row_ptr / nnz_v are int32: refuse matrices whose vector count could reach 2^31
+  if (M > 0 && (M + V - 1) / V * K >= (int64_t(1) << 31)) return VS_ERROR_NOT_SUPPORTED;
   return VS_SUCCESS;
 }
 

@@ -82,7 +82,7 @@ def test_no_shared_code_between_oracle_and_cuda_path():
             assert not any("oracle" in h for h in inc.findall(text)), f
             assert not any(m.split(".")[0] == "oracle" for m in imp.findall(text)), f
     otext = open(os.path.join(ROOT, "oracle", "oracle.c")).read()
-    assert set(inc.findall(otext)) <= {"stdint.h", "stddef.h", "math.h", "string.h"}
+    assert set(inc.findall(otext)) <= {"stdint.h", "stddef.h", "stdlib.h", "math.h", "string.h", "time.h"}
     ptext = open(os.path.join(ROOT, "oracle", "__init__.py")).read()
     assert not any(m.split(".")[0] in ("paper_conf_sc_chenqldx21_b200", "synth")
                    for m in imp.findall(ptext))

@@ -50,6 +50,29 @@ def test_softmax_parity(vs, V, M, N):
     assert torch.equal(xd.view(torch.int16), out.view(torch.int16))
 
 
+@pytest.mark.parametrize("V", [1, 2, 4, 8])
+def test_softmax_minus_inf_scores(vs, V):
+    """-inf scores add nothing; a row whose stored scores are all -inf outputs 0 (R23), no NaN."""
+    M, N = 8 * 20 + 5, 200
+    rng = gen.make_rng(f"gsminf_{V}")
+    mask = gen.colvec_mask(rng, M, N, V, 0.3)
+    rp, ci, _ = vs.encode(V, mask=dev(mask))
+    rph = host(rp)
+    nnz = int(rph[-1])
+    x = gen.fp16_values(rng, nnz * V).copy()
+    x[rng.random(nnz * V) < 0.4] = -np.inf
+    x2 = x.reshape(-1, V)
+    x2[rph[3]:rph[4], :] = -np.inf           # window 3 fully masked
+    x2[rph[5]:rph[6], 0] = -np.inf           # one row of window 5 fully masked
+    xd = dev(x)
+    out = torch.empty_like(xd)
+    vs.vs_softmax_colvec(M, V, rp, xd, out, 0.7)
+    g = host(out).astype(np.float64)
+    assert not np.isnan(g).any()
+    p64 = oracle.softmax(M, V, rph, x, 0.7)
+    assert np.all(np.abs(g - p64) <= oracle.softmax_tolerance(p64))
+
+
 @pytest.mark.parametrize("V", [8, 4])
 def test_sparse_attention_chain(vs, V):
     l, k = 1024, 64

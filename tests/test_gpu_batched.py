@@ -48,11 +48,8 @@ def make(p, i):
     return A, B, G
 
 
-@pytest.mark.parametrize("sddmm_tc", ["0", "1"])
-def test_batched_matches_single_calls(vs, sddmm_tc, monkeypatch):
-    """Batched == single calls bit for bit, with SDDMM on the mma.sync path and on the
-    tcgen05 path (VS_SDDMM_TC, read by libvs at every call)."""
-    monkeypatch.setenv("VS_SDDMM_TC", sddmm_tc)
+def test_batched_matches_single_calls(vs):
+    """Batched == single calls bit for bit (encode, SpMM, SDDMM)."""
     probs = problem_mix()
     data = [make(p, i) for i, p in enumerate(probs)]
     enc_single, enc_batch, sp_b, sd_b = [], [], [], []

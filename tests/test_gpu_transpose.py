@@ -23,6 +23,10 @@ def vs():
     return m
 
 
+def host(t):
+    return t.cpu().numpy()
+
+
 def dev(x):
     return torch.from_numpy(np.ascontiguousarray(x)).cuda()
 
@@ -137,3 +141,40 @@ def test_transpose_values_refresh(vs, V, blocks):
     oT, ocT, ovT = oracle.transpose(M, K, V, orp, oci, ova)
     assert np.array_equal(rT.cpu().numpy(), oT) and np.array_equal(cT2[:nT].cpu().numpy(), ocT)
     assert np.array_equal(vT2[:nT * V].cpu().numpy().view(np.uint16), ovT.view(np.uint16))
+
+
+@pytest.mark.parametrize("V", [1, 2, 4, 8])
+def test_transpose_pattern_refresh_places_new_nonzeros(vs, V):
+    """a pattern built from W's STORED pattern (vals = NULL) gives every stored
+    element of W a slot, so values that were +0.0 at build time and are nonzero after the
+    update reach W^T.  valsT[q*V + j] = W2[colT[q]][kw*V + j] by definition (the transposed
+    element), against the oracle's pattern transpose; dX = W^T dY against the oracle."""
+    rng = gen.make_rng(f"gtr_pat_{V}")
+    M, K, N = 41 * V + 3, 23 * V + 5, 64
+    W1 = gen.colvec_dense(rng, M, K, V, 0.3, inner_zero_frac=0.4)
+    rp, ci, va = vs.encode(V, dense=dev(W1))
+    n = int(rp[-1].item())
+    rT, cT, vT, ws = vs.transpose_pattern(rp, ci[:n], M, K, V)
+    # new values on every stored element of W1's pattern, zeros inside vectors included
+    orp, oci, ova = oracle.encode(M, K, V, dense=W1)
+    ova2 = gen.fp16_values(rng, n * V)
+    vs.vs_transpose_colvec_values(M, K, V, rp, ci[:n], dev(ova2), rT, vT, ws)
+    torch.cuda.synchronize()
+    W2 = oracle.decode(M, K, V, orp, oci, ova2)
+    oT, ocT, _ = oracle.transpose(M, K, V, orp, oci, None)
+    assert np.array_equal(host(rT), oT) and np.array_equal(host(cT), ocT)
+    KT = len(oT) - 1
+    exp = np.zeros((len(ocT), V), np.float16)
+    for kw in range(KT):
+        for q in range(oT[kw], oT[kw + 1]):
+            for j in range(V):
+                if kw * V + j < K:
+                    exp[q, j] = W2[ocT[q], kw * V + j]
+    assert np.array_equal(host(vT).reshape(-1, V).view(np.uint16), exp.view(np.uint16))
+    dY = gen.dense_operand(rng, M, N)
+    dX = host(vs.spmm(rT, cT, vT, dev(dY), K, V))
+    o2rp, o2ci, o2va = oracle.encode(M, K, V, dense=W2)
+    tT, tcT, tvT = oracle.transpose(M, K, V, o2rp, o2ci, o2va)
+    X64, S64 = oracle.spmm(K, M, N, V, tT, tcT, tvT, dY)
+    err = np.abs(dX.astype(np.float64) - X64)
+    assert np.all(err <= oracle.tolerance(S64)), f"max err {err.max()}"
