@@ -48,7 +48,9 @@ def parse_args(argv=None):
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--workload", default=DEFAULT_WORKLOAD)
+    ap.add_argument("--workload", default=None,
+                    help="default: dlmc_layer at --gpus 1 (configs[1] x configs[2]); c5 at --gpus N > 1 "
+                         "(configs[4], the case that shards)")
     ap.add_argument("--priority", choices=["none", "first", "sddmm", "encode"], default="sddmm",
                     help="high stream priority for part of the chain schedule (see step_chains)")
     ap.add_argument("--schedule", choices=["chains", "phases"], default="chains",
@@ -315,6 +317,8 @@ def run_reference(args):
         return 0
     import oracle
     from synth.workloads import WORKLOADS
+    if args.workload == "c5":
+        return run_reference_c5(args)
     problems = sample_order(WORKLOADS[args.workload]())
     per_step = max(2.0, min(20.0, 150.0 / max(1, args.steps + args.warmup)))
     for _ in range(args.warmup):
@@ -339,6 +343,30 @@ def run_reference(args):
                          "sample": f"{nprob} problems (~{per_step:.0f} s of fp64 oracle work) per step"},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def run_reference_c5(args):
+    """Reference arm for configs[4]: the fp64 oracle on the deterministic C5 sample
+    (c5_oracle_sample), one sample per step, throughput extrapolated in flops."""
+    import oracle
+    ws, _, _ = dist_env()
+    for _ in range(args.warmup):
+        c5_oracle_sample()
+    tot_f, tot_t = 0.0, 0.0
+    for _ in range(args.steps):
+        f, t, desc = c5_oracle_sample()
+        tot_f += f
+        tot_t += t
+    value = tot_f / tot_t / 1e12
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": ws,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot_t / max(1, args.steps),
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "config": {"workload": "c5", "sample": desc},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": oracle.num_threads(),
+                             "kind": "oracle", "sample": desc},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
 
@@ -870,12 +898,37 @@ def ctypes_int():
     return ctypes.c_int(0)
 
 
+C5_BLOCK = 4096  # B is generated in 4096-column blocks: the same global B for every world size
+
+
+def c5_plan(ws: int, rank: int, mask_row_ptr=None):
+    """Host-side partition of configs[4]: SpMM N-panels of B / C (widths whole
+    generator blocks, dist.panel_bounds) and SDDMM row windows balanced by stored vectors
+    (dist.window_bounds on the global mask's row_ptr).  Pure bookkeeping (gloo-tested)."""
+    from paper_conf_sc_chenqldx21_b200 import dist as vsd
+    M = K = 16384
+    N, V, S = 65536, 8, 0.9
+    W = M // V
+    pb = vsd.panel_bounds(N, ws, align=C5_BLOCK)
+    plan = {"M": M, "K": K, "N": N, "V": V, "S": S, "W": W, "panel_bounds": pb,
+            "n0": pb[rank], "n1": pb[rank + 1]}
+    if mask_row_ptr is not None:
+        wb = vsd.window_bounds(mask_row_ptr, ws)
+        sh = vsd.sddmm_shard(mask_row_ptr, M, V, wb, rank)
+        plan.update({"window_bounds": wb, "shard": sh})
+    return plan
+
+
 def run_c5(args):
-    """configs[4]: M=K=16384, N=65536, V=8, S=0.9 -- SpMM sharded over N-panels of B/C (A
-    replicated) and SDDMM (mask 16384 x 65536, inner K=16384) sharded over row windows (Bt
-    replicated), no collective on the data path.  Strong scaling: the total
-    problem is fixed, each rank encodes and computes its shard.  Inputs are generated on the
-    device (seeded) and are far larger than L2, so no flush is needed."""
+    """configs[4]: M=K=16384, N=65536, V=8, S=0.9.  SpMM sharded over N-panels of B/C (A
+    replicated) and SDDMM (mask 16384 x 65536, inner K=16384) sharded over row windows balanced
+    by stored vectors (dist.window_bounds; Bt replicated), no collective on the data path
+    (SURVEY §8(e)).  Strong scaling: the total problem is fixed; every rank generates the same
+    global operands (seeded) and computes its shard.  Timed separately: the optional replicated
+    output, through NCCL (gather_panels / gather_segments) and through the fused SpMM scatter
+    epilogue into symmetric memory (dist.spmm_npanel_replicated).  Same-box dense cuBLAS
+    (Hgemm, GemmEx) on this rank's dense counterpart.  Inputs are far larger than L2."""
+    import numpy as np
     import torch
     import paper_conf_sc_chenqldx21_b200 as vs
     from paper_conf_sc_chenqldx21_b200 import dist as vsd
@@ -891,35 +944,41 @@ def run_c5(args):
     dev = torch.device("cuda", torch.cuda.current_device())
     vs.load()
     peaks = load_peaks()
-    M = K = 16384
-    N, V, S = 65536, 8, 0.9
-    W = M // V
-    # SpMM shard: A replicated, this rank's N-panel of B and C
-    pb = vsd.panel_bounds(N, ws)
-    n0, n1 = pb[rank], pb[rank + 1]
+    plan = c5_plan(ws, rank)
+    M, K, N, V, S, W = (plan[k] for k in ("M", "K", "N", "V", "S", "W"))
+    n0, n1 = plan["n0"], plan["n1"]
     Np = n1 - n0
+    # ---- SpMM shard: A replicated, this rank's N-panel of the global B (4096-column blocks)
     Ad = gen.torch_colvec_dense(M, K, V, 1 - S, seed=gen.config_seed("c5_A"), device=dev)
-    Bp = gen.torch_dense_operand(K, Np, seed=gen.config_seed(f"c5_B_{n0}"), device=dev)
+    Bp = torch.empty((K, Np), dtype=torch.float16, device=dev)
+    for blk in range(n0 // C5_BLOCK, -(-n1 // C5_BLOCK)):
+        c0, c1 = blk * C5_BLOCK, min(N, (blk + 1) * C5_BLOCK)
+        Bp[:, c0 - n0:c1 - n0] = gen.torch_dense_operand(K, c1 - c0, seed=gen.config_seed(f"c5_Bblk_{blk}"),
+                                                         device=dev)
     Cp = torch.empty((M, Np), dtype=torch.float16, device=dev)
     capA = W * K
     rpA = torch.empty(W + 1, dtype=torch.int32, device=dev)
     ciA = torch.empty(capA, dtype=torch.int32, device=dev)
     vaA = torch.empty(capA * V, dtype=torch.float16, device=dev)
-    # SDDMM shard: this rank's row windows of the mask [M x N], Bt [N x K] replicated
-    wb = [(W * r) // ws for r in range(ws + 1)]
-    w0, w1 = wb[rank], wb[rank + 1]
-    Ml = (w1 - w0) * V
+    # ---- SDDMM: the global mask (same seed on every rank) -> its row_ptr -> balanced windows
     g = torch.Generator(device=dev)
-    g.manual_seed(gen.config_seed(f"c5_mask_{w0}"))
-    keep = torch.rand((w1 - w0, N), generator=g, device=dev) < (1 - S)
-    maskl = keep.repeat_interleave(V, dim=0).to(torch.uint8).contiguous()
+    g.manual_seed(gen.config_seed("c5_mask"))
+    keep = torch.rand((W, N), generator=g, device=dev) < (1 - S)
+    mask = keep.repeat_interleave(V, dim=0).to(torch.uint8).contiguous()
     del keep
-    Al = gen.torch_dense_operand(Ml, K, seed=gen.config_seed(f"c5_Arows_{w0}"), device=dev)
+    rp_glob = torch.empty(W + 1, dtype=torch.int32, device=dev)
+    vs.vs_encode_colvec(M, N, V, None, mask, rp_glob)              # count mode (setup)
+    plan = c5_plan(ws, rank, rp_glob.cpu().numpy())
+    sh = plan["shard"]
+    Ml = sh.row1 - sh.row0
+    maskl = mask[sh.row0:sh.row1]                                  # contiguous row slice
+    A_sd = gen.torch_dense_operand(M, K, seed=gen.config_seed("c5_Asd"), device=dev)
+    Al = A_sd[sh.row0:sh.row1]
     Bt = gen.torch_dense_operand(N, K, seed=gen.config_seed("c5_Bt"), device=dev)
-    capM = (w1 - w0) * N // 8  # >= nnz for density 0.1 with margin (checked below)
-    rpM = torch.empty(w1 - w0 + 1, dtype=torch.int32, device=dev)
-    ciM = torch.empty(capM, dtype=torch.int32, device=dev)
-    outM = torch.empty(capM * V, dtype=torch.float16, device=dev)
+    nnzM = sh.p1 - sh.p0
+    rpM = torch.empty(sh.w1 - sh.w0 + 1, dtype=torch.int32, device=dev)
+    ciM = torch.empty(max(nnzM, 1), dtype=torch.int32, device=dev)
+    outM = torch.empty(max(nnzM, 1) * V, dtype=torch.float16, device=dev)
 
     def step():
         vs.vs_encode_colvec(M, K, V, Ad, None, rpA, ciA, vaA)
@@ -932,8 +991,8 @@ def run_c5(args):
         step()
     stream.synchronize()
     nnzA = int(rpA[-1].item())
-    nnzM = int(rpM[-1].item())
-    assert nnzM <= capM, "mask capacity"
+    assert int(rpM[-1].item()) == nnzM, "local mask encoding disagrees with the global row_ptr"
+    assert torch.equal(rpM.cpu(), torch.from_numpy(sh.row_ptr.astype(np.int32))), "shard row_ptr"
     flops = 2.0 * nnzA * V * Np + 2.0 * nnzM * V * K
     ev = {k: (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
           for k in ("encA", "spmm", "encM", "sddmm")}
@@ -982,13 +1041,27 @@ def run_c5(args):
         torch.distributed.all_reduce(f)
         tot_flops = float(f.item())
     value = tot_flops / (ms * 1e-3) / 1e12
-    # roofline of the dominant kernel class on this rank (algorithmic bytes)
+
+    # ---- parity: sampled outputs of this rank's shard against the fp64 oracle
+    gate = c5_parity_gate(rank, M, K, N, V, n0, Np, rpA, ciA, vaA, Bp, Cp, sh, ciM, Al, Bt, outM)
+
+    # ---- replicated output (optional for callers; timed apart from the step)
+    rep_out = None
+    if ws > 1:
+        rep_out = c5_replicated_output(args, torch, vs, vsd, plan, rpA, ciA, vaA, Bp, Cp, outM, nnzM,
+                                       stream, dev)
+
+    # ---- same-box dense cuBLAS on this rank's dense counterpart (M x K x Np)
+    dense = c5_dense_cublas(torch, Ad, Bp, Cp, stream) if not args.no_baselines else None
+
     kref = K  # every column of B is referenced at 10% density over 2048 windows
     bytes_spmm = 4 * (W + 1) + nnzA * (4 + 2 * V) + 2 * kref * Np + 2 * M * Np
-    bytes_sddmm = 4 * (w1 - w0 + 1) + 4 * nnzM + 2 * Ml * K + 2 * N * K + 2 * nnzM * V
+    bytes_sddmm = 4 * (sh.w1 - sh.w0 + 1) + 4 * nnzM + 2 * Ml * K + 2 * N * K + 2 * nnzM * V
     dom = "spmm" if cls["spmm"] >= cls["sddmm"] else "sddmm"
     db = bytes_spmm if dom == "spmm" else bytes_sddmm
     ach = db / (cls[dom] * 1e-3) / 1e9
+    flops_dom = 2.0 * nnzA * V * Np if dom == "spmm" else 2.0 * nnzM * V * K
+    gb = 2.0 * nnzA * Np if dom == "spmm" else 2.0 * nnzM * K
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": ws, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "strong",
@@ -997,31 +1070,243 @@ def run_c5(args):
                    "step": "encode A, SpMM on this rank's N-panel (A replicated); encode this "
                            "rank's mask rows, SDDMM (mask 16384x65536, inner 16384, Bt replicated)",
                    "l2": "inputs far larger than L2 (no flush)", "nnz_v_spmm": nnzA,
-                   "nnz_v_sddmm_rank0": nnzM, "parallelism": f"spmm N-panels x{ws}, sddmm row windows x{ws}"},
+                   "nnz_v_sddmm_this_rank": nnzM, "panel": [n0, n1],
+                   "windows": [sh.w0, sh.w1],
+                   "parallelism": f"spmm N-panels x{ws} (dist.panel_bounds), sddmm row windows x{ws} "
+                                  "(dist.window_bounds, balanced by stored vectors)"},
         "roofline": {"bound": "hbm", "achieved": ach, "peak": peaks["hbm_gbs"], "unit": "GB/s",
                      "frac": ach / peaks["hbm_gbs"], "traffic": None, "kernel": dom,
                      "algorithmic_bytes_per_launch": db, "avg_launch_us": cls[dom] * 1e3,
                      "peak_source": peaks["source"]},
-        "roofline_tensor": {"bound": "tensor", "achieved": (flops_dom := (2.0 * nnzA * V * Np if dom == "spmm"
-                                                                          else 2.0 * nnzM * V * K)) / (cls[dom] * 1e-3) / 1e12,
+        "roofline_tensor": {"bound": "tensor", "achieved": flops_dom / (cls[dom] * 1e-3) / 1e12,
                             "peak": peaks["bf16_tflops_sustained"], "unit": "TFLOP/s",
                             "frac": flops_dom / (cls[dom] * 1e-3) / 1e12 / peaks["bf16_tflops_sustained"],
                             "kernel": dom, "peak_source": "sustained dense bf16 (MEASURED_PEAKS.json)"},
-        "roofline_gather": {"bound": "l2_gather",
-                            "achieved": (gb := (2.0 * nnzA * Np if dom == "spmm" else 2.0 * nnzM * K)) / (cls[dom] * 1e-3) / 1e9,
+        "roofline_gather": {"bound": "l2_gather", "achieved": gb / (cls[dom] * 1e-3) / 1e9,
                             "peak": GATHER_PEAK_GBS, "unit": "GB/s",
                             "frac": gb / (cls[dom] * 1e-3) / 1e9 / GATHER_PEAK_GBS, "kernel": dom,
                             "peak_source": "measured: tools/gather_bench.cu ldg_line (profiles/r01e_gather.md)"},
         "kernels": {k: {"ms": v} for k, v in cls.items()},
         "gpu_launches": 8 * args.steps,
         "clocks": clk,
+        "parity_gate": gate,
+        "replicated_output": rep_out,
+        "dense_cublas_this_rank": dense,
         "e2e": None,
     }
+    if dense:
+        line["speedup_vs_cublas_hgemm"] = {
+            "spmm": dense["hgemm_ms"] / cls["spmm"], "sddmm": dense["hgemm_ms"] * (Ml / M) / cls["sddmm"],
+            "spmm_vs_best_cublas": min(dense["hgemm_ms"], dense["gemmex_ms"]) / cls["spmm"],
+            "step_vs_dense_pair": 2 * min(dense["hgemm_ms"], dense["gemmex_ms"]) / ms,
+            "note": "dense counterpart of this rank's SpMM = M x K x Np GEMM; of its SDDMM = the "
+                    "same GEMM restricted to its rows (Ml/M of it); step_vs_dense_pair compares "
+                    "the step with two dense GEMMs (forward + weight gradient)"}
+    if not args.no_e2e:
+        line["e2e"] = c5_e2e(torch, step, stream, [Ad, Bp, maskl, Al, Bt], [Cp, outM[:nnzM * V]],
+                             tot_flops, ws, dev)
+    if not args.no_cpu and rank == 0 and ws == 1:
+        line["cpu_baseline"] = c5_cpu_baseline(args.cpu_seconds)
     if rank == 0:
         print(json.dumps(line), flush=True)
     if ws > 1:
         torch.distributed.destroy_process_group()
     return 0
+
+
+def c5_parity_gate(rank, M, K, N, V, n0, Np, rpA, ciA, vaA, Bp, Cp, sh, ciM, Al, Bt, outM,
+                   n_spmm=2048, n_sddmm=256):
+    """Sampled oracle check of the timed C5 launch on this rank (the full problem is too large
+    for the host): SpMM outputs C[i][n0 + j] and SDDMM stored vectors of this rank's windows,
+    against oracle.spmm_sample / sddmm_sample (2e-3*sum|ab| + 2^-24).  Raises on failure."""
+    import numpy as np
+    import torch
+    import oracle
+    nnzA = int(rpA[-1].item())
+    rng = np.random.default_rng(11 + rank)
+    rows = rng.integers(0, M, n_spmm)
+    cols = rng.integers(0, Np, n_spmm)
+    ucols = np.unique(cols)
+    Bsub = Bp[:, torch.from_numpy(ucols).to(Bp.device)].cpu().numpy()
+    o, s = oracle.spmm_sample(M, K, ucols.size, V, rpA.cpu().numpy(), ciA[:nnzA].cpu().numpy(),
+                              vaA[:nnzA * V].cpu().numpy(), Bsub, rows, np.searchsorted(ucols, cols))
+    g = Cp[torch.from_numpy(rows).to(Cp.device), torch.from_numpy(cols).to(Cp.device)].cpu().numpy()
+    e1 = np.abs(g.astype(np.float64) - o) / oracle.tolerance(s)
+    nnzM = sh.p1 - sh.p0
+    worst = float(e1.max())
+    if nnzM:
+        ps = rng.integers(0, nnzM, n_sddmm)
+        ci = ciM[:nnzM].cpu().numpy()
+        used = np.unique(ci[ps])
+        Btsub = Bt[torch.from_numpy(used).to(Bt.device)].cpu().numpy()
+        remap = np.zeros(N, np.int32)
+        remap[used] = np.arange(used.size, dtype=np.int32)
+        od, sd = oracle.sddmm_sample(sh.row1 - sh.row0, used.size, K, V, sh.row_ptr, remap[ci],
+                                     Al.cpu().numpy(), Btsub, ps)
+        gd = outM.view(-1, V)[torch.from_numpy(ps).to(outM.device)].cpu().numpy()
+        worst = max(worst, float((np.abs(gd.astype(np.float64) - od) / oracle.tolerance(sd)).max()))
+    if worst > 1.0:
+        raise AssertionError(f"C5 parity gate failed on rank {rank}: err/tol {worst:.3g}")
+    return {"spmm_samples": n_spmm, "sddmm_vectors": n_sddmm if nnzM else 0,
+            "worst_err_over_tol": worst, "tolerance": "2e-3*sum|ab| + 2^-24",
+            "oracle": "oracle.spmm_sample / sddmm_sample on this rank's shard"}
+
+
+def c5_replicated_output(args, torch, vs, vsd, plan, rpA, ciA, vaA, Bp, Cp, outM, nnzM, stream, dev):
+    """Replicated outputs of the sharded C5 (caller option), each timed
+    with CUDA events over `reps` rounds, max over ranks:
+      nccl_allgather_ms : gather_panels (all_gather_into_tensor + permute into row-major C)
+      scatter_spmm_ms   : the SpMM whose epilogue stores into every rank's symmetric-memory C
+                          (vs_spmm_scatter) + the stream barrier -- compare with spmm_ms +
+                          nccl_allgather_ms, the unfused pair
+      sddmm_allgather_ms: gather_segments of the out_vals segments."""
+    import torch.distributed as dist
+    M, K, V = plan["M"], plan["K"], plan["V"]
+    pb, n0, n1 = plan["panel_bounds"], plan["n0"], plan["n1"]
+    Np = n1 - n0
+    counts = [int(plan["shard"].p1 - plan["shard"].p0)]
+    allc = [None] * dist.get_world_size()
+    dist.all_gather_object(allc, counts[0])
+    counts = [c * V for c in allc]
+    reps = 3
+    out = {"world": dist.get_world_size(), "reps": reps}
+
+    def timed(fn):
+        torch.cuda.synchronize()
+        dist.barrier()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        with torch.cuda.stream(stream):
+            fn()  # warm
+            a.record()
+            for _ in range(reps):
+                fn()
+            b.record()
+        b.synchronize()
+        t = torch.tensor([a.elapsed_time(b) / reps], device=dev, dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    out["spmm_ms"] = timed(lambda: vs.vs_spmm(M, K, Np, V, rpA, ciA, vaA, Bp, Cp))
+    out["nccl_allgather_ms"] = timed(lambda: vsd.gather_panels(Cp, pb))
+    out["sddmm_allgather_ms"] = timed(lambda: vsd.gather_segments(outM[:nnzM * V], counts))
+    try:
+        rep = vsd.ReplicatedC(M, plan["N"], dev)
+        out["scatter_spmm_ms"] = timed(lambda: vsd.spmm_npanel_replicated(rpA, ciA, vaA, Bp, M, V, pb,
+                                                                          dist.get_rank(), rep))
+        # parity: the fused replica equals the NCCL-gathered one bit for bit
+        full = vsd.gather_panels(Cp, pb)
+        torch.cuda.synchronize()
+        out["scatter_equals_allgather"] = bool(torch.equal(full.view(torch.int16), rep.C.view(torch.int16)))
+        out["unfused_pair_ms"] = out["spmm_ms"] + out["nccl_allgather_ms"]
+    except Exception as exc:  # symmetric memory needs a capable NCCL / driver; report, do not fail
+        out["scatter_error"] = repr(exc)[:300]
+    return out
+
+
+def c5_dense_cublas(torch, Ad, Bp, Cp, stream, reps=3):
+    """cublasHgemm / cublasGemmEx (fp32 compute) of the dense M x K x Np product on this rank,
+    CUDA events, mean of `reps` after one warm-up (paper's comparison point)."""
+    import baselines
+    L = baselines.lib()
+    h = L.bl_create()
+    M, K = Ad.shape
+    Np = Bp.shape[1]
+    out = {}
+    try:
+        for name, fn in (("hgemm_ms", L.bl_hgemm), ("gemmex_ms", L.bl_gemmex)):
+            with torch.cuda.stream(stream):
+                fn(h, M, Np, K, Ad.data_ptr(), Bp.data_ptr(), Cp.data_ptr(), stream.cuda_stream)
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record()
+                for _ in range(reps):
+                    fn(h, M, Np, K, Ad.data_ptr(), Bp.data_ptr(), Cp.data_ptr(), stream.cuda_stream)
+                b.record()
+            b.synchronize()
+            out[name] = a.elapsed_time(b) / reps
+        out["dense_tflops_hgemm"] = 2.0 * M * K * Np / (out["hgemm_ms"] * 1e-3) / 1e12
+        out["dense_tflops_gemmex"] = 2.0 * M * K * Np / (out["gemmex_ms"] * 1e-3) / 1e12
+        out["shape"] = [M, K, Np]
+    finally:
+        L.bl_destroy(h)
+    return out
+
+
+def c5_e2e(torch, step, stream, inputs, outputs, tot_flops, ws, dev, reps=2):
+    """End to end through the public API: pinned host -> device copies of this rank's inputs,
+    the step, device -> pinned host copies of its outputs, all inside the timed region."""
+    try:
+        h_in = [t.cpu().pin_memory() for t in inputs]
+        h_out = [torch.empty(t.shape, dtype=t.dtype).pin_memory() for t in outputs]
+    except Exception as exc:
+        return {"value": None, "error": f"pinned host buffers: {exc!r}"[:200]}
+
+    def run():
+        for d, h in zip(inputs, h_in):
+            d.copy_(h, non_blocking=True)
+        step()
+        for d, h in zip(outputs, h_out):
+            h.copy_(d, non_blocking=True)
+    with torch.cuda.stream(stream):
+        run()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        for _ in range(reps):
+            run()
+        b.record()
+    b.synchronize()
+    ms = a.elapsed_time(b) / reps
+    if ws > 1:
+        t = torch.tensor([ms], device=dev, dtype=torch.float64)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        ms = float(t.item())
+    return {"value": tot_flops / (ms * 1e-3) / 1e12, "unit": UNIT, "ms_per_step": ms,
+            "h2d_bytes_per_step": int(sum(t.numel() * t.element_size() for t in inputs)),
+            "d2h_bytes_per_step": int(sum(t.numel() * t.element_size() for t in outputs)),
+            "path": "pinned host -> device, step (vs_encode_colvec, vs_spmm, vs_sddmm), device -> pinned host"}
+
+
+def c5_oracle_sample(seconds_hint=None):
+    """The fp64 oracle on a deterministic sample of configs[4]: SpMM of
+    8 windows x 4096 output columns and SDDMM of 8 windows x all their stored vectors, with
+    host-generated inputs of the C5 distribution (V = 8, density 0.1, K = 16384).  Returns
+    (flops, seconds, description); throughput extrapolates linearly in flops."""
+    import numpy as np
+    import oracle
+    from synth import gen
+    K, V, d, Ns = 16384, 8, 0.1, 4096
+    rng = gen.make_rng("c5_cpu_sample")
+    Ms = 8 * V
+    A = gen.colvec_dense(rng, Ms, K, V, d)
+    B = gen.dense_operand(rng, K, Ns)
+    t0 = time.perf_counter()
+    rp, ci, va = oracle.encode(Ms, K, V, dense=A)
+    oracle.spmm(Ms, K, Ns, V, rp, ci, va, B)
+    t_spmm = time.perf_counter() - t0
+    f_spmm = 2.0 * int(rp[-1]) * V * Ns
+    # SDDMM: 8 windows of the 16384 x 65536 mask, all their vectors; Bt rows restricted to the
+    # columns they reference (the oracle reads only those)
+    Nm = 65536
+    mask = gen.colvec_mask(rng, Ms, Nm, V, d)
+    mrp, mci, _ = oracle.encode(Ms, Nm, V, mask=mask)
+    used = np.unique(mci)
+    remap = np.zeros(Nm, np.int32)
+    remap[used] = np.arange(used.size, dtype=np.int32)
+    Al = gen.dense_operand(rng, Ms, K)
+    Bt = gen.dense_operand(rng, used.size, K)
+    t0 = time.perf_counter()
+    oracle.sddmm(Ms, used.size, K, V, mrp, remap[mci], Al, Bt)
+    t_sd = time.perf_counter() - t0
+    f_sd = 2.0 * int(mrp[-1]) * V * K
+    return (f_spmm + f_sd, t_spmm + t_sd,
+            "C5 sample: SpMM 8 windows x 4096 columns + SDDMM 8 windows x all stored vectors "
+            "(host-generated inputs of the C5 distribution), extrapolated linearly in flops")
+
+
+def c5_cpu_baseline(seconds):
+    import oracle
+    f, t, desc = c5_oracle_sample()
+    return {"value": f / t / 1e12, "unit": UNIT, "cores": oracle.num_threads(), "kind": "oracle",
+            "sample": desc + f" ({t:.1f} s, all cores, time.perf_counter)", "extrapolated": True}
 
 
 def run_attention(args):
@@ -1214,8 +1499,48 @@ def run_train(args):
     return 0
 
 
+def free_port() -> int:
+    import socket
+    sk = socket.socket()
+    sk.bind(("127.0.0.1", 0))
+    port = sk.getsockname()[1]
+    sk.close()
+    return port
+
+
+def launch_command(gpus: int, argv, port: int = None):
+    """torchrun command that runs this file on `gpus` ranks of one node (one process per GPU),
+    rendezvous on 127.0.0.1."""
+    return [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={gpus}",
+            "--master-addr=127.0.0.1", f"--master-port={port or free_port()}",
+            os.path.abspath(__file__), *argv]
+
+
+def check_world(args) -> str:
+    """'spawn' when --gpus N > 1 was asked for outside torchrun, 'run' when the rank count
+    matches; raises SystemExit when WORLD_SIZE disagrees with --gpus (never falls back to a
+    1-GPU run under a multi-GPU flag)."""
+    ws = os.environ.get("WORLD_SIZE")
+    if ws is None:
+        return "spawn" if args.gpus > 1 else "run"
+    if int(ws) != args.gpus:
+        raise SystemExit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={ws}")
+    return "run"
+
+
 def main(argv=None):
+    argv = list(sys.argv[1:] if argv is None else argv)
     args = parse_args(argv)
+    if check_world(args) == "spawn":
+        env = dict(os.environ)
+        # NCCL init lines (communicator size, transport) go to per-rank files, not stdout
+        env.setdefault("NCCL_DEBUG", "INFO")
+        env.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+        os.makedirs(os.path.join(ROOT, "gpurun_out"), exist_ok=True)
+        env.setdefault("NCCL_DEBUG_FILE", os.path.join(ROOT, "gpurun_out", "nccl_init.%h.%p.log"))
+        return subprocess.call(launch_command(args.gpus, argv), env=env)
+    if args.workload is None:
+        args.workload = "c5" if args.gpus > 1 else DEFAULT_WORKLOAD
     if args.impl == "reference":
         return run_reference(args)
     if args.workload == "c5":

@@ -167,6 +167,29 @@ vs_status_t vs_spmm(int64_t M, int64_t K, int64_t N, int V,
                     const void* B, void* C, vs_stream_t stream);
 
 /*
+ * vs_spmm_scatter — vs_spmm whose output tiles are stored into n_dst destinations: the fused
+ * replicated-output epilogue of the multi-GPU N-panel sharding (the
+ * paper is single-GPU, the sharding follows the north star).  For d < n_dst:
+ *   C_dst[d][i*ldc + j] = fp16_rn( sum_p vals[p*V + i%V] * B[col_idx[p]][j] ),  i < M, j < N,
+ * bit-identical to vs_spmm's C[i][j]; columns >= N of a destination row are not touched.
+ *   B      : fp16 [K x N] row-major (this rank's panel).
+ *   C_dst  : HOST array of n_dst (1 <= n_dst <= VS_SPMM_SCATTER_MAX) device-addressable
+ *            pointers, read during the call: e.g. every rank's symmetric-memory C buffer
+ *            (peer pointers over NVLink / NVSwitch), each offset to this rank's first column,
+ *            so one kernel writes the rank's panel into every replica of the row-major C.
+ *   ldc    : leading dimension (elements) of every destination, ldc >= N.
+ * The caller orders the peers' reads after the stores (e.g. a symmetric-memory barrier on
+ * the stream).  Errors as vs_spmm, plus VS_ERROR_INVALID_VALUE for a NULL C_dst, n_dst out of
+ * range or ldc < N.  The 16-byte store path needs 16-byte aligned destinations and
+ * ldc % 8 == 0; anything else takes the guarded path (same bits).
+ */
+#define VS_SPMM_SCATTER_MAX 8
+vs_status_t vs_spmm_scatter(int64_t M, int64_t K, int64_t N, int V,
+                            const int32_t* row_ptr, const int32_t* col_idx, const void* vals,
+                            const void* B, void* const* C_dst, int n_dst, int64_t ldc,
+                            vs_stream_t stream);
+
+/*
  * vs_sddmm — out = (A * B) sampled at a column-vector mask D [M x N].
  * Problem statement §4.1 P:589-593 (C in CSR, A row-major, B column-major "to replace
  * the transpose"); kernel §6.3-6.4; D a binary mask stored in the

@@ -21,7 +21,7 @@ import ctypes
 import os
 import threading
 
-__all__ = ["VSError", "lib_path", "load", "vs_encode_colvec", "vs_spmm", "vs_sddmm",
+__all__ = ["VSError", "lib_path", "load", "vs_encode_colvec", "vs_spmm", "vs_spmm_scatter", "vs_sddmm",
            "vs_softmax_colvec", "vs_encode_colvec_batched", "vs_spmm_batched", "vs_sddmm_batched",
            "vs_softmax_colvec_batched", "sparse_attention",
            "encode", "spmm", "sddmm", "transpose", "transpose_pattern", "num_windows"]
@@ -92,6 +92,9 @@ def load():
                                            ctypes.POINTER(ctypes.c_int64), _P]
             L.vs_spmm.restype = ctypes.c_int
             L.vs_spmm.argtypes = [_I64, _I64, _I64, ctypes.c_int, _P, _P, _P, _P, _P, _P]
+            L.vs_spmm_scatter.restype = ctypes.c_int
+            L.vs_spmm_scatter.argtypes = [_I64, _I64, _I64, ctypes.c_int, _P, _P, _P, _P,
+                                          ctypes.POINTER(ctypes.c_void_p), ctypes.c_int, _I64, _P]
             L.vs_sddmm.restype = ctypes.c_int
             L.vs_sddmm.argtypes = [_I64, _I64, _I64, ctypes.c_int, _P, _P, _P, _P, _P, _P]
             L.vs_transpose_colvec_workspace.restype = _I64
@@ -172,6 +175,19 @@ def vs_spmm(M, K, N, V, row_ptr, col_idx, vals, B, C, stream=None):
                         _ptr(col_idx, torch.int32, "col_idx"), _ptr(vals, torch.float16, "vals"),
                         _ptr(B, torch.float16, "B"), _ptr(C, torch.float16, "C"), _stream(stream))
     _check(st, "vs_spmm")
+
+
+def vs_spmm_scatter(M, K, N, V, row_ptr, col_idx, vals, B, dst_ptrs, ldc, stream=None):
+    """Mirror of vs_spmm_scatter: ``dst_ptrs`` is a list of integer device addresses (e.g.
+    symmetric-memory peer buffers offset to this rank's first column), ``ldc`` their leading
+    dimension in elements."""
+    import torch
+    n = len(dst_ptrs)
+    arr = (ctypes.c_void_p * max(n, 1))(*[int(p) for p in dst_ptrs])
+    st = load().vs_spmm_scatter(int(M), int(K), int(N), int(V), _ptr(row_ptr, torch.int32, "row_ptr"),
+                                _ptr(col_idx, torch.int32, "col_idx"), _ptr(vals, torch.float16, "vals"),
+                                _ptr(B, torch.float16, "B"), arr, n, int(ldc), _stream(stream))
+    _check(st, "vs_spmm_scatter")
 
 
 def vs_sddmm(M, N, K, V, row_ptr, col_idx, A, Bt, out_vals, stream=None):

@@ -29,6 +29,20 @@ namespace vs {
 
 constexpr int kSpmmWarps = 4;
 
+// Output destinations of a C tile: ND (compile-time bound) row-major matrices with leading
+// dimension ldc, each pointer at element (0, 0) of this launch's C.  ND = 1 is the plain
+// vs_spmm output (p[0] = C, ldc = N); vs_spmm_scatter stores every tile into n <= ND
+// destinations -- e.g. the symmetric-memory C buffers of all ranks, mapped into this GPU's
+// address space, so an N-panel shard lands in every rank's replicated row-major C directly
+// from the epilogue (no all-gather, no permute).
+constexpr int kMaxScatter = 8;
+template <int ND>
+struct CDst {
+  uint16_t* p[ND];
+  int n;
+  int64_t ldc;
+};
+
 template <int NC, bool VEC>
 __device__ __forceinline__ void load_brow(const uint16_t* __restrict__ B, int64_t N, int col,
                                           bool valid, int64_t ncol0, uint4 (&r)[NC]) {
@@ -72,12 +86,12 @@ struct SpmmCta {
   static constexpr int kUnits = kWarps / SPLIT;
 };
 
-template <int V, int NC, bool VEC, int SPLIT, int UNROLL>
+template <int V, int NC, bool VEC, int SPLIT, int UNROLL, int ND>
 __device__ __forceinline__ void spmm_body(int64_t M, int64_t N, int64_t W, int64_t n_wgroups,
                                           int64_t bid, const int32_t* __restrict__ row_ptr,
                                           const int32_t* __restrict__ col_idx,
                                           const uint16_t* __restrict__ vals,
-                                          const uint16_t* __restrict__ B, uint16_t* __restrict__ C) {
+                                          const uint16_t* __restrict__ B, const CDst<ND>& cd) {
   constexpr int UPC = SpmmCta<SPLIT>::kUnits;  // units per CTA
   constexpr int NACC = NC * 16;                // accumulator floats per thread
   constexpr int HALF = SPLIT > 1 ? SPLIT / 2 : 1;
@@ -261,13 +275,17 @@ __device__ __forceinline__ void spmm_body(int64_t M, int64_t N, int64_t W, int64
       uint32_t o[4];
 #pragma unroll
       for (int j = 0; j < 4; ++j) o[j] = f2_to_h2(acc[c][j][rr], acc[c][j][rr + 2]);
-      uint16_t* dst = C + i * N + n;
-      if (VEC) {
-        if (n < N) stg128(dst, make_uint4(o[0], o[1], o[2], o[3]));
-      } else {
 #pragma unroll
-        for (int e = 0; e < 8; ++e)
-          if (n + e < N) dst[e] = (uint16_t)((o[e >> 1] >> (16 * (e & 1))) & 0xFFFF);
+      for (int d = 0; d < ND; ++d) {
+        if (d >= cd.n) break;
+        uint16_t* dst = cd.p[d] + i * cd.ldc + n;
+        if (VEC) {
+          if (n < N) stg128(dst, make_uint4(o[0], o[1], o[2], o[3]));
+        } else {
+#pragma unroll
+          for (int e = 0; e < 8; ++e)
+            if (n + e < N) dst[e] = (uint16_t)((o[e >> 1] >> (16 * (e & 1))) & 0xFFFF);
+        }
       }
     }
   }
@@ -281,7 +299,19 @@ __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32)
                 const int32_t* __restrict__ row_ptr, const int32_t* __restrict__ col_idx,
                 const uint16_t* __restrict__ vals, const uint16_t* __restrict__ B,
                 uint16_t* __restrict__ C) {
-  spmm_body<V, NC, VEC, SPLIT, UNROLL>(M, N, W, n_wgroups, blockIdx.x, row_ptr, col_idx, vals, B, C);
+  const CDst<1> cd = {{C}, 1, N};
+  spmm_body<V, NC, VEC, SPLIT, UNROLL, 1>(M, N, W, n_wgroups, blockIdx.x, row_ptr, col_idx, vals, B, cd);
+}
+
+// vs_spmm_scatter, register path (unaligned operands or destinations, V = 1)
+template <int V, int NC, bool VEC, int SPLIT>
+__global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32)
+    spmm_scatter_kernel(int64_t M, int64_t N, int64_t W, int64_t n_wgroups,
+                        const int32_t* __restrict__ row_ptr, const int32_t* __restrict__ col_idx,
+                        const uint16_t* __restrict__ vals, const uint16_t* __restrict__ B,
+                        const __grid_constant__ CDst<kMaxScatter> cd) {
+  spmm_body<V, NC, VEC, SPLIT, 1, kMaxScatter>(M, N, W, n_wgroups, blockIdx.x, row_ptr, col_idx,
+                                               vals, B, cd);
 }
 
 // Batched launch: one grid over the units of up to kSpmmMaxBatch problems that share a
@@ -315,8 +345,9 @@ __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32)
   for (int64_t bid = blockIdx.x; bid < total; bid += gridDim.x) {
     while (b.first_block[p + 1] <= bid) ++p;
     const SpmmDesc& d = b.d[p];
-    spmm_body<V, NC, VEC, SPLIT, UNROLL>(d.M, d.N, d.W, d.n_wgroups, bid - b.first_block[p],
-                                         d.row_ptr, d.col_idx, d.vals, d.B, d.C);
+    const CDst<1> cd = {{d.C}, 1, d.N};
+    spmm_body<V, NC, VEC, SPLIT, UNROLL, 1>(d.M, d.N, d.W, d.n_wgroups, bid - b.first_block[p],
+                                            d.row_ptr, d.col_idx, d.vals, d.B, cd);
   }
   pdl_wait_prior();
 }
@@ -359,13 +390,13 @@ struct CpRing {
   static constexpr int kWarpBytes = (kRaw + 127) / 128 * 128;
 };
 
-template <int V, int NC, int SPLIT, int D>
+template <int V, int NC, int SPLIT, int D, int ND>
 __device__ __forceinline__ void spmm_cp_body(int64_t M, int64_t N, int64_t W, int64_t n_wgroups,
                                              int64_t bid, const int32_t* __restrict__ row_ptr,
                                              const int32_t* __restrict__ col_idx,
                                              const uint16_t* __restrict__ vals,
                                              const uint16_t* __restrict__ B,
-                                             uint16_t* __restrict__ C, unsigned char* smem) {
+                                             const CDst<ND>& cd, unsigned char* smem) {
   using R = CpRing<V, NC, D>;
   constexpr int UPC = SpmmCta<SPLIT>::kUnits;
   constexpr int HALF = SPLIT > 1 ? SPLIT / 2 : 1;
@@ -537,7 +568,13 @@ __device__ __forceinline__ void spmm_cp_body(int64_t M, int64_t N, int64_t W, in
     const int64_t i = w * V + r;
     const int64_t n = n0 + 8 * ch;
     const uint4 v = lds128_u32(s_out + r * (128 * NC) + (((ch & ~7) | ((ch ^ r) & 7)) * 16));
-    if (i < M && n < N) stg128(C + i * N + n, v);
+    if (i < M && n < N) {
+#pragma unroll
+      for (int d = 0; d < ND; ++d) {
+        if (d >= cd.n) break;
+        stg128(cd.p[d] + i * cd.ldc + n, v);
+      }
+    }
   }
 }
 
@@ -561,7 +598,20 @@ __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32, CpMinBlocks<SPLIT
                    const uint16_t* __restrict__ vals, const uint16_t* __restrict__ B,
                    uint16_t* __restrict__ C) {
   extern __shared__ __align__(128) unsigned char smem[];
-  spmm_cp_body<V, NC, SPLIT, D>(M, N, W, n_wgroups, blockIdx.x, row_ptr, col_idx, vals, B, C, smem);
+  const CDst<1> cd = {{C}, 1, N};
+  spmm_cp_body<V, NC, SPLIT, D, 1>(M, N, W, n_wgroups, blockIdx.x, row_ptr, col_idx, vals, B, cd, smem);
+}
+
+// vs_spmm_scatter, cp.async path: the same body, every output tile stored into cd.n destinations
+template <int V, int NC, int SPLIT, int D>
+__global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32, CpMinBlocks<SPLIT>::v)
+    spmm_cp_scatter_kernel(int64_t M, int64_t N, int64_t W, int64_t n_wgroups,
+                           const int32_t* __restrict__ row_ptr, const int32_t* __restrict__ col_idx,
+                           const uint16_t* __restrict__ vals, const uint16_t* __restrict__ B,
+                           const __grid_constant__ CDst<kMaxScatter> cd) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  spmm_cp_body<V, NC, SPLIT, D, kMaxScatter>(M, N, W, n_wgroups, blockIdx.x, row_ptr, col_idx, vals, B,
+                                             cd, smem);
 }
 
 template <int V, int NC, int SPLIT, int D>
@@ -574,8 +624,9 @@ __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32, CpMinBlocks<SPLIT
   for (int64_t bid = blockIdx.x; bid < total; bid += gridDim.x) {
     while (b.first_block[p + 1] <= bid) ++p;
     const SpmmDesc& d = b.d[p];
-    spmm_cp_body<V, NC, SPLIT, D>(d.M, d.N, d.W, d.n_wgroups, bid - b.first_block[p], d.row_ptr,
-                                  d.col_idx, d.vals, d.B, d.C, smem);
+    const CDst<1> cd = {{d.C}, 1, d.N};
+    spmm_cp_body<V, NC, SPLIT, D, 1>(d.M, d.N, d.W, d.n_wgroups, bid - b.first_block[p], d.row_ptr,
+                                     d.col_idx, d.vals, d.B, cd, smem);
   }
   pdl_wait_prior();
 }
@@ -619,7 +670,12 @@ static int64_t cp_smem_bytes(int V, int NC, int SPLIT, int D) {
   return warps * ((raw + 127) / 128 * 128);
 }
 
+static SpmmCfg spmm_config_al(int64_t K, int64_t N, int V, bool b_al16, bool c_al16);
 SpmmCfg spmm_config(int64_t K, int64_t N, int V, const void* B, const void* C) {
+  return spmm_config_al(K, N, V, (reinterpret_cast<uintptr_t>(B) & 15) == 0,
+                        (reinterpret_cast<uintptr_t>(C) & 15) == 0);
+}
+static SpmmCfg spmm_config_al(int64_t K, int64_t N, int V, bool b_al16, bool c_al16) {
   SpmmCfg c;
   c.V = V;
   // register path: 64-column panels (a K x 64 panel of B stays L1-resident for K <= ~1500;
@@ -630,8 +686,7 @@ SpmmCfg spmm_config(int64_t K, int64_t N, int V, const void* B, const void* C) {
   c.NC = (N <= 64 || VS_SPMM_NC != 2) ? 1 : 2;
   const int64_t q = K >> 8;
   c.SPLIT = q >= 16 ? 16 : q >= 8 ? 8 : q >= 4 ? 4 : q >= 2 ? 2 : 1;
-  c.VEC = (N % 8 == 0) && ((reinterpret_cast<uintptr_t>(B) & 15) == 0) &&
-          ((reinterpret_cast<uintptr_t>(C) & 15) == 0);
+  c.VEC = (N % 8 == 0) && b_al16 && c_al16;
   // cp.async path: 16-byte row copies and stores (VEC), vals copies of 2V >= 4 bytes; panel
   // width follows N (it does not change any element's accumulation order)
   c.CP = (c.VEC && V >= 2) ? spmm_cp_stages() : 0;
@@ -648,6 +703,8 @@ struct SpmmKernels {
   void (*single)(int64_t, int64_t, int64_t, int64_t, const int32_t*, const int32_t*,
                  const uint16_t*, const uint16_t*, uint16_t*);
   void (*batched)(SpmmBatch);
+  void (*scatter)(int64_t, int64_t, int64_t, int64_t, const int32_t*, const int32_t*,
+                  const uint16_t*, const uint16_t*, CDst<kMaxScatter>);
   int threads, units_per_cta, batched_ctas_per_sm;
   int smem;  // dynamic shared memory bytes (cp.async path), 0 otherwise
 };
@@ -666,9 +723,12 @@ static SpmmKernels cp_kernels_of() {
       cudaFuncSetAttribute(spmm_cp_kernel<V, NC, SPLIT, D>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
       cudaFuncSetAttribute(spmm_cp_batched_kernel<V, NC, SPLIT, D>,
                            cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+      cudaFuncSetAttribute(spmm_cp_scatter_kernel<V, NC, SPLIT, D>,
+                           cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     });
   }
   return {spmm_cp_kernel<V, NC, SPLIT, D>, spmm_cp_batched_kernel<V, NC, SPLIT, D>,
+          spmm_cp_scatter_kernel<V, NC, SPLIT, D>,
           SpmmCta<SPLIT>::kWarps * 32, SpmmCta<SPLIT>::kUnits, 0, smem};
 }
 
@@ -714,10 +774,9 @@ static constexpr int spmm_pipe() { return VS_SPMM_PIPE; }
 
 template <int V, int NC, bool VEC, int SPLIT>
 static SpmmKernels kernels_of() {
-  if (spmm_pipe())
-    return {spmm_kernel<V, NC, VEC, SPLIT, 0>, spmm_batched_kernel<V, NC, VEC, SPLIT, 0>,
-            SpmmCta<SPLIT>::kWarps * 32, SpmmCta<SPLIT>::kUnits, 0, 0};
-  return {spmm_kernel<V, NC, VEC, SPLIT, 1>, spmm_batched_kernel<V, NC, VEC, SPLIT, 1>,
+  constexpr int U = spmm_pipe() ? 0 : 1;
+  return {spmm_kernel<V, NC, VEC, SPLIT, U>, spmm_batched_kernel<V, NC, VEC, SPLIT, U>,
+          spmm_scatter_kernel<V, NC, VEC, SPLIT>,
           SpmmCta<SPLIT>::kWarps * 32, SpmmCta<SPLIT>::kUnits, 0, 0};
 }
 
@@ -777,6 +836,33 @@ cudaError_t launch_spmm(int64_t M, int64_t K, int64_t N, int V, const int32_t* r
                                                      static_cast<const uint16_t*>(vals),
                                                      static_cast<const uint16_t*>(B),
                                                      static_cast<uint16_t*>(C));
+  return cudaGetLastError();
+}
+
+// vs_spmm_scatter: the launch of vs_spmm, every output tile stored into n_dst destinations
+// (row-major, leading dimension ldc).  The 16-byte store path needs every destination and
+// ldc * 2 bytes 16-byte aligned (and B aligned, N % 8 == 0), as for vs_spmm.
+cudaError_t launch_spmm_scatter(int64_t M, int64_t K, int64_t N, int V, const int32_t* row_ptr,
+                                const int32_t* col_idx, const void* vals, const void* B,
+                                void* const* C_dst, int n_dst, int64_t ldc, cudaStream_t s) {
+  if (n_dst < 1 || n_dst > kMaxScatter) return cudaErrorInvalidValue;
+  bool c_al = (ldc % 8) == 0;
+  CDst<kMaxScatter> cd = {};
+  for (int d = 0; d < n_dst; ++d) {
+    cd.p[d] = static_cast<uint16_t*>(C_dst[d]);
+    c_al = c_al && ((reinterpret_cast<uintptr_t>(C_dst[d]) & 15) == 0);
+  }
+  cd.n = n_dst;
+  cd.ldc = ldc;
+  const SpmmCfg c = spmm_config_al(K, N, V, (reinterpret_cast<uintptr_t>(B) & 15) == 0, c_al);
+  const SpmmKernels k = pick(c);
+  int64_t W, nwg;
+  const int64_t grid = spmm_blocks(k, c, M, N, V, &W, &nwg);
+  if (grid > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
+  if (grid == 0) return cudaSuccess;
+  k.scatter<<<(unsigned)grid, k.threads, k.smem, s>>>(M, N, W, nwg, row_ptr, col_idx,
+                                                      static_cast<const uint16_t*>(vals),
+                                                      static_cast<const uint16_t*>(B), cd);
   return cudaGetLastError();
 }
 

@@ -12,6 +12,9 @@ cudaError_t launch_encode(int64_t M, int64_t K, int V, const void* dense, const 
 cudaError_t launch_spmm(int64_t M, int64_t K, int64_t N, int V, const int32_t* row_ptr,
                         const int32_t* col_idx, const void* vals, const void* B, void* C,
                         int num_sms, cudaStream_t s);
+cudaError_t launch_spmm_scatter(int64_t M, int64_t K, int64_t N, int V, const int32_t* row_ptr,
+                                const int32_t* col_idx, const void* vals, const void* B,
+                                void* const* C_dst, int n_dst, int64_t ldc, cudaStream_t s);
 cudaError_t launch_sddmm(int64_t M, int64_t N, int64_t K, int V, const int32_t* row_ptr,
                          const int32_t* col_idx, const void* A, const void* Bt, void* out,
                          int num_sms, cudaStream_t s);
@@ -183,6 +186,30 @@ vs_status_t vs_spmm(int64_t M, int64_t K, int64_t N, int V, const int32_t* row_p
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   if (K == 0) return from_cuda(cudaMemsetAsync(C, 0, (size_t)(M * N) * 2, s));
   return from_cuda(vs::launch_spmm(M, K, N, V, row_ptr, col_idx, vals, B, C, info.num_sms, s));
+}
+
+vs_status_t vs_spmm_scatter(int64_t M, int64_t K, int64_t N, int V, const int32_t* row_ptr,
+                            const int32_t* col_idx, const void* vals, const void* B,
+                            void* const* C_dst, int n_dst, int64_t ldc, vs_stream_t stream) {
+  if (C_dst == nullptr || n_dst < 1 || n_dst > VS_SPMM_SCATTER_MAX || ldc < N)
+    return VS_ERROR_INVALID_VALUE;
+  for (int d = 0; d < n_dst; ++d) {
+    // each destination is checked like vs_spmm's C
+    const vs_status_t st = check_spmm(M, K, N, V, row_ptr, col_idx, vals, B, C_dst[d]);
+    if (st != VS_SUCCESS) return st;
+  }
+  if (M == 0 || N == 0) return VS_SUCCESS;
+  DevInfo info;
+  vs_status_t st = check_device(&info);
+  if (st != VS_SUCCESS) return st;
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  if (K == 0) {  // zero fill of the N columns of every destination
+    for (int d = 0; d < n_dst; ++d)
+      if (cudaMemset2DAsync(C_dst[d], (size_t)ldc * 2, 0, (size_t)N * 2, (size_t)M, s) != cudaSuccess)
+        return VS_ERROR_CUDA;
+    return VS_SUCCESS;
+  }
+  return from_cuda(vs::launch_spmm_scatter(M, K, N, V, row_ptr, col_idx, vals, B, C_dst, n_dst, ldc, s));
 }
 
 vs_status_t vs_sddmm(int64_t M, int64_t N, int64_t K, int V, const int32_t* row_ptr,

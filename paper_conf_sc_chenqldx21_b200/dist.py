@@ -24,7 +24,8 @@ from dataclasses import dataclass
 import numpy as np
 
 __all__ = ["panel_bounds", "window_bounds", "SddmmShard", "sddmm_shard", "spmm_npanel",
-           "sddmm_rowwin", "gather_panels", "gather_segments"]
+           "sddmm_rowwin", "gather_panels", "gather_segments", "scatter_dst_ptrs",
+           "ReplicatedC", "spmm_npanel_replicated"]
 
 
 def panel_bounds(N: int, world: int, align: int = 64) -> list:
@@ -123,3 +124,55 @@ def gather_segments(segment, counts: list, group=None):
     dist.all_gather_into_tensor(recv, send, group=group)
     recv = recv.view(world, cmax)
     return torch.cat([recv[i, :counts[i]] for i in range(world)])
+
+
+# ------------------------------------------- fused replicated-output epilogue (§8(f)-4)
+#
+# Instead of computing the panel into a local buffer and all-gathering + permuting it
+# (gather_panels), every rank's SpMM epilogue stores its C tiles straight into EVERY rank's
+# row-major C [M x N] (vs_spmm_scatter): the C buffers are symmetric memory
+# (torch.distributed._symmetric_memory), so each rank holds device pointers to all peers'
+# buffers (NVLink / NVSwitch peer stores).  One barrier on the stream afterwards orders the
+# peers' reads after every rank's stores.  Same bits as gather_panels (same kernel body and
+# accumulation order; only the store addresses differ).
+
+def scatter_dst_ptrs(buffer_ptrs, n0: int, elem_bytes: int = 2) -> list:
+    """Destination pointers of this rank's panel [*, n0:...] in every rank's row-major C:
+    each peer buffer's base address + n0 elements."""
+    return [int(p) + int(n0) * elem_bytes for p in buffer_ptrs]
+
+
+class ReplicatedC:
+    """Symmetric-memory C [M x N] fp16 on this rank, rendezvoused over ``group``; holds the
+    peer pointers the scatter epilogue writes to."""
+
+    def __init__(self, M: int, N: int, device, group=None):
+        import torch
+        import torch.distributed as dist
+        import torch.distributed._symmetric_memory as symm_mem
+        self.M, self.N = M, N
+        self.group = group if group is not None else dist.group.WORLD
+        self.C = symm_mem.empty((M, N), dtype=torch.float16, device=device)
+        self.hdl = symm_mem.rendezvous(self.C, self.group)
+        self.world = self.hdl.world_size
+        self.buffer_ptrs = list(self.hdl.buffer_ptrs)
+
+    def barrier(self):
+        """Stream-ordered barrier across the ranks: after it, every rank's stores into every
+        replica are visible to this rank."""
+        self.hdl.barrier(channel=0)
+
+
+def spmm_npanel_replicated(row_ptr, col_idx, vals, B_panel, M: int, V: int, bounds: list,
+                           rank: int, rep: "ReplicatedC", barrier: bool = True):
+    """This rank's panel of C = A B, stored by the kernel epilogue into every rank's
+    replicated row-major C (rep.C holds the full C on every rank after the barrier)."""
+    from . import vs_spmm_scatter
+    K, Np = B_panel.shape
+    n0 = bounds[rank]
+    assert bounds[rank + 1] - n0 == Np and rep.N == bounds[-1]
+    vs_spmm_scatter(M, K, Np, V, row_ptr, col_idx, vals, B_panel,
+                    scatter_dst_ptrs(rep.buffer_ptrs, n0), rep.N)
+    if barrier:
+        rep.barrier()
+    return rep.C

@@ -67,6 +67,16 @@ def test_host_argument_checks_before_any_device_work(lib):
     assert lib.vs_encode_colvec(8, 8, 4, None, None, fake, None, None, None, None) == 1
     assert lib.vs_spmm(8, 8, 8, 4, P(4098), fake, fake, fake, fake, None) == 4  # row_ptr misaligned
     assert lib.vs_sddmm(8, 8, 8, 4, fake, fake, P(4097), fake, fake, None) == 4  # A misaligned
+    lib.vs_spmm_scatter.argtypes = [i64, i64, i64, ctypes.c_int, P, P, P, P,
+                                    ctypes.POINTER(P), ctypes.c_int, i64, P]
+    dsts = (P * 2)(4096, 8192)
+    assert lib.vs_spmm_scatter(8, 8, 8, 4, fake, fake, fake, fake, None, 1, 8, None) == 1
+    assert lib.vs_spmm_scatter(8, 8, 8, 4, fake, fake, fake, fake, dsts, 0, 8, None) == 1
+    assert lib.vs_spmm_scatter(8, 8, 8, 4, fake, fake, fake, fake, dsts, 9, 8, None) == 1
+    assert lib.vs_spmm_scatter(8, 8, 8, 4, fake, fake, fake, fake, dsts, 2, 7, None) == 1  # ldc < N
+    bad = (P * 2)(4096, 8193)
+    assert lib.vs_spmm_scatter(8, 8, 8, 4, fake, fake, fake, fake, bad, 2, 8, None) == 4
+    assert lib.vs_spmm_scatter(0, 8, 8, 4, fake, fake, fake, fake, dsts, 2, 8, None) == 0
 
 
 def test_no_shared_code_between_oracle_and_cuda_path():

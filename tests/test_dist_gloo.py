@@ -123,3 +123,70 @@ def test_two_rank_gloo_sharding_matches_unsharded():
         assert ok_spmm, f"rank {r}: gathered SpMM panels differ from the unsharded result"
         assert ok_sddmm, f"rank {r}: gathered SDDMM segments differ from the unsharded result"
         assert nloc > 0
+
+
+# ------------------------------------------- bench.py multi-GPU launcher and C5 plan
+
+def test_bench_launch_command_and_world_check(monkeypatch):
+    """`bench.py --gpus N` outside torchrun re-launches itself as N ranks (one node,
+    127.0.0.1); under torchrun a WORLD_SIZE that disagrees with --gpus is an error, never a
+    silent 1-GPU run."""
+    import bench
+    cmd = bench.launch_command(4, ["--gpus", "4", "--steps", "2"], port=12345)
+    assert cmd[1:3] == ["-m", "torch.distributed.run"]
+    assert "--nproc-per-node=4" in cmd and "--master-addr=127.0.0.1" in cmd
+    assert "--master-port=12345" in cmd and cmd[-3:] == ["--gpus", "4", "--steps", "2"][-3:]
+    assert cmd[cmd.index("--master-port=12345") + 1].endswith("bench.py")
+    monkeypatch.delenv("WORLD_SIZE", raising=False)
+    assert bench.check_world(bench.parse_args(["--gpus", "8"])) == "spawn"
+    assert bench.check_world(bench.parse_args(["--gpus", "1"])) == "run"
+    monkeypatch.setenv("WORLD_SIZE", "8")
+    assert bench.check_world(bench.parse_args(["--gpus", "8"])) == "run"
+    with pytest.raises(SystemExit):
+        bench.check_world(bench.parse_args(["--gpus", "4"]))
+    monkeypatch.setenv("WORLD_SIZE", "1")
+    with pytest.raises(SystemExit):
+        bench.check_world(bench.parse_args(["--gpus", "2"]))
+
+
+def _plan_worker(rank, world, port, results):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import bench
+        # the global C5 mask's row_ptr (same seed on every rank, as in bench.run_c5)
+        rng = gen.make_rng("c5_plan_rowptr")
+        counts = rng.binomial(65536, 0.1, size=2048)
+        rp = np.concatenate([[0], np.cumsum(counts)]).astype(np.int64)
+        plan = bench.c5_plan(world, rank, rp)
+        mine = (plan["n0"], plan["n1"], plan["shard"].w0, plan["shard"].w1,
+                plan["shard"].p1 - plan["shard"].p0)
+        allp = [None] * world
+        dist.all_gather_object(allp, mine)
+        results[rank] = (allp, plan["panel_bounds"], plan["window_bounds"], int(rp[-1]))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_c5_plan_partitions_cover_once(world):
+    mgr = mp.Manager()
+    results = mgr.dict()
+    mp.spawn(_plan_worker, args=(world, _free_port(), results), nprocs=world, join=True)
+    allp, pb, wb, nnz = results[0]
+    for r in range(world):
+        assert results[r][0] == allp and results[r][1] == pb and results[r][2] == wb
+    # panels tile [0, N) in whole 4096-column generator blocks; windows tile [0, W)
+    assert allp[0][0] == 0 and allp[-1][1] == 65536
+    assert all(allp[r][1] == allp[r + 1][0] for r in range(world - 1))
+    assert all(a[0] % 4096 == 0 for a in allp)
+    assert allp[0][2] == 0 and allp[-1][3] == 2048
+    assert all(allp[r][3] == allp[r + 1][2] for r in range(world - 1))
+    loads = [a[4] for a in allp]
+    assert sum(loads) == nnz and max(loads) - nnz / world <= 0.002 * nnz
+
+
+def test_scatter_dst_ptrs():
+    assert vsd.scatter_dst_ptrs([1000, 5000], 64) == [1128, 5128]
+    assert vsd.scatter_dst_ptrs([0], 0, elem_bytes=4) == [0]

@@ -1,7 +1,7 @@
-set -x
-nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o /tmp/mb tools/microbench.cu && /tmp/mb > gpurun_out/microbench_r02.jsonl 2>&1
-timeout 900 python -m pytest tests -m gpu -x -q 2>&1 | tail -25 > gpurun_out/gputests.log
-timeout 600 python tools/tune.py --op spmm --cfg VS_SPMM_CP=0 --cfg VS_SPMM_CP=3 --cfg VS_SPMM_CP=4 --cfg VS_SPMM_CP=6 --out gpurun_out/tune_spmm.json > gpurun_out/tune_spmm.log 2>&1
-timeout 600 python tools/tune.py --op spmm_batched --cfg VS_SPMM_CP=0 --cfg VS_SPMM_CP=3 --cfg VS_SPMM_CP=4 --cfg VS_SPMM_CP=6 --out gpurun_out/tune_spmmb.json > gpurun_out/tune_spmmb.log 2>&1
-timeout 600 python bench.py --no-baselines --no-cpu > gpurun_out/bench2.json 2> gpurun_out/bench2.err
-cat gpurun_out/microbench_r02.jsonl gpurun_out/gputests.log gpurun_out/tune_spmm.log gpurun_out/tune_spmmb.log
+#!/bin/bash
+# r02a: GPU suite after the round-2 parity additions + frozen knobs, then the default bench
+python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/r02a_smoke.log 2>&1
+timeout 1500 python -m pytest tests -m gpu -x -q > gpurun_out/r02a_gputest.log 2>&1
+echo "pytest rc=$?" >> gpurun_out/r02a_gputest.log
+timeout 600 python bench.py > gpurun_out/r02a_bench.json 2> gpurun_out/r02a_bench.err
+tail -3 gpurun_out/r02a_gputest.log

@@ -1,6 +1,7 @@
-set -x
-timeout 900 python -m pytest tests -m gpu -x -q 2>&1 | tail -5 > gpurun_out/gputests.log
-python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.log 2>&1
-timeout 600 python tools/tune.py --op sddmm_batched --cfg X=1 --out gpurun_out/tune_sddmmb.json > gpurun_out/tune_sddmmb.log 2>&1
-timeout 900 python bench.py > gpurun_out/bench.json 2> gpurun_out/bench.err
-cat gpurun_out/gputests.log gpurun_out/smoke.log gpurun_out/tune_sddmmb.log gpurun_out/bench.json
+#!/bin/bash
+# r02f: scatter / coverage tests, then C5 (1 GPU, strong-scaling point) and C4 (rn50) bench lines
+timeout 900 python -m pytest tests/test_gpu_scatter.py tests/test_gpu_coverage.py tests/test_gpu_transpose.py tests/test_gpu_attention.py -x -q > gpurun_out/r02f_tests.log 2>&1
+echo "rc=$?" >> gpurun_out/r02f_tests.log
+timeout 900 python bench.py --workload c5 --steps 3 --warmup 1 > gpurun_out/r02f_c5.json 2> gpurun_out/r02f_c5.err
+timeout 900 python bench.py --workload rn50_layer > gpurun_out/r02f_rn50.json 2> gpurun_out/r02f_rn50.err
+tail -2 gpurun_out/r02f_tests.log
