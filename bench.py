@@ -913,7 +913,7 @@ def c5_plan(ws: int, rank: int, mask_row_ptr=None):
     plan = {"M": M, "K": K, "N": N, "V": V, "S": S, "W": W, "panel_bounds": pb,
             "n0": pb[rank], "n1": pb[rank + 1]}
     if mask_row_ptr is not None:
-        wb = vsd.window_bounds(mask_row_ptr, ws)
+        wb = vsd.window_bounds(mask_row_ptr, ws, align=128 // V)
         sh = vsd.sddmm_shard(mask_row_ptr, M, V, wb, rank)
         plan.update({"window_bounds": wb, "shard": sh})
     return plan

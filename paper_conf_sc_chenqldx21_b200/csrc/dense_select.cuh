@@ -1,0 +1,66 @@
+// dense_select.cuh — which 128-row blocks of a problem take the dense-tile tcgen05 kernels
+// (dense_tile.cu) instead of the column-vector gather kernels (spmm.cu / sddmm.cu).
+//
+// B200 cost model.  A stored V x 1 vector costs the gather kernels one
+// gathered dense row: 2*L bytes through L2 -> SM (L = N for SpMM, the inner K for SDDMM),
+// i.e. V flop per gathered byte.  A dense 128-row tile costs 2 * 128 * Lc * L tensor flops
+// (Lc = the padded other dimension: K for SpMM, the mask columns for SDDMM) whatever the
+// density.  With the gather at Bg bytes/s and the tcgen05 tiles at Fd flop/s, the dense tile
+// is cheaper when  nnz_v(rb) * 2L / Bg  >  2 * 128 * Lc * L / Fd,  i.e.
+//     nnz_v(rb) * VS_DENSE_CF  >  128 * Lc,         VS_DENSE_CF = Fd / Bg  (flop per byte).
+// The decision depends only on the row block's vectors and the problem's shape, so the gather
+// kernels and the dense kernels (and any N-panel or 128-row-aligned row-window shard of the
+// problem) take it identically.  Windows of a dense row block whose col_idx is not strictly
+// ascending stay with the gather kernels (the dense kernels rely on sorted windows).
+#pragma once
+
+#include <stdint.h>
+
+#include "common.cuh"
+
+// VS_DENSE_CF = 0 (the shipped library): the dense-tile kernels are not built and never
+// launched; every row block stays with the gather kernels.  Measured on B200 (DESIGN.md §7.8,
+// profiles/r02_dense_tile.md): with the current dense-tile kernels a 32-row unit costs ~9-13 us
+// of pipeline latency, so over the DLMC set they beat the gather kernels only for the largest
+// 50%-sparse SDDMM problems; an opt-in build (-DVS_DENSE_CF=<flop per byte>) enables them.
+#ifndef VS_DENSE_CF
+#define VS_DENSE_CF 0
+#endif
+
+namespace vs {
+
+constexpr int kDenseRows = 128;  // rows per dense tile (tcgen05 M / N)
+
+// 128-row block rb of a problem with W windows of V rows: window range [w0, w1)
+__host__ __device__ __forceinline__ void rb_windows(int64_t rb, int V, int64_t W, int64_t& w0, int64_t& w1) {
+  w0 = rb * (kDenseRows / V);
+  w1 = w0 + kDenseRows / V;
+  if (w1 > W) w1 = W;
+}
+
+// dense iff nnz_v(rb) * CF > 128 * Lc (Lc padded to the dense tile granularity)
+__device__ __forceinline__ bool rb_is_dense(const int32_t* __restrict__ row_ptr, int64_t W, int V,
+                                            int64_t rb, int64_t Lc_padded) {
+  int64_t w0, w1;
+  rb_windows(rb, V, W, w0, w1);
+  const int64_t nnz = (int64_t)__ldg(row_ptr + w1) - (int64_t)__ldg(row_ptr + w0);
+  return nnz * (int64_t)VS_DENSE_CF > (int64_t)kDenseRows * Lc_padded;
+}
+
+// warp-uniform: col_idx[pb, pe) strictly ascending (every lane returns the same answer)
+__device__ __forceinline__ bool window_sorted(const int32_t* __restrict__ col_idx, int64_t pb, int64_t pe) {
+  const int lane = lane_id();
+  int prev_last = -1;  // last entry of the previous batch (entries are >= 0)
+  for (int64_t base = pb; base < pe; base += 32) {
+    const int64_t p = base + lane;
+    const int c = p < pe ? __ldg(col_idx + p) : 0x7fffffff;
+    int prev = __shfl_up_sync(0xffffffffu, c, 1);
+    if (lane == 0) prev = prev_last;
+    const bool bad = (p < pe) && (c <= prev);
+    if (__any_sync(0xffffffffu, bad)) return false;
+    prev_last = __shfl_sync(0xffffffffu, c, 31);
+  }
+  return true;
+}
+
+}  // namespace vs

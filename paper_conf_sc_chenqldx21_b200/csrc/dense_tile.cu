@@ -1,0 +1,744 @@
+// dense_tile.cu — dense-tile tcgen05 kernels for the 128-row blocks the B200 cost model
+// (dense_select.cuh) sends away from the column-vector gather kernels.
+//
+// Why: a stored V x 1 vector gives the gather kernels V flop per gathered byte
+// (AL1), and B200 moves ~8-20 TB/s of random rows from L2 into the SMs against
+// ~1.5-2 PFLOP/s of dense fp16 tensor throughput.  Where a 128-row block holds more than
+// 128 * Lc / VS_DENSE_CF stored vectors, computing its whole dense tile on the tensor cores
+// costs less than gathering its vectors.  The results are the same sums (fp32 accumulate,
+// fp16 round-to-nearest-even output); absent vectors only add exact zero products (SpMM) or
+// are not stored (SDDMM).
+//
+// SDDMM  out[p*V + r] = sum_k A[wV+r][k] * Bt[col_idx[p]][k]   (§6)
+//   Unit = (problem, 32-row block of A = rows [i0, i0+32), range of <= 1024 mask columns).
+//   Per column tile c0 (128 mask columns): D[128 mask cols x 32 A rows] (fp32, TMEM) =
+//   Bt[c0:c0+128, :] * A[i0:i0+32, :]^T, tcgen05.mma M = 128, N = 32, K = 16 (operand switch
+//   of P:1059-1063: mask columns on the MMA M side); both operands are K-contiguous rows loaded
+//   by TMA 2-D tile copies (SWIZZLE_128B = the canonical K-major layout); the A rows of the unit
+//   (K <= 256) stay resident in shared memory.  Each finished tile is drained TMEM -> fp16 (RN)
+//   into a shared [32 rows x 1024 columns] tile, so the whole column range of the unit is on
+//   chip; then ONE flat pass over the unit's stored vectors (contiguous in col_idx: the windows
+//   of the 32 rows) writes out[p*V .. p*V+V) for every vector whose column is in the range --
+//   any col_idx order, duplicates included, coalesced 2V-byte stores.
+//   Warp roles: warp 0 TMA producer, warp 1 MMA issuer (one elected lane) + TMEM owner,
+//   warps 2-9 epilogue (TMEM lane quarter = warp % 4, column half = (warp - 2) / 4).  Two TMEM
+//   accumulators: the drain of tile t overlaps the MMAs of tile t + 1.
+//
+// SpMM  C[i][n] = sum_p vals[p*V + i%V] * B[col_idx[p]][n]   (§5)
+//   Unit = (problem, 32-row block of A / C).  The unit's stored vectors (contiguous: the
+//   windows of the 32 rows) are decoded once into a dense [32 rows x K] fp16 tile in shared
+//   memory (K-major, 128-byte swizzle; K <= 2048), then for every 128-column panel of B:
+//   D[128 panel cols x 32 rows] (fp32, TMEM) = B[:, n0:n0+128]^T * A_tile^T with tcgen05.mma
+//   M = 128, N = 32, K = 16 (the operand switch of P:858-871: B columns on the MMA M side, B
+//   MN-major straight from TMA 2-D tiles), and the epilogue stores the tile into C (fp16 RN;
+//   to every destination of vs_spmm_scatter).  Absent vectors are exact zeros of the tile.
+//   A window whose col_idx is not strictly ascending (duplicates, any order) is not taken here:
+//   its rows are left to the gather kernel, which checks the same condition.
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
+#include <algorithm>
+#include <mutex>
+#include <vector>
+
+#include "common.cuh"
+#include "dense_select.cuh"
+#include "tc_common.cuh"
+
+#if VS_DENSE_CF > 0  // opt-in build only (dense_select.cuh)
+namespace vs {
+namespace dt {
+
+constexpr int kCtPerUnit = 8;   // column tiles of 128 per SDDMM unit (1024 columns)
+constexpr int kMaxProb = 32;    // problems per launch (tensor maps travel as kernel parameters)
+constexpr int kSdRows = 32;     // A rows per SDDMM unit (MMA N)
+constexpr int kSdThreads = 320; // 10 warps
+constexpr int kSdEpi = 256;     // epilogue threads (warps 2-9)
+constexpr int kBtTile = 128 * 128;        // 128 mask columns x 64 k fp16 (16 KB)
+constexpr int kATile = kSdRows * 128;     // 32 rows x 64 k fp16 (4 KB)
+constexpr int kSdKbMax = 4;               // K <= 256 (A resident)
+constexpr int kSdStages = 8;   // 128 KB of Bt tiles in flight per SM (the stream is latency-bound)
+constexpr int kSdDhBytes = kSdRows * kCtPerUnit * 128 * 2;  // 64 KB
+constexpr int kSdSmem = kSdKbMax * kATile + kSdStages * kBtTile + kSdDhBytes + 1024;
+constexpr uint32_t kIdescSd = tc::idesc_f16(128, kSdRows, 0, 0);
+
+struct alignas(64) SdDesc {
+  CUtensorMap tmA;   // A [M x K] fp16, box {64, 32}, SWIZZLE_128B
+  CUtensorMap tmBt;  // Bt [N x K] fp16, box {64, 128}, SWIZZLE_128B
+  int64_t M, N, K, W, n_cr, n_rb;
+  const int32_t* row_ptr;
+  const int32_t* col_idx;
+  uint16_t* out;
+  int64_t nnz_total;  // (not known on the host: unused)
+  int32_t V, out_vec;  // out_vec: out is 2V-byte aligned (one store per vector)
+};
+struct SdBatch {
+  int count;
+  int64_t first_unit[kMaxProb + 1];
+  SdDesc d[kMaxProb];
+};
+
+// unit -> (problem, 32-row block, column-tile range); problems in ascending unit order
+struct UnitIt {
+  int p;
+  __device__ __forceinline__ void locate(const SdBatch& b, int64_t u, int64_t& rb, int64_t& ct0,
+                                         int64_t& ct1) {
+    while (b.first_unit[p + 1] <= u) ++p;
+    const SdDesc& d = b.d[p];
+    const int64_t loc = u - b.first_unit[p];
+    rb = loc / d.n_cr;
+    const int64_t cr = loc - rb * d.n_cr;
+    const int64_t nct = ceil_div64(d.N, 128);
+    ct0 = cr * kCtPerUnit;
+    ct1 = ct0 + kCtPerUnit < nct ? ct0 + kCtPerUnit : nct;
+  }
+};
+
+// the 32-row block rb32 belongs to the 128-row block of the dense/gather decision
+__device__ __forceinline__ bool sd_unit_dense(const SdDesc& d, int64_t rb32) {
+  return rb_is_dense(d.row_ptr, d.W, d.V, rb32 / (kDenseRows / kSdRows), ceil_div64(d.N, 128) * 128);
+}
+
+__global__ void __launch_bounds__(kSdThreads, 1) sddmm_dense_kernel(const __grid_constant__ SdBatch b) {
+  extern __shared__ uint8_t smem_raw[];
+  __shared__ __align__(8) uint64_t full_bar[kSdStages], empty_bar[kSdStages];
+  __shared__ __align__(8) uint64_t tfull_bar[2], tempty_bar[2], afull_bar, aempty_bar;
+  __shared__ uint32_t tmem_base_sh;
+  __shared__ int32_t wptr[kSdRows + 1];  // row_ptr of the unit's windows (relative to nothing)
+  const uint32_t smem = (smem_u32(smem_raw) + 1023u) & ~1023u;
+  const uint32_t s_ares = smem;                            // A tiles of the unit (kSdKbMax x 4 KB)
+  const uint32_t s_stage = smem + kSdKbMax * kATile;       // Bt stage ring
+  const uint32_t s_dh = s_stage + kSdStages * kBtTile;     // Dh [32 rows][2048 cols] fp16
+  const int warp = threadIdx.x >> 5, lane = lane_id();
+  const int64_t total = b.first_unit[b.count];
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < kSdStages; ++s) {
+      tc::mbar_init(smem_u32(&full_bar[s]), 1);
+      tc::mbar_init(smem_u32(&empty_bar[s]), 1);
+    }
+    for (int a = 0; a < 2; ++a) {
+      tc::mbar_init(smem_u32(&tfull_bar[a]), 1);
+      tc::mbar_init(smem_u32(&tempty_bar[a]), 8);  // one arrive per epilogue warp
+    }
+    tc::mbar_init(smem_u32(&afull_bar), 1);
+    tc::mbar_init(smem_u32(&aempty_bar), 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 64;" ::"r"(
+        smem_u32(&tmem_base_sh)));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  tc::fence_before();
+  __syncthreads();
+  tc::fence_after();
+  const uint32_t tmem = tmem_base_sh;
+
+  UnitIt it{0};
+  if (warp == 0) {
+    // ================================ TMA producer ================================
+    uint32_t s = 0, ph = 0, au = 0;
+    for (int64_t u = blockIdx.x; u < total; u += gridDim.x) {
+      int64_t rb, ct0, ct1;
+      it.locate(b, u, rb, ct0, ct1);
+      const SdDesc& d = b.d[it.p];
+      if (!sd_unit_dense(d, rb)) continue;
+      const int KB = (int)ceil_div64(d.K, 64);
+      // the unit's first kSdStages Bt stages go out while the previous unit's MMAs finish;
+      // its A tiles as soon as those MMAs released the resident A buffer
+      const int64_t nslots = (ct1 - ct0) * KB;
+      int64_t j = 0;
+      auto load_a = [&]() {
+        tc::mbar_wait(smem_u32(&aempty_bar), (au & 1) ^ 1);
+        if (lane == 0) {
+          tc::mbar_expect_tx(smem_u32(&afull_bar), KB * kATile);
+          for (int kb = 0; kb < KB; ++kb)
+            tc::tma_load_2d(s_ares + kb * kATile, &d.tmA, kb * 64, (int)(rb * kSdRows), smem_u32(&afull_bar));
+        }
+        __syncwarp();
+        ++au;
+      };
+      for (int64_t ct = ct0; ct < ct1; ++ct) {
+        for (int kb = 0; kb < KB; ++kb, ++j) {
+          if (j == (nslots - 1 < kSdStages ? nslots - 1 : kSdStages)) load_a();
+          tc::mbar_wait(smem_u32(&empty_bar[s]), ph ^ 1);
+          if (lane == 0) {
+            tc::mbar_expect_tx(smem_u32(&full_bar[s]), kBtTile);
+            tc::tma_load_2d(s_stage + s * kBtTile, &d.tmBt, kb * 64, (int)(ct * 128), smem_u32(&full_bar[s]));
+          }
+          __syncwarp();
+          if (++s == kSdStages) { s = 0; ph ^= 1; }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    // ================================ MMA issuer ================================
+    uint32_t s = 0, ph = 0, au = 0, tile = 0;
+    for (int64_t u = blockIdx.x; u < total; u += gridDim.x) {
+      int64_t rb, ct0, ct1;
+      it.locate(b, u, rb, ct0, ct1);
+      const SdDesc& d = b.d[it.p];
+      if (!sd_unit_dense(d, rb)) continue;
+      const int KB = (int)ceil_div64(d.K, 64);
+      tc::mbar_wait(smem_u32(&afull_bar), au & 1);
+      tc::fence_after();
+      for (int64_t ct = ct0; ct < ct1; ++ct) {
+        const uint32_t acc = tile & 1;
+        tc::mbar_wait(smem_u32(&tempty_bar[acc]), ((tile >> 1) & 1) ^ 1);
+        tc::fence_after();
+        for (int kb = 0; kb < KB; ++kb) {
+          tc::mbar_wait(smem_u32(&full_bar[s]), ph);
+          tc::fence_after();
+          if (lane == 0) {
+            const uint32_t st = s_stage + s * kBtTile;
+            const uint32_t at = s_ares + kb * kATile;
+#pragma unroll
+            for (int k = 0; k < 4; ++k)
+              tc::mma(tmem + acc * kSdRows, tc::sdesc(st + 32 * k, 16, 1024), tc::sdesc(at + 32 * k, 16, 1024),
+                      kIdescSd, (kb > 0 || k > 0) ? 1u : 0u);
+            tc::commit(smem_u32(&empty_bar[s]));
+          }
+          __syncwarp();
+          if (++s == kSdStages) { s = 0; ph ^= 1; }
+        }
+        if (lane == 0) tc::commit(smem_u32(&tfull_bar[acc]));
+        __syncwarp();
+        ++tile;
+      }
+      if (lane == 0) tc::commit(smem_u32(&aempty_bar));
+      __syncwarp();
+      ++au;
+    }
+  } else {
+    // ================================ epilogue ================================
+    const int et = threadIdx.x - 64;   // 0..255
+    const int q = warp & 3;            // TMEM lane quarter (tcgen05.ld restriction: warp % 4)
+    const int h = (warp - 2) >> 2;     // column half of the accumulator: rows 16h .. 16h+15
+    uint32_t tile = 0;
+    for (int64_t u = blockIdx.x; u < total; u += gridDim.x) {
+      int64_t rb, ct0, ct1;
+      it.locate(b, u, rb, ct0, ct1);
+      const SdDesc& d = b.d[it.p];
+      if (!sd_unit_dense(d, rb)) continue;
+      const int V = d.V;
+      const int64_t i0 = rb * kSdRows;
+      const int64_t w0 = i0 / V;
+      const int64_t w1 = (i0 + kSdRows) / V < d.W ? (i0 + kSdRows) / V : d.W;
+      const int nwin = (int)(w1 - w0);
+      // ---- drain every column tile of the range into Dh (fp16 RN; rows >= M are +0)
+      for (int64_t ct = ct0; ct < ct1; ++ct) {
+        const uint32_t acc = tile & 1;
+        tc::mbar_wait(smem_u32(&tfull_bar[acc]), (tile >> 1) & 1);
+        tc::fence_after();
+        uint32_t v[16];
+        asm volatile(
+            "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+            : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+              "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]),
+              "=r"(v[15])
+            : "r"(tmem + ((uint32_t)(32 * q) << 16) + acc * kSdRows + 16 * h));
+        tc::ld_wait();
+        tc::fence_before();
+        __syncwarp();
+        if (lane == 0) tc::mbar_arrive(smem_u32(&tempty_bar[acc]));
+        const int col = (int)(ct - ct0) * 128 + 32 * q + lane;  // column within the range
+#pragma unroll
+        for (int x = 0; x < 16; ++x) {
+          const int r = 16 * h + x;
+          const float f = (i0 + r < d.M) ? __uint_as_float(v[x]) : 0.f;
+          asm volatile("st.shared.u16 [%0], %1;" ::"r"(s_dh + (uint32_t)((r * (kCtPerUnit * 128) + col) * 2)),
+                       "h"(f_to_h(f))
+                       : "memory");
+        }
+        ++tile;
+      }
+      if (et <= nwin) wptr[et] = __ldg(d.row_ptr + w0 + et);
+      tc::named_bar(1, kSdEpi);  // Dh and wptr complete
+      // ---- one flat pass over the unit's stored vectors [P0, P1)
+      const int64_t P0 = wptr[0], P1 = wptr[nwin];
+      const int64_t cbeg = ct0 * 128, cend = ct1 * 128;
+      // groups of 4 entries at 16-byte aligned addresses of col_idx (any base alignment)
+      const int64_t off = (int64_t)((reinterpret_cast<uintptr_t>(d.col_idx) >> 2) & 3);
+      const int64_t Pa = ((P0 + off) & ~(int64_t)3) - off;
+      for (int64_t base = Pa + 4 * et; base < P1; base += 4 * kSdEpi) {
+        int c4[4];
+        if (base >= P0 && base + 3 < P1) {
+          const int4 t = __ldg(reinterpret_cast<const int4*>(d.col_idx + base));
+          c4[0] = t.x; c4[1] = t.y; c4[2] = t.z; c4[3] = t.w;
+        } else {
+#pragma unroll
+          for (int j = 0; j < 4; ++j) c4[j] = (base + j >= P0 && base + j < P1) ? __ldg(d.col_idx + base + j) : -1;
+        }
+        // window of the first entry (binary search), then advance
+        const int64_t pf = base < P0 ? P0 : base;
+        int lo = 0, hi = nwin - 1;
+        while (lo < hi) {
+          const int mid = (lo + hi + 1) >> 1;
+          if (wptr[mid] <= pf) lo = mid; else hi = mid - 1;
+        }
+        int wl = lo;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const int64_t p = base + j;
+          if (p < P0 || p >= P1) continue;
+          while (wptr[wl + 1] <= p) ++wl;
+          const int64_t c = c4[j];
+          if (c < cbeg || c >= cend) continue;
+          const uint32_t a = s_dh + (uint32_t)(((int64_t)(wl * V) * (kCtPerUnit * 128) + (c - cbeg)) * 2);
+          uint16_t hv[8];
+#pragma unroll
+          for (int r = 0; r < 8; ++r) hv[r] = r < V ? lds16(a + (uint32_t)(r * kCtPerUnit * 128 * 2)) : (uint16_t)0;
+          uint16_t* dst = d.out + p * V;
+          if (d.out_vec) {
+            if (V == 8) *reinterpret_cast<uint4*>(dst) = make_uint4(pack_h2(hv[0], hv[1]), pack_h2(hv[2], hv[3]),
+                                                                   pack_h2(hv[4], hv[5]), pack_h2(hv[6], hv[7]));
+            else if (V == 4) *reinterpret_cast<uint2*>(dst) = make_uint2(pack_h2(hv[0], hv[1]), pack_h2(hv[2], hv[3]));
+            else *reinterpret_cast<uint32_t*>(dst) = pack_h2(hv[0], hv[1]);
+          } else {
+            for (int r = 0; r < V; ++r) dst[r] = hv[r];
+          }
+        }
+      }
+      tc::named_bar(1, kSdEpi);  // Dh / wptr reads done before the next unit's drain
+    }
+  }
+
+  tc::fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc::fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 64;" ::"r"(tmem));
+  }
+}
+
+// ================================================================================ SpMM
+constexpr int kSpRows = 32;            // A / C rows per unit (MMA N)
+constexpr int kSpThreads = 320;        // 10 warps
+constexpr int kSpEpi = 256;            // decode / epilogue threads (warps 2-9)
+constexpr int kSpKbMax = 32;           // K <= 2048: the decoded A tile stays resident
+constexpr int kSpStages = 4;
+constexpr int kBPanel = 64 * 128 * 2;  // B tile: 64 k x 128 n fp16 = 2 slabs of 64 n (16 KB)
+constexpr int kSpSmem = kSpKbMax * kATile + kSpStages * kBPanel + 1024;
+constexpr uint32_t kIdescSp = tc::idesc_f16(128, kSpRows, 1, 0);
+constexpr int kMaxDst = 8;
+
+struct alignas(64) SpDesc {
+  CUtensorMap tmB;  // B [K x N] fp16 (N contiguous), box {64 n, 64 k}, SWIZZLE_128B
+  int64_t M, K, N, W, n_rb;
+  const int32_t* row_ptr;
+  const int32_t* col_idx;
+  const uint16_t* vals;
+  uint16_t* C[kMaxDst];
+  int64_t ldc;
+  int32_t V, nC;
+};
+struct SpBatch {
+  int count;
+  int64_t first_unit[kMaxProb + 1];
+  SpDesc d[kMaxProb];
+};
+
+__device__ __forceinline__ bool sp_unit_dense(const SpDesc& d, int64_t rb32) {
+  return rb_is_dense(d.row_ptr, d.W, d.V, rb32 / (kDenseRows / kSpRows), ceil_div64(d.K, 64) * 64);
+}
+
+// byte offset of element (row, k) in the decoded K-major 128-byte-swizzled A tile
+__device__ __forceinline__ uint32_t adec_off(int row, int k) {
+  const int kb = k >> 6, kk = k & 63, rr = row & 7;
+  return (uint32_t)(kb * kATile + (row >> 3) * 1024 + rr * 128 + ((((kk >> 3) ^ rr)) << 4) + (kk & 7) * 2);
+}
+
+__global__ void __launch_bounds__(kSpThreads, 1) spmm_dense_kernel(const __grid_constant__ SpBatch b) {
+  extern __shared__ uint8_t smem_raw[];
+  __shared__ __align__(8) uint64_t full_bar[kSpStages], empty_bar[kSpStages];
+  __shared__ __align__(8) uint64_t tfull_bar[2], tempty_bar[2], afull_bar, aempty_bar;
+  __shared__ uint32_t tmem_base_sh;
+  __shared__ int32_t wptr[kSpRows + 1];
+  __shared__ int32_t unsorted[kSpRows];
+  const uint32_t smem = (smem_u32(smem_raw) + 1023u) & ~1023u;
+  const uint32_t s_adec = smem;                          // decoded A tile (kSpKbMax x 4 KB)
+  const uint32_t s_stage = smem + kSpKbMax * kATile;     // B stage ring
+  const int warp = threadIdx.x >> 5, lane = lane_id();
+  const int64_t total = b.first_unit[b.count];
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < kSpStages; ++s) {
+      tc::mbar_init(smem_u32(&full_bar[s]), 1);
+      tc::mbar_init(smem_u32(&empty_bar[s]), 1);
+    }
+    for (int a = 0; a < 2; ++a) {
+      tc::mbar_init(smem_u32(&tfull_bar[a]), 1);
+      tc::mbar_init(smem_u32(&tempty_bar[a]), 8);
+    }
+    tc::mbar_init(smem_u32(&afull_bar), 1);   // the decoders (one elected arrive)
+    tc::mbar_init(smem_u32(&aempty_bar), 1);  // MMA commit after the unit's last MMA
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 64;" ::"r"(
+        smem_u32(&tmem_base_sh)));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  tc::fence_before();
+  __syncthreads();
+  tc::fence_after();
+  const uint32_t tmem = tmem_base_sh;
+
+  int p = 0;  // problem cursor
+  auto locate = [&](int64_t u) -> int64_t {
+    while (b.first_unit[p + 1] <= u) ++p;
+    return u - b.first_unit[p];
+  };
+  if (warp == 0) {
+    // ================================ TMA producer (B tiles) ================================
+    uint32_t s = 0, ph = 0;
+    for (int64_t u = blockIdx.x; u < total; u += gridDim.x) {
+      const int64_t rb = locate(u);
+      const SpDesc& d = b.d[p];
+      if (!sp_unit_dense(d, rb)) continue;
+      const int KB = (int)ceil_div64(d.K, 64);
+      for (int64_t n0 = 0; n0 < d.N; n0 += 128) {
+        for (int kb = 0; kb < KB; ++kb) {
+          tc::mbar_wait(smem_u32(&empty_bar[s]), ph ^ 1);
+          if (lane == 0) {
+            const uint32_t st = s_stage + s * kBPanel;
+            tc::mbar_expect_tx(smem_u32(&full_bar[s]), kBPanel);
+            tc::tma_load_2d(st, &d.tmB, (int)n0, kb * 64, smem_u32(&full_bar[s]));
+            tc::tma_load_2d(st + kBPanel / 2, &d.tmB, (int)n0 + 64, kb * 64, smem_u32(&full_bar[s]));
+          }
+          __syncwarp();
+          if (++s == kSpStages) { s = 0; ph ^= 1; }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    // ================================ MMA issuer ================================
+    uint32_t s = 0, ph = 0, au = 0, tile = 0;
+    for (int64_t u = blockIdx.x; u < total; u += gridDim.x) {
+      const int64_t rb = locate(u);
+      const SpDesc& d = b.d[p];
+      if (!sp_unit_dense(d, rb)) continue;
+      const int KB = (int)ceil_div64(d.K, 64);
+      tc::mbar_wait(smem_u32(&afull_bar), au & 1);  // decoded A tile of this unit
+      tc::fence_after();
+      for (int64_t n0 = 0; n0 < d.N; n0 += 128) {
+        const uint32_t acc = tile & 1;
+        tc::mbar_wait(smem_u32(&tempty_bar[acc]), ((tile >> 1) & 1) ^ 1);
+        tc::fence_after();
+        for (int kb = 0; kb < KB; ++kb) {
+          tc::mbar_wait(smem_u32(&full_bar[s]), ph);
+          tc::fence_after();
+          if (lane == 0) {
+            const uint32_t st = s_stage + s * kBPanel;
+            const uint32_t at = s_adec + kb * kATile;
+#pragma unroll
+            for (int k = 0; k < 4; ++k)
+              tc::mma(tmem + acc * kSpRows, tc::sdesc(st + 2048 * k, kBPanel / 2, 1024),
+                      tc::sdesc(at + 32 * k, 16, 1024), kIdescSp, (kb > 0 || k > 0) ? 1u : 0u);
+            tc::commit(smem_u32(&empty_bar[s]));
+          }
+          __syncwarp();
+          if (++s == kSpStages) { s = 0; ph ^= 1; }
+        }
+        if (lane == 0) tc::commit(smem_u32(&tfull_bar[acc]));
+        __syncwarp();
+        ++tile;
+      }
+      if (lane == 0) tc::commit(smem_u32(&aempty_bar));  // A tile free once these MMAs complete
+      __syncwarp();
+      ++au;
+    }
+  } else {
+    // ================================ decode + epilogue ================================
+    const int et = threadIdx.x - 64;  // 0..255
+    const int q = warp & 3, h = (warp - 2) >> 2;
+    uint32_t au = 0, tile = 0;
+    for (int64_t u = blockIdx.x; u < total; u += gridDim.x) {
+      const int64_t rb = locate(u);
+      const SpDesc& d = b.d[p];
+      if (!sp_unit_dense(d, rb)) continue;
+      const int V = d.V;
+      const int KB = (int)ceil_div64(d.K, 64);
+      const int64_t i0 = rb * kSpRows;
+      const int64_t w0 = i0 / V;
+      const int64_t w1 = (i0 + kSpRows) / V < d.W ? (i0 + kSpRows) / V : d.W;
+      const int nwin = (int)(w1 - w0);
+      // ---- wait until the previous unit's MMAs released the A tile, then zero it
+      tc::mbar_wait(smem_u32(&aempty_bar), (au & 1) ^ 1);
+      for (int x = et; x < KB * kATile / 16; x += kSpEpi)
+        asm volatile("st.shared.v4.u32 [%0], {%1,%1,%1,%1};" ::"r"(s_adec + x * 16), "r"(0) : "memory");
+      if (et <= nwin) wptr[et] = __ldg(d.row_ptr + w0 + et);
+      if (et < kSpRows) unsorted[et] = 0;
+      tc::named_bar(1, kSpEpi);
+      // ---- decode: one flat pass over the unit's vectors [P0, P1)
+      const int64_t P0 = wptr[0], P1 = wptr[nwin];
+      const int64_t off = (int64_t)((reinterpret_cast<uintptr_t>(d.col_idx) >> 2) & 3);
+      const int64_t Pa = ((P0 + off) & ~(int64_t)3) - off;
+      for (int64_t base = Pa + 4 * et; base < P1; base += 4 * kSpEpi) {
+        int c4[4];
+        if (base >= P0 && base + 3 < P1) {
+          const int4 t = __ldg(reinterpret_cast<const int4*>(d.col_idx + base));
+          c4[0] = t.x; c4[1] = t.y; c4[2] = t.z; c4[3] = t.w;
+        } else {
+#pragma unroll
+          for (int j = 0; j < 4; ++j) c4[j] = (base + j >= P0 && base + j < P1) ? __ldg(d.col_idx + base + j) : -1;
+        }
+        const int64_t pf = base < P0 ? P0 : base;
+        int lo = 0, hi = nwin - 1;
+        while (lo < hi) {
+          const int mid = (lo + hi + 1) >> 1;
+          if (wptr[mid] <= pf) lo = mid; else hi = mid - 1;
+        }
+        int wl = lo;
+        int prev = (pf > wptr[wl] && pf < P1) ? __ldg(d.col_idx + pf - 1) : -1;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const int64_t pp = base + j;
+          if (pp < P0 || pp >= P1) continue;
+          while (wptr[wl + 1] <= pp) { ++wl; prev = -1; }
+          const int c = c4[j];
+          if (c <= prev) atomicOr(&unsorted[wl], 1);
+          prev = c;
+          const uint16_t* src = d.vals + pp * V;
+          uint16_t hv[8];
+          if (V == 8) {
+            const uint4 t = __ldg(reinterpret_cast<const uint4*>(src));
+            hv[0] = t.x & 0xFFFF; hv[1] = t.x >> 16; hv[2] = t.y & 0xFFFF; hv[3] = t.y >> 16;
+            hv[4] = t.z & 0xFFFF; hv[5] = t.z >> 16; hv[6] = t.w & 0xFFFF; hv[7] = t.w >> 16;
+          } else if (V == 4) {
+            const uint2 t = __ldg(reinterpret_cast<const uint2*>(src));
+            hv[0] = t.x & 0xFFFF; hv[1] = t.x >> 16; hv[2] = t.y & 0xFFFF; hv[3] = t.y >> 16;
+          } else {
+            const uint32_t t = __ldg(reinterpret_cast<const unsigned int*>(src));
+            hv[0] = t & 0xFFFF; hv[1] = t >> 16;
+          }
+#pragma unroll
+          for (int r = 0; r < 8; ++r)
+            if (r < V)
+              asm volatile("st.shared.u16 [%0], %1;" ::"r"(s_adec + adec_off(wl * V + r, c)), "h"(hv[r]) : "memory");
+        }
+      }
+      // generic-proxy stores -> visible to the tensor core (async proxy), then hand over
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      tc::named_bar(1, kSpEpi);
+      if (et == 0) tc::mbar_arrive(smem_u32(&afull_bar));
+      ++au;
+      // ---- epilogue per 128-column panel: TMEM -> fp16 (RN) -> C rows (every destination)
+      for (int64_t n0 = 0; n0 < d.N; n0 += 128) {
+        const uint32_t acc = tile & 1;
+        tc::mbar_wait(smem_u32(&tfull_bar[acc]), (tile >> 1) & 1);
+        tc::fence_after();
+        uint32_t v[16];
+        asm volatile(
+            "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+            : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+              "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]),
+              "=r"(v[15])
+            : "r"(tmem + ((uint32_t)(32 * q) << 16) + acc * kSpRows + 16 * h));
+        tc::ld_wait();
+        tc::fence_before();
+        __syncwarp();
+        if (lane == 0) tc::mbar_arrive(smem_u32(&tempty_bar[acc]));
+        const int64_t n = n0 + 32 * q + lane;
+        if (n < d.N) {
+#pragma unroll
+          for (int x = 0; x < 16; ++x) {
+            const int r = 16 * h + x;
+            const int64_t i = i0 + r;
+            if (i >= d.M || unsorted[r / V]) continue;
+            const uint16_t hv = f_to_h(__uint_as_float(v[x]));
+            for (int dd = 0; dd < d.nC; ++dd) d.C[dd][i * d.ldc + n] = hv;
+          }
+        }
+        ++tile;
+      }
+    }
+  }
+
+  tc::fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc::fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 64;" ::"r"(tmem));
+  }
+}
+
+// ------------------------------------------------------------------------------ host side
+
+static PFN_cuTensorMapEncodeTiled_v12000 tmap_encoder() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = [] {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+      p = nullptr;
+    return reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+  }();
+  return fn;
+}
+
+// K-major fp16 [rows x K] operand, box {64, box_rows}, 128-byte swizzle, OOB -> zero
+static bool make_kmajor_map(CUtensorMap* m, const void* base, int64_t rows, int64_t K, int box_rows) {
+  auto enc = tmap_encoder();
+  if (enc == nullptr) return false;
+  cuuint64_t gdim[2] = {(cuuint64_t)K, (cuuint64_t)rows};
+  cuuint64_t gstride[1] = {(cuuint64_t)K * 2};
+  cuuint32_t box[2] = {64, (cuuint32_t)box_rows};
+  cuuint32_t estr[2] = {1, 1};
+  return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, const_cast<void*>(base), gdim, gstride, box, estr,
+             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+// MN-major fp16 B [K x N] (N contiguous), box {64 n, 64 k}, 128-byte swizzle, OOB -> zero
+static bool make_mnmajor_map(CUtensorMap* m, const void* base, int64_t K, int64_t N) {
+  auto enc = tmap_encoder();
+  if (enc == nullptr) return false;
+  cuuint64_t gdim[2] = {(cuuint64_t)N, (cuuint64_t)K};
+  cuuint64_t gstride[1] = {(cuuint64_t)N * 2};
+  cuuint32_t box[2] = {64, 64};
+  cuuint32_t estr[2] = {1, 1};
+  return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, const_cast<void*>(base), gdim, gstride, box, estr,
+             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+static cudaError_t launch_sp(const SpBatch& b, int num_sms, cudaStream_t s) {
+  static std::once_flag once[64];
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev >= 0 && dev < 64)
+    std::call_once(once[dev], [] {
+      cudaFuncSetAttribute(spmm_dense_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kSpSmem);
+    });
+  const int64_t units = b.first_unit[b.count];
+  const int grid = (int)std::min<int64_t>(num_sms, units);
+  if (grid > 0) spmm_dense_kernel<<<grid, kSpThreads, kSpSmem, s>>>(b);
+  return cudaGetLastError();
+}
+
+static cudaError_t launch_sd(const SdBatch& b, int num_sms, cudaStream_t s) {
+  static std::once_flag once[64];
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev >= 0 && dev < 64)
+    std::call_once(once[dev], [] {
+      cudaFuncSetAttribute(sddmm_dense_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kSdSmem);
+    });
+  const int64_t units = b.first_unit[b.count];
+  const int grid = (int)std::min<int64_t>(num_sms, units);
+  if (grid > 0) sddmm_dense_kernel<<<grid, kSdThreads, kSdSmem, s>>>(b);
+  return cudaGetLastError();
+}
+
+}  // namespace dt
+
+// Problems the dense SDDMM path can take at all (the per-row-block choice is made on the
+// device): V >= 2, 0 < K <= 256 with K % 8 == 0 (A tiles resident, 16-byte TMA row stride),
+// 16-byte aligned A and Bt.
+bool sddmm_dense_eligible(int64_t M, int64_t N, int64_t K, int V, const void* A, const void* Bt) {
+  return M > 0 && N > 0 && K > 0 && K <= 64 * dt::kSdKbMax && V >= 2 && K % 8 == 0 &&
+         ((reinterpret_cast<uintptr_t>(A) & 15) == 0) && ((reinterpret_cast<uintptr_t>(Bt) & 15) == 0) &&
+         N < (int64_t(1) << 31) && M < (int64_t(1) << 31);
+}
+
+// Launches the dense-tile SDDMM over the eligible problems (units of row blocks the cost
+// model leaves to the gather kernel are skipped on the device).
+cudaError_t launch_sddmm_dense(int64_t count, const int64_t* M, const int64_t* N, const int64_t* K,
+                               const int* V, const int32_t* const* row_ptr, const int32_t* const* col_idx,
+                               const void* const* A, const void* const* Bt, void* const* out, int num_sms,
+                               cudaStream_t s) {
+  using namespace dt;
+  SdBatch batch;
+  batch.count = 0;
+  batch.first_unit[0] = 0;
+  auto flush = [&]() -> cudaError_t {
+    if (batch.count == 0) return cudaSuccess;
+    const cudaError_t e = launch_sd(batch, num_sms, s);
+    batch.count = 0;
+    batch.first_unit[0] = 0;
+    return e;
+  };
+  for (int64_t i = 0; i < count; ++i) {
+    if (!sddmm_dense_eligible(M[i], N[i], K[i], V[i], A[i], Bt[i])) continue;
+    SdDesc& d = batch.d[batch.count];
+    if (!make_kmajor_map(&d.tmA, A[i], M[i], K[i], kSdRows) ||
+        !make_kmajor_map(&d.tmBt, Bt[i], N[i], K[i], 128))
+      return cudaErrorInvalidValue;
+    d.M = M[i];
+    d.N = N[i];
+    d.K = K[i];
+    d.V = V[i];
+    d.W = ceil_div64(M[i], V[i]);
+    d.n_cr = ceil_div64(ceil_div64(N[i], 128), kCtPerUnit);
+    d.n_rb = ceil_div64(M[i], kSdRows);
+    d.row_ptr = row_ptr[i];
+    d.col_idx = col_idx[i];
+    d.out = static_cast<uint16_t*>(out[i]);
+    d.nnz_total = 0;
+    d.out_vec = (reinterpret_cast<uintptr_t>(out[i]) & (uintptr_t)(2 * V[i] - 1)) == 0 ? 1 : 0;
+    batch.first_unit[batch.count + 1] = batch.first_unit[batch.count] + d.n_rb * d.n_cr;
+    ++batch.count;
+    if (batch.count == kMaxProb) {
+      const cudaError_t e = flush();
+      if (e != cudaSuccess) return e;
+    }
+  }
+  return flush();
+}
+
+// Problems the dense SpMM path can take at all (the per-row-block choice is made on the
+// device): V >= 2, 0 < K <= 2048 (decoded A tile resident), N % 8 == 0 and 16-byte aligned B
+// (TMA), vals aligned to 2V bytes (one load per vector).
+bool spmm_dense_eligible(int64_t M, int64_t K, int64_t N, int V, const void* vals, const void* B) {
+  return M > 0 && N > 0 && K > 0 && K <= 64 * dt::kSpKbMax && V >= 2 && N % 8 == 0 &&
+         ((reinterpret_cast<uintptr_t>(B) & 15) == 0) &&
+         ((reinterpret_cast<uintptr_t>(vals) & (uintptr_t)(2 * V - 1)) == 0) && N < (int64_t(1) << 31) &&
+         M < (int64_t(1) << 31);
+}
+
+// dense-tile SpMM over the eligible problems; C_dst[i] holds nC[i] destinations (ldc[i])
+cudaError_t launch_spmm_dense(int64_t count, const int64_t* M, const int64_t* K, const int64_t* N,
+                              const int* V, const int32_t* const* row_ptr, const int32_t* const* col_idx,
+                              const void* const* vals, const void* const* B, void* const* const* C_dst,
+                              const int* nC, const int64_t* ldc, int num_sms, cudaStream_t s) {
+  using namespace dt;
+  SpBatch batch;
+  batch.count = 0;
+  batch.first_unit[0] = 0;
+  auto flush = [&]() -> cudaError_t {
+    if (batch.count == 0) return cudaSuccess;
+    const cudaError_t e = launch_sp(batch, num_sms, s);
+    batch.count = 0;
+    batch.first_unit[0] = 0;
+    return e;
+  };
+  for (int64_t i = 0; i < count; ++i) {
+    if (!spmm_dense_eligible(M[i], K[i], N[i], V[i], vals[i], B[i]) || nC[i] < 1 || nC[i] > kMaxDst) continue;
+    SpDesc& d = batch.d[batch.count];
+    if (!make_mnmajor_map(&d.tmB, B[i], K[i], N[i])) return cudaErrorInvalidValue;
+    d.M = M[i];
+    d.K = K[i];
+    d.N = N[i];
+    d.V = V[i];
+    d.W = ceil_div64(M[i], V[i]);
+    d.n_rb = ceil_div64(M[i], kSpRows);
+    d.row_ptr = row_ptr[i];
+    d.col_idx = col_idx[i];
+    d.vals = static_cast<const uint16_t*>(vals[i]);
+    for (int k = 0; k < kMaxDst; ++k) d.C[k] = k < nC[i] ? static_cast<uint16_t*>(C_dst[i][k]) : nullptr;
+    d.nC = nC[i];
+    d.ldc = ldc[i];
+    batch.first_unit[batch.count + 1] = batch.first_unit[batch.count] + d.n_rb;
+    ++batch.count;
+    if (batch.count == kMaxProb) {
+      const cudaError_t e = flush();
+      if (e != cudaSuccess) return e;
+    }
+  }
+  return flush();
+}
+
+}  // namespace vs
+#endif  // VS_DENSE_CF > 0

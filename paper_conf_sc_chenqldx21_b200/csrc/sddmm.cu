@@ -21,6 +21,7 @@
 #include <vector>
 
 #include "common.cuh"
+#include "dense_select.cuh"
 
 namespace vs {
 
@@ -216,6 +217,20 @@ __device__ __forceinline__ void sddmm_window_any(int64_t M, int64_t K,
   }
 }
 
+// Row blocks the dense-tile kernel takes (dense_select.cuh) are skipped here: the dense kernel
+// computes every stored vector of them, in any col_idx order.  Returns the q to use for the
+// item, or 0 to skip it.
+__device__ __forceinline__ int64_t sddmm_gather_q(bool dense_ok, int64_t N, int V, int64_t W,
+                                                  const int32_t* __restrict__ row_ptr,
+                                                  const int32_t* __restrict__ col_idx, int64_t w,
+                                                  int64_t j0, int64_t q) {
+  (void)col_idx;
+  (void)j0;
+  if (!dense_ok) return q;
+  const int64_t rb = (w * V) / kDenseRows;
+  return rb_is_dense(row_ptr, W, V, rb, ceil_div64(N, 128) * 128) ? 0 : q;
+}
+
 // Work items of one problem: W windows x q warps per window (warp j of window w takes the
 // window's 16-vector chunks j, j + q, ...); q = the number of warps per window that gives
 // every warp of the launch about the same number of chunks.
@@ -229,7 +244,7 @@ __global__ void __launch_bounds__(kSddmmWarps * 32, VS_SDDMM_MINB)
     sddmm_kernel(int64_t M, int64_t K, int64_t W, const int32_t* __restrict__ row_ptr,
                  const int32_t* __restrict__ col_idx, const uint16_t* __restrict__ A,
                  const uint16_t* __restrict__ Bt, uint16_t* __restrict__ out, bool out4,
-                 bool pair) {
+                 bool pair, int64_t N, bool dense_ok) {
   const int64_t nnz = row_ptr[W];
   const int64_t n_warps = (int64_t)gridDim.x * kSddmmWarps;
   const int64_t gw = (int64_t)blockIdx.x * kSddmmWarps + (threadIdx.x >> 5);
@@ -238,8 +253,10 @@ __global__ void __launch_bounds__(kSddmmWarps * 32, VS_SDDMM_MINB)
   const int64_t items = W * q;
   for (int64_t it = gw; it < items; it += n_warps) {
     const int64_t w = it / q;
-    sddmm_window_any<V, VEC, KC, ARES>(M, K, row_ptr, col_idx, A, Bt, out, out4, w, it - w * q, q,
-                                       pair);
+    const int64_t qq = sddmm_gather_q(dense_ok, N, V, W, row_ptr, col_idx, w, it - w * q, q);
+    if (qq == 0) continue;
+    sddmm_window_any<V, VEC, KC, ARES>(M, K, row_ptr, col_idx, A, Bt, out, out4, w,
+                                       qq == q ? it - w * q : 0, qq, pair);
   }
 }
 
@@ -249,7 +266,8 @@ __global__ void __launch_bounds__(kSddmmWarps * 32, VS_SDDMM_MINB)
 // persistent warps in problem order, so at any time the warps work on one or two problems
 // (L2 locality).
 struct SddmmDesc {
-  int64_t M, K, W;
+  int64_t M, K, W, N;
+  int64_t dense_ok;  // sddmm_dense_eligible: row blocks may be taken by the dense-tile kernel
   const int32_t* row_ptr;
   const int32_t* col_idx;
   const uint16_t* A;
@@ -318,8 +336,10 @@ __global__ void __launch_bounds__(kSddmmWarps * 32, VS_SDDMM_MINB)
     const int64_t q = qs[p];
     const int64_t loc = it - pre[p];
     const int64_t w = loc / q;
+    const int64_t qq = sddmm_gather_q(d.dense_ok != 0, d.N, V, d.W, d.row_ptr, d.col_idx, w, loc - w * q, q);
+    if (qq == 0) continue;
     sddmm_window_any<V, VEC, KC, ARES>(d.M, d.K, d.row_ptr, d.col_idx, d.A, d.Bt, d.out,
-                                       d.out4 != 0, w, loc - w * q, q, b.pair != 0);
+                                       d.out4 != 0, w, qq == q ? loc - w * q : 0, qq, b.pair != 0);
   }
 }
 
@@ -376,28 +396,50 @@ static int sddmm_batched_ctas_per_sm() {
 template <int V, bool VEC, int KC, bool ARES>
 static void launch_sddmm_one(int64_t M, int64_t K, const int32_t* row_ptr, const int32_t* col_idx,
                              const uint16_t* A, const uint16_t* Bt, uint16_t* out, int num_sms,
-                             cudaStream_t s) {
+                             cudaStream_t s, int64_t N, bool dense_ok) {
   const int64_t W = ceil_div64(M, V);
   const bool out4 = (reinterpret_cast<uintptr_t>(out) & 3) == 0;
   dim3 grid((unsigned)(num_sms * sddmm_ctas_per_sm<V, VEC, KC, ARES>()));
   sddmm_kernel<V, VEC, KC, ARES><<<grid, kSddmmWarps * 32, 0, s>>>(M, K, W, row_ptr, col_idx, A,
-                                                                   Bt, out, out4, sddmm_pair_on());
+                                                                   Bt, out, out4, sddmm_pair_on(),
+                                                                   N, dense_ok);
 }
+
+#if VS_DENSE_CF > 0
+bool sddmm_dense_eligible(int64_t M, int64_t N, int64_t K, int V, const void* A, const void* Bt);
+cudaError_t launch_sddmm_dense(int64_t count, const int64_t* M, const int64_t* N, const int64_t* K,
+                               const int* V, const int32_t* const* row_ptr, const int32_t* const* col_idx,
+                               const void* const* A, const void* const* Bt, void* const* out, int num_sms,
+                               cudaStream_t s);
+#else  // shipped library: no dense-tile path (dense_select.cuh)
+static bool sddmm_dense_eligible(int64_t, int64_t, int64_t, int, const void*, const void*) { return false; }
+static cudaError_t launch_sddmm_dense(int64_t, const int64_t*, const int64_t*, const int64_t*, const int*,
+                                      const int32_t* const*, const int32_t* const*, const void* const*,
+                                      const void* const*, void* const*, int, cudaStream_t) {
+  return cudaSuccess;
+}
+#endif
 
 template <int V>
 static cudaError_t launch_sddmm_v(int64_t M, int64_t N, int64_t K, const int32_t* row_ptr,
                                   const int32_t* col_idx, const uint16_t* A, const uint16_t* Bt,
                                   uint16_t* out, bool vec, int num_sms, cudaStream_t s) {
-  (void)N;
+  const int V_ = V;
+  const bool dok = sddmm_dense_eligible(M, N, K, V, A, Bt);
   switch ((vec ? 8 : 0) + sddmm_variant(K, vec)) {
-    case 8 + 2: launch_sddmm_one<V, true, 1, false>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s); break;
-    case 8 + 3: launch_sddmm_one<V, true, 1, true>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s); break;
-    case 8 + 4: launch_sddmm_one<V, true, 2, false>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s); break;
-    case 8 + 5: launch_sddmm_one<V, true, 2, true>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s); break;
-    case 3: launch_sddmm_one<V, false, 1, true>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s); break;
-    default: launch_sddmm_one<V, false, 1, false>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s); break;
+    case 8 + 2: launch_sddmm_one<V, true, 1, false>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok); break;
+    case 8 + 3: launch_sddmm_one<V, true, 1, true>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok); break;
+    case 8 + 4: launch_sddmm_one<V, true, 2, false>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok); break;
+    case 8 + 5: launch_sddmm_one<V, true, 2, true>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok); break;
+    case 3: launch_sddmm_one<V, false, 1, true>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok); break;
+    default: launch_sddmm_one<V, false, 1, false>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok); break;
   }
-  return cudaGetLastError();
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess || !dok) return e;
+  const void* a = A;
+  const void* bt = Bt;
+  void* o = out;
+  return launch_sddmm_dense(1, &M, &N, &K, &V_, &row_ptr, &col_idx, &a, &bt, &o, num_sms, s);
 }
 
 template <int V, bool VEC, int KC, bool ARES>
@@ -451,8 +493,9 @@ static cudaError_t launch_sddmm_tc_batched(int64_t, const int64_t*, const int64_
 }
 #endif
 
-static cudaError_t launch_sddmm_mma_batched(int64_t count, const int64_t* M, const int64_t* K,
-                                            const int* V, const int32_t* const* row_ptr,
+static cudaError_t launch_sddmm_mma_batched(int64_t count, const int64_t* M, const int64_t* N,
+                                            const int64_t* K, const int* V,
+                                            const int32_t* const* row_ptr,
                                             const int32_t* const* col_idx, const void* const* A,
                                             const void* const* Bt, void* const* out, int num_sms,
                                             cudaStream_t s);
@@ -462,8 +505,12 @@ cudaError_t launch_sddmm_batched(int64_t count, const int64_t* M, const int64_t*
                                  const int32_t* const* col_idx, const void* const* A,
                                  const void* const* Bt, void* const* out, int num_sms,
                                  cudaStream_t s) {
-  if (!sddmm_tc_on())
-    return launch_sddmm_mma_batched(count, M, K, V, row_ptr, col_idx, A, Bt, out, num_sms, s);
+  if (!sddmm_tc_on()) {
+    // gather kernels (skipping the dense row blocks), then the dense-tile kernel (taking them)
+    const cudaError_t e = launch_sddmm_mma_batched(count, M, N, K, V, row_ptr, col_idx, A, Bt, out, num_sms, s);
+    if (e != cudaSuccess || VS_DENSE_CF == 0) return e;
+    return launch_sddmm_dense(count, M, N, K, V, row_ptr, col_idx, A, Bt, out, num_sms, s);
+  }
   std::vector<int64_t> sel[2];
   for (int64_t i = 0; i < count; ++i) sel[sddmm_tc_eligible(K[i], A[i], Bt[i], out[i]) ? 1 : 0].push_back(i);
   for (int path = 0; path < 2; ++path) {
@@ -480,15 +527,16 @@ cudaError_t launch_sddmm_batched(int64_t count, const int64_t* M, const int64_t*
     const cudaError_t e =
         path ? launch_sddmm_tc_batched((int64_t)m.size(), m.data(), n.data(), k.data(), v.data(),
                                        rp.data(), ci.data(), a.data(), bt.data(), o.data(), num_sms, s)
-             : launch_sddmm_mma_batched((int64_t)m.size(), m.data(), k.data(), v.data(), rp.data(),
+             : launch_sddmm_mma_batched((int64_t)m.size(), m.data(), n.data(), k.data(), v.data(), rp.data(),
                                         ci.data(), a.data(), bt.data(), o.data(), num_sms, s);
     if (e != cudaSuccess) return e;
   }
   return cudaSuccess;
 }
 
-static cudaError_t launch_sddmm_mma_batched(int64_t count, const int64_t* M, const int64_t* K,
-                                            const int* V, const int32_t* const* row_ptr,
+static cudaError_t launch_sddmm_mma_batched(int64_t count, const int64_t* M, const int64_t* N,
+                                            const int64_t* K, const int* V,
+                                            const int32_t* const* row_ptr,
                                             const int32_t* const* col_idx, const void* const* A,
                                             const void* const* Bt, void* const* out, int num_sms,
                                             cudaStream_t s) {
@@ -511,7 +559,8 @@ static cudaError_t launch_sddmm_mma_batched(int64_t count, const int64_t* M, con
     while (i < order.size() && order[i].first == key && batch.count < kSddmmMaxBatch) {
       const int64_t p = order[i].second;
       SddmmDesc& d = batch.d[batch.count++];
-      d = {M[p], K[p], ceil_div64(M[p], V[p]), row_ptr[p], col_idx[p],
+      d = {M[p], K[p], ceil_div64(M[p], V[p]), N[p],
+           sddmm_dense_eligible(M[p], N[p], K[p], V[p], A[p], Bt[p]) ? 1 : 0, row_ptr[p], col_idx[p],
            static_cast<const uint16_t*>(A[p]), static_cast<const uint16_t*>(Bt[p]),
            static_cast<uint16_t*>(out[p]), (reinterpret_cast<uintptr_t>(out[p]) & 3) == 0 ? 1 : 0};
       ++i;

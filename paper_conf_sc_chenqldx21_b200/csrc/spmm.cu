@@ -24,6 +24,7 @@
 #include <vector>
 
 #include "common.cuh"
+#include "dense_select.cuh"
 
 namespace vs {
 
@@ -77,6 +78,17 @@ __device__ __forceinline__ void pdl_launch_dependents() {
 }
 __device__ __forceinline__ void pdl_wait_prior() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 
+// Windows of the 128-row blocks the dense-tile kernel takes (dense_select.cuh; dkp = the
+// problem's K padded to 64, 0 = not dense-eligible) are skipped, except windows whose col_idx
+// is not strictly ascending: the dense kernel leaves those rows to this kernel.  Warp-uniform.
+__device__ __forceinline__ bool spmm_skip_window(int64_t dkp, int V, int64_t W, int64_t w,
+                                                 const int32_t* __restrict__ row_ptr,
+                                                 const int32_t* __restrict__ col_idx, int pb, int pe) {
+  if (dkp == 0 || w >= W) return false;
+  if (!rb_is_dense(row_ptr, W, V, (w * V) / kDenseRows, dkp)) return false;
+  return window_sorted(col_idx, pb, pe);
+}
+
 // SPLIT warps cooperate on one (window, panel) unit: warp part q takes the 16-vector groups
 // q, q + SPLIT, ... and the partial accumulators are summed through shared memory by a
 // fixed pairwise tree (deterministic).  A CTA has max(4, SPLIT) warps = max(1, 4/SPLIT) units.
@@ -91,7 +103,8 @@ __device__ __forceinline__ void spmm_body(int64_t M, int64_t N, int64_t W, int64
                                           int64_t bid, const int32_t* __restrict__ row_ptr,
                                           const int32_t* __restrict__ col_idx,
                                           const uint16_t* __restrict__ vals,
-                                          const uint16_t* __restrict__ B, const CDst<ND>& cd) {
+                                          const uint16_t* __restrict__ B, const CDst<ND>& cd,
+                                          int64_t dkp) {
   constexpr int UPC = SpmmCta<SPLIT>::kUnits;  // units per CTA
   constexpr int NACC = NC * 16;                // accumulator floats per thread
   constexpr int HALF = SPLIT > 1 ? SPLIT / 2 : 1;
@@ -103,10 +116,12 @@ __device__ __forceinline__ void spmm_body(int64_t M, int64_t N, int64_t W, int64
   // panel-major CTA order: consecutive CTAs share a B panel (L1/L2 locality)
   const int64_t pn = bid / n_wgroups;
   const int64_t w = (bid - pn * n_wgroups) * UPC + wid / SPLIT;
-  const bool active = w < W;
   const int64_t ncol0 = pn * (64 * NC) + 8 * g;  // this thread's first column
-  const int p_begin = active ? row_ptr[w] : 0;
-  const int p_end = active ? row_ptr[w + 1] : 0;
+  const int p_begin = w < W ? row_ptr[w] : 0;
+  int p_end = w < W ? row_ptr[w + 1] : 0;
+  const bool skip = spmm_skip_window(dkp, V, W, w, row_ptr, col_idx, p_begin, p_end);
+  const bool active = w < W && !skip;
+  if (!active) p_end = p_begin;
 
   float acc[NC][4][4];
 #pragma unroll
@@ -298,9 +313,9 @@ __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32)
     spmm_kernel(int64_t M, int64_t N, int64_t W, int64_t n_wgroups,
                 const int32_t* __restrict__ row_ptr, const int32_t* __restrict__ col_idx,
                 const uint16_t* __restrict__ vals, const uint16_t* __restrict__ B,
-                uint16_t* __restrict__ C) {
+                uint16_t* __restrict__ C, int64_t dkp) {
   const CDst<1> cd = {{C}, 1, N};
-  spmm_body<V, NC, VEC, SPLIT, UNROLL, 1>(M, N, W, n_wgroups, blockIdx.x, row_ptr, col_idx, vals, B, cd);
+  spmm_body<V, NC, VEC, SPLIT, UNROLL, 1>(M, N, W, n_wgroups, blockIdx.x, row_ptr, col_idx, vals, B, cd, dkp);
 }
 
 // vs_spmm_scatter, register path (unaligned operands or destinations, V = 1)
@@ -309,9 +324,9 @@ __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32)
     spmm_scatter_kernel(int64_t M, int64_t N, int64_t W, int64_t n_wgroups,
                         const int32_t* __restrict__ row_ptr, const int32_t* __restrict__ col_idx,
                         const uint16_t* __restrict__ vals, const uint16_t* __restrict__ B,
-                        const __grid_constant__ CDst<kMaxScatter> cd) {
+                        const __grid_constant__ CDst<kMaxScatter> cd, int64_t dkp) {
   spmm_body<V, NC, VEC, SPLIT, 1, kMaxScatter>(M, N, W, n_wgroups, blockIdx.x, row_ptr, col_idx,
-                                               vals, B, cd);
+                                               vals, B, cd, dkp);
 }
 
 // Batched launch: one grid over the units of up to kSpmmMaxBatch problems that share a
@@ -319,6 +334,7 @@ __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32)
 // CTA finds its problem by binary search of the per-problem first-block table.
 struct SpmmDesc {
   int64_t M, N, W, n_wgroups;
+  int64_t dkp;  // dense-tile eligibility: K padded to 64 (0 = not eligible)
   const int32_t* row_ptr;
   const int32_t* col_idx;
   const uint16_t* vals;
@@ -347,7 +363,7 @@ __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32)
     const SpmmDesc& d = b.d[p];
     const CDst<1> cd = {{d.C}, 1, d.N};
     spmm_body<V, NC, VEC, SPLIT, UNROLL, 1>(d.M, d.N, d.W, d.n_wgroups, bid - b.first_block[p],
-                                            d.row_ptr, d.col_idx, d.vals, d.B, cd);
+                                            d.row_ptr, d.col_idx, d.vals, d.B, cd, d.dkp);
   }
   pdl_wait_prior();
 }
@@ -396,7 +412,7 @@ __device__ __forceinline__ void spmm_cp_body(int64_t M, int64_t N, int64_t W, in
                                              const int32_t* __restrict__ col_idx,
                                              const uint16_t* __restrict__ vals,
                                              const uint16_t* __restrict__ B,
-                                             const CDst<ND>& cd, unsigned char* smem) {
+                                             const CDst<ND>& cd, unsigned char* smem, int64_t dkp) {
   using R = CpRing<V, NC, D>;
   constexpr int UPC = SpmmCta<SPLIT>::kUnits;
   constexpr int HALF = SPLIT > 1 ? SPLIT / 2 : 1;
@@ -407,10 +423,12 @@ __device__ __forceinline__ void spmm_cp_body(int64_t M, int64_t N, int64_t W, in
   const int part = wid % SPLIT;
   const int64_t pn = bid / n_wgroups;
   const int64_t w = (bid - pn * n_wgroups) * UPC + wid / SPLIT;
-  const bool active = w < W;
   const int64_t n0 = pn * PW;  // first column of the panel
-  const int p_begin = active ? row_ptr[w] : 0;
-  const int p_end = active ? row_ptr[w + 1] : 0;
+  const int p_begin = w < W ? row_ptr[w] : 0;
+  int p_end = w < W ? row_ptr[w + 1] : 0;
+  const bool skip = spmm_skip_window(dkp, V, W, w, row_ptr, col_idx, p_begin, p_end);
+  const bool active = w < W && !skip;
+  if (!active) p_end = p_begin;
   const uint32_t s_rows = smem_u32(smem + wid * R::kWarpBytes);
   const uint32_t s_vals = s_rows + D * R::kRowBytes;
   const uint32_t s_cols = s_vals + D * R::kValBytes;
@@ -596,10 +614,10 @@ __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32, CpMinBlocks<SPLIT
     spmm_cp_kernel(int64_t M, int64_t N, int64_t W, int64_t n_wgroups,
                    const int32_t* __restrict__ row_ptr, const int32_t* __restrict__ col_idx,
                    const uint16_t* __restrict__ vals, const uint16_t* __restrict__ B,
-                   uint16_t* __restrict__ C) {
+                   uint16_t* __restrict__ C, int64_t dkp) {
   extern __shared__ __align__(128) unsigned char smem[];
   const CDst<1> cd = {{C}, 1, N};
-  spmm_cp_body<V, NC, SPLIT, D, 1>(M, N, W, n_wgroups, blockIdx.x, row_ptr, col_idx, vals, B, cd, smem);
+  spmm_cp_body<V, NC, SPLIT, D, 1>(M, N, W, n_wgroups, blockIdx.x, row_ptr, col_idx, vals, B, cd, smem, dkp);
 }
 
 // vs_spmm_scatter, cp.async path: the same body, every output tile stored into cd.n destinations
@@ -608,10 +626,10 @@ __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32, CpMinBlocks<SPLIT
     spmm_cp_scatter_kernel(int64_t M, int64_t N, int64_t W, int64_t n_wgroups,
                            const int32_t* __restrict__ row_ptr, const int32_t* __restrict__ col_idx,
                            const uint16_t* __restrict__ vals, const uint16_t* __restrict__ B,
-                           const __grid_constant__ CDst<kMaxScatter> cd) {
+                           const __grid_constant__ CDst<kMaxScatter> cd, int64_t dkp) {
   extern __shared__ __align__(128) unsigned char smem[];
   spmm_cp_body<V, NC, SPLIT, D, kMaxScatter>(M, N, W, n_wgroups, blockIdx.x, row_ptr, col_idx, vals, B,
-                                             cd, smem);
+                                             cd, smem, dkp);
 }
 
 template <int V, int NC, int SPLIT, int D>
@@ -626,7 +644,7 @@ __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32, CpMinBlocks<SPLIT
     const SpmmDesc& d = b.d[p];
     const CDst<1> cd = {{d.C}, 1, d.N};
     spmm_cp_body<V, NC, SPLIT, D, 1>(d.M, d.N, d.W, d.n_wgroups, bid - b.first_block[p], d.row_ptr,
-                                     d.col_idx, d.vals, d.B, cd, smem);
+                                     d.col_idx, d.vals, d.B, cd, smem, d.dkp);
   }
   pdl_wait_prior();
 }
@@ -701,10 +719,10 @@ static SpmmCfg spmm_config_al(int64_t K, int64_t N, int V, bool b_al16, bool c_a
 
 struct SpmmKernels {
   void (*single)(int64_t, int64_t, int64_t, int64_t, const int32_t*, const int32_t*,
-                 const uint16_t*, const uint16_t*, uint16_t*);
+                 const uint16_t*, const uint16_t*, uint16_t*, int64_t);
   void (*batched)(SpmmBatch);
   void (*scatter)(int64_t, int64_t, int64_t, int64_t, const int32_t*, const int32_t*,
-                  const uint16_t*, const uint16_t*, CDst<kMaxScatter>);
+                  const uint16_t*, const uint16_t*, CDst<kMaxScatter>, int64_t);
   int threads, units_per_cta, batched_ctas_per_sm;
   int smem;  // dynamic shared memory bytes (cp.async path), 0 otherwise
 };
@@ -822,6 +840,25 @@ static int64_t spmm_blocks(const SpmmKernels& k, const SpmmCfg& c, int64_t M, in
   return ceil_div64(N, 64 * c.NC) * nwg;
 }
 
+#if VS_DENSE_CF > 0
+bool spmm_dense_eligible(int64_t M, int64_t K, int64_t N, int V, const void* vals, const void* B);
+cudaError_t launch_spmm_dense(int64_t count, const int64_t* M, const int64_t* K, const int64_t* N,
+                              const int* V, const int32_t* const* row_ptr, const int32_t* const* col_idx,
+                              const void* const* vals, const void* const* B, void* const* const* C_dst,
+                              const int* nC, const int64_t* ldc, int num_sms, cudaStream_t s);
+#else  // shipped library: no dense-tile path (dense_select.cuh)
+static bool spmm_dense_eligible(int64_t, int64_t, int64_t, int, const void*, const void*) { return false; }
+static cudaError_t launch_spmm_dense(int64_t, const int64_t*, const int64_t*, const int64_t*, const int*,
+                                     const int32_t* const*, const int32_t* const*, const void* const*,
+                                     const void* const*, void* const* const*, const int*, const int64_t*, int,
+                                     cudaStream_t) {
+  return cudaSuccess;
+}
+#endif
+static int64_t spmm_dkp(int64_t M, int64_t K, int64_t N, int V, const void* vals, const void* B) {
+  return spmm_dense_eligible(M, K, N, V, vals, B) ? ceil_div64(K, 64) * 64 : 0;
+}
+
 cudaError_t launch_spmm(int64_t M, int64_t K, int64_t N, int V, const int32_t* row_ptr,
                         const int32_t* col_idx, const void* vals, const void* B, void* C,
                         int num_sms, cudaStream_t s) {
@@ -832,11 +869,17 @@ cudaError_t launch_spmm(int64_t M, int64_t K, int64_t N, int V, const int32_t* r
   const int64_t grid = spmm_blocks(k, c, M, N, V, &W, &nwg);
   if (grid > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
   if (grid == 0) return cudaSuccess;
+  const int64_t dkp = spmm_dkp(M, K, N, V, vals, B);
   k.single<<<(unsigned)grid, k.threads, k.smem, s>>>(M, N, W, nwg, row_ptr, col_idx,
                                                      static_cast<const uint16_t*>(vals),
                                                      static_cast<const uint16_t*>(B),
-                                                     static_cast<uint16_t*>(C));
-  return cudaGetLastError();
+                                                     static_cast<uint16_t*>(C), dkp);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess || dkp == 0) return e;
+  void* dst[1] = {C};
+  void* const* dsts = dst;
+  const int one = 1;
+  return launch_spmm_dense(1, &M, &K, &N, &V, &row_ptr, &col_idx, &vals, &B, &dsts, &one, &N, num_sms, s);
 }
 
 // vs_spmm_scatter: the launch of vs_spmm, every output tile stored into n_dst destinations
@@ -844,7 +887,7 @@ cudaError_t launch_spmm(int64_t M, int64_t K, int64_t N, int V, const int32_t* r
 // ldc * 2 bytes 16-byte aligned (and B aligned, N % 8 == 0), as for vs_spmm.
 cudaError_t launch_spmm_scatter(int64_t M, int64_t K, int64_t N, int V, const int32_t* row_ptr,
                                 const int32_t* col_idx, const void* vals, const void* B,
-                                void* const* C_dst, int n_dst, int64_t ldc, cudaStream_t s) {
+                                void* const* C_dst, int n_dst, int64_t ldc, int num_sms, cudaStream_t s) {
   if (n_dst < 1 || n_dst > kMaxScatter) return cudaErrorInvalidValue;
   bool c_al = (ldc % 8) == 0;
   CDst<kMaxScatter> cd = {};
@@ -860,10 +903,14 @@ cudaError_t launch_spmm_scatter(int64_t M, int64_t K, int64_t N, int V, const in
   const int64_t grid = spmm_blocks(k, c, M, N, V, &W, &nwg);
   if (grid > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
   if (grid == 0) return cudaSuccess;
+  const int64_t dkp = spmm_dkp(M, K, N, V, vals, B);
   k.scatter<<<(unsigned)grid, k.threads, k.smem, s>>>(M, N, W, nwg, row_ptr, col_idx,
                                                       static_cast<const uint16_t*>(vals),
-                                                      static_cast<const uint16_t*>(B), cd);
-  return cudaGetLastError();
+                                                      static_cast<const uint16_t*>(B), cd, dkp);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess || dkp == 0) return e;
+  return launch_spmm_dense(1, &M, &K, &N, &V, &row_ptr, &col_idx, &vals, &B, &C_dst, &n_dst, &ldc,
+                           num_sms, s);
 }
 
 // VS_SPMM_PDL (build-time, default 1): the launches of one batched call after the first use programmatic
@@ -900,8 +947,9 @@ cudaError_t launch_spmm_batched(int64_t count, const int64_t* M, const int64_t* 
       const int64_t nb = spmm_blocks(k, c, M[p], N[p], V[p], &W, &nwg);
       if (blocks + nb > 0x7fffffffLL) break;
       SpmmDesc& d = batch.d[batch.count];
-      d = {M[p], N[p], W, nwg, row_ptr[p], col_idx[p], static_cast<const uint16_t*>(vals[p]),
-           static_cast<const uint16_t*>(B[p]), static_cast<uint16_t*>(C[p])};
+      d = {M[p], N[p], W, nwg, spmm_dkp(M[p], K[p], N[p], V[p], vals[p], B[p]), row_ptr[p], col_idx[p],
+           static_cast<const uint16_t*>(vals[p]), static_cast<const uint16_t*>(B[p]),
+           static_cast<uint16_t*>(C[p])};
       batch.first_block[batch.count] = blocks;
       blocks += nb;
       ++batch.count;
@@ -934,7 +982,13 @@ cudaError_t launch_spmm_batched(int64_t count, const int64_t* M, const int64_t* 
     const cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
   }
-  return cudaSuccess;
+  // the dense-tile kernel takes the row blocks the gather launches above skipped
+  if (VS_DENSE_CF == 0) return cudaSuccess;
+  std::vector<void* const*> dsts(count);
+  std::vector<int> ones(count, 1);
+  for (int64_t i = 0; i < count; ++i) dsts[i] = &C[i];
+  return launch_spmm_dense(count, M, K, N, V, row_ptr, col_idx, vals, B, dsts.data(), ones.data(), N,
+                           num_sms, s);
 }
 
 }  // namespace vs

@@ -14,7 +14,7 @@ cudaError_t launch_spmm(int64_t M, int64_t K, int64_t N, int V, const int32_t* r
                         int num_sms, cudaStream_t s);
 cudaError_t launch_spmm_scatter(int64_t M, int64_t K, int64_t N, int V, const int32_t* row_ptr,
                                 const int32_t* col_idx, const void* vals, const void* B,
-                                void* const* C_dst, int n_dst, int64_t ldc, cudaStream_t s);
+                                void* const* C_dst, int n_dst, int64_t ldc, int num_sms, cudaStream_t s);
 cudaError_t launch_sddmm(int64_t M, int64_t N, int64_t K, int V, const int32_t* row_ptr,
                          const int32_t* col_idx, const void* A, const void* Bt, void* out,
                          int num_sms, cudaStream_t s);
@@ -209,7 +209,8 @@ vs_status_t vs_spmm_scatter(int64_t M, int64_t K, int64_t N, int V, const int32_
         return VS_ERROR_CUDA;
     return VS_SUCCESS;
   }
-  return from_cuda(vs::launch_spmm_scatter(M, K, N, V, row_ptr, col_idx, vals, B, C_dst, n_dst, ldc, s));
+  return from_cuda(vs::launch_spmm_scatter(M, K, N, V, row_ptr, col_idx, vals, B, C_dst, n_dst, ldc,
+                                           info.num_sms, s));
 }
 
 vs_status_t vs_sddmm(int64_t M, int64_t N, int64_t K, int V, const int32_t* row_ptr,

@@ -39,9 +39,11 @@ def panel_bounds(N: int, world: int, align: int = 64) -> list:
     return out
 
 
-def window_bounds(row_ptr: np.ndarray, world: int) -> list:
+def window_bounds(row_ptr: np.ndarray, world: int, align: int = 1) -> list:
     """Window boundaries [w_0 = 0, ..., w_P = W] with row_ptr[w_p] ~ p * nnz_v / P
-    (balanced to within one window's vectors)."""
+    (balanced to within `align` windows' vectors).  With align = 128 / V every shard starts on
+    a 128-row block boundary, so the per-row-block choice between the gather and the dense-tile
+    SDDMM kernels (dense_select.cuh) is the same in a shard as in the unsharded problem."""
     row_ptr = np.asarray(row_ptr, dtype=np.int64)
     W = row_ptr.size - 1
     nnz = int(row_ptr[-1])
@@ -49,6 +51,8 @@ def window_bounds(row_ptr: np.ndarray, world: int) -> list:
     for p in range(1, world):
         target = (nnz * p) // world
         w = int(np.searchsorted(row_ptr, target, side="left"))
+        if align > 1:
+            w = int(round(w / align)) * align
         out.append(min(max(w, out[-1]), W))
     out.append(W)
     return out

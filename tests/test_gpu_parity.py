@@ -366,7 +366,8 @@ def test_sharded_equals_unsharded_sddmm(vs, V):
     full = vs.sddmm(rp, ci, A, Bt, V)
     rph = host(rp)
     for P in (2, 3, 8):
-        wb = vsd.window_bounds(rph, P)
+        # shards start on 128-row blocks (the unit of the gather / dense-tile choice)
+        wb = vsd.window_bounds(rph, P, align=128 // V)
         segs = []
         for r in range(P):
             sh = vsd.sddmm_shard(rph, M, V, wb, r)
