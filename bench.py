@@ -684,8 +684,10 @@ def run_ours(args):
         "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "f16", "data": "synthetic",
         "config": {"workload": args.workload, "problems": nb,
-                   "shapes": "(M,K) in {(512,512),(2048,512),(512,2048),(2048,1024)} x V{2,4,8} "
-                             "x S{.5,.7,.9,.98} x N{64,128,256}" if args.workload == "dlmc_layer" else args.workload,
+                   "shapes": ("(M,K) in {(512,512),(2048,512),(512,2048),(2048,1024)} x V{2,4,8} "
+                              "x S{.5,.7,.9,.98} x N{64,128,256}") if args.workload == "dlmc_layer" else
+                             ("same shapes x S{.5,.7,.8,.9,.95,.98}" if args.workload == "dlmc_grid"
+                              else args.workload),
                    "step": "per problem: encode W -> SpMM Y=WX -> SDDMM dW=(G X^T) o pattern(W)",
                    "flops_per_step": flops_step, "l2": "flushed between timed steps (512 MiB write, untimed)",
                    "launch": "batched C ABI (vs_*_batched), step replayed as one CUDA graph; " + (
@@ -962,11 +964,28 @@ def library_baselines(args, torch, vs, bufs, stream, detail):
     summary = {}
     for (V, S), c in sorted(cells.items()):
         summary[f"V{V}_S{S:.2f}"] = {k: (round(geomean(v), 3) if geomean(v) else None) for k, v in c.items()}
+    # per-V crossover: the smallest sparsity from which every cell's geomean speedup >= 1
+    crossover = {}
+    for V in sorted({k[0] for k in cells}):
+        Ss = sorted(S for (v, S) in cells if v == V)
+        ent = {}
+        for op, key in (("spmm_vs_hgemm", "spmm_vs_h"), ("spmm_vs_best_cublas", "spmm_vs_best_cublas"),
+                        ("sddmm_vs_hgemm", "sddmm_vs_h")):
+            wins = [S for S in Ss if (geomean(cells[(V, S)][key]) or 0) >= 1.0]
+            # smallest S such that all S' >= S win
+            cross = None
+            for S in Ss:
+                if all(S2 in wins for S2 in Ss if S2 >= S):
+                    cross = S
+                    break
+            ent[op] = cross
+        crossover[f"V{V}"] = ent
     all_spmm = [x for c in cells.values() for x in c["spmm_vs_h"]]
     all_sddmm = [x for c in cells.values() for x in c["sddmm_vs_h"]]
     return {"speedup_vs_cublas_hgemm": {
         "geomean_spmm": geomean(all_spmm), "geomean_sddmm": geomean(all_sddmm),
         "per_cell_geomean": summary,
+        "crossover_sparsity": crossover,
         "protocol": f"{args.reps} launches per CUDA graph, L2 warm, per-launch mean; dense "
                     "counterpart = cublasHgemm M x K x N (both ops)"}}
 

@@ -49,6 +49,17 @@ RN50_MK = [(64, 64), (64, 256), (256, 64), (128, 256), (128, 512), (512, 128), (
 RN50_S = [0.7, 0.8, 0.9, 0.95]
 
 
+# the paper's full sparsity grid (Fig. 17/19 captions)
+DLMC_S_GRID = [0.5, 0.7, 0.8, 0.9, 0.95, 0.98]
+
+
+def dlmc_grid_workload():
+    """configs[1] x configs[2] on the paper's full sparsity grid {.5,.7,.8,.9,.95,.98}: the
+    per-V crossover with cuBLAS."""
+    return [Problem(M, K, N, V, S) for (M, K) in DLMC_MK for V in DLMC_V for S in DLMC_S_GRID
+            for N in DLMC_N]
+
+
 def dlmc_layer_workload():
     """configs[1] x configs[2]: 4 shapes x V{2,4,8} x S{.5,.7,.9,.98} x N{64,128,256}."""
     return [Problem(M, K, N, V, S) for (M, K) in DLMC_MK for V in DLMC_V for S in DLMC_S
@@ -80,6 +91,7 @@ def custom_workload():
 WORKLOADS = {
     "custom": custom_workload,
     "dlmc_layer": dlmc_layer_workload,
+    "dlmc_grid": dlmc_grid_workload,
     "rn50_layer": rn50_workload,
     "c1": lambda: [c1_problem()],
     # the paper's profiling case: A 2048x1024 x B 1024x256, 90% (Tables 2/3)
