@@ -859,11 +859,39 @@ static int64_t spmm_dkp(int64_t M, int64_t K, int64_t N, int V, const void* vals
   return spmm_dense_eligible(M, K, N, V, vals, B) ? ceil_div64(K, 64) * 64 : 0;
 }
 
+// tcgen05 gather-ring SpMM (spmm_tc.cu), build-time variant -DVS_SPMM_TC=1: it takes the problems
+// of the cp.async path (V >= 2, 16-byte aligned B and C, N % 8 == 0).
+#ifndef VS_SPMM_TC
+#define VS_SPMM_TC 0
+#endif
+#if VS_SPMM_TC
+bool spmm_tc_eligible(int64_t K, int64_t N, int V, const void* vals, const void* B);
+cudaError_t launch_spmm_tc(int64_t count, const int64_t* M, const int64_t* N, const int* V,
+                           const int32_t* const* row_ptr, const int32_t* const* col_idx,
+                           const void* const* vals, const void* const* B, void* const* const* C_dst,
+                           const int* nC, const int64_t* ldc, int num_sms, cudaStream_t s);
+static bool spmm_use_tc(const SpmmCfg& c, int64_t K, int64_t N, int V, const void* vals, const void* B) {
+  return c.CP != 0 && spmm_tc_eligible(K, N, V, vals, B);
+}
+#else
+static bool spmm_use_tc(const SpmmCfg&, int64_t, int64_t, int, const void*, const void*) { return false; }
+static cudaError_t launch_spmm_tc(int64_t, const int64_t*, const int64_t*, const int*, const int32_t* const*,
+                                  const int32_t* const*, const void* const*, const void* const*,
+                                  void* const* const*, const int*, const int64_t*, int, cudaStream_t) {
+  return cudaErrorNotSupported;
+}
+#endif
+
 cudaError_t launch_spmm(int64_t M, int64_t K, int64_t N, int V, const int32_t* row_ptr,
                         const int32_t* col_idx, const void* vals, const void* B, void* C,
                         int num_sms, cudaStream_t s) {
-  (void)num_sms;
   const SpmmCfg c = spmm_config(K, N, V, B, C);
+  if (spmm_use_tc(c, K, N, V, vals, B)) {
+    void* dst[1] = {C};
+    void* const* dsts = dst;
+    const int one = 1;
+    return launch_spmm_tc(1, &M, &N, &V, &row_ptr, &col_idx, &vals, &B, &dsts, &one, &N, num_sms, s);
+  }
   const SpmmKernels k = pick(c);
   int64_t W, nwg;
   const int64_t grid = spmm_blocks(k, c, M, N, V, &W, &nwg);
@@ -898,6 +926,8 @@ cudaError_t launch_spmm_scatter(int64_t M, int64_t K, int64_t N, int V, const in
   cd.n = n_dst;
   cd.ldc = ldc;
   const SpmmCfg c = spmm_config_al(K, N, V, (reinterpret_cast<uintptr_t>(B) & 15) == 0, c_al);
+  if (spmm_use_tc(c, K, N, V, vals, B))
+    return launch_spmm_tc(1, &M, &N, &V, &row_ptr, &col_idx, &vals, &B, &C_dst, &n_dst, &ldc, num_sms, s);
   const SpmmKernels k = pick(c);
   int64_t W, nwg;
   const int64_t grid = spmm_blocks(k, c, M, N, V, &W, &nwg);
@@ -928,8 +958,27 @@ cudaError_t launch_spmm_batched(int64_t count, const int64_t* M, const int64_t* 
   // group problem indices by configuration (stable: keeps the caller's order inside a group)
   std::vector<std::pair<SpmmCfg, int64_t>> order;
   order.reserve(count);
-  for (int64_t i = 0; i < count; ++i)
-    order.push_back({spmm_config(K[i], N[i], V[i], B[i], C[i]), i});
+  std::vector<int64_t> tcM, tcN, tcL;
+  std::vector<int> tcV, tcn;
+  std::vector<const int32_t*> tcR, tcI;
+  std::vector<const void*> tcA, tcB;
+  std::vector<void* const*> tcC;
+  for (int64_t i = 0; i < count; ++i) {
+    const SpmmCfg c = spmm_config(K[i], N[i], V[i], B[i], C[i]);
+    if (spmm_use_tc(c, K[i], N[i], V[i], vals[i], B[i])) {
+      tcM.push_back(M[i]); tcN.push_back(N[i]); tcL.push_back(N[i]); tcV.push_back(V[i]); tcn.push_back(1);
+      tcR.push_back(row_ptr[i]); tcI.push_back(col_idx[i]); tcA.push_back(vals[i]); tcB.push_back(B[i]);
+      tcC.push_back(&C[i]);
+      continue;
+    }
+    order.push_back({c, i});
+  }
+  if (!tcM.empty()) {
+    const cudaError_t e = launch_spmm_tc((int64_t)tcM.size(), tcM.data(), tcN.data(), tcV.data(), tcR.data(),
+                                         tcI.data(), tcA.data(), tcB.data(), tcC.data(), tcn.data(), tcL.data(),
+                                         num_sms, s);
+    if (e != cudaSuccess) return e;
+  }
   std::stable_sort(order.begin(), order.end(),
                    [](const auto& a, const auto& b) { return a.first < b.first; });
   SpmmBatch batch;
