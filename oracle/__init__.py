@@ -66,6 +66,8 @@ def lib():
             L.oracle_time_layer.restype = _I64
             L.oracle_time_layer.argtypes = [_I64, _I64, _I64, ctypes.c_int, _P, _P, _P,
                                             ctypes.c_int, ctypes.c_int, _P]
+            L.oracle_set_num_threads.restype = ctypes.c_int
+            L.oracle_set_num_threads.argtypes = [ctypes.c_int]
             L.oracle_num_threads.restype = ctypes.c_int
             L.oracle_num_threads.argtypes = []
             _lib = L
@@ -84,6 +86,16 @@ def _f16(a):
 
 def num_threads() -> int:
     return int(lib().oracle_num_threads())
+
+
+def use_all_cores() -> int:
+    """OpenMP team = every core this process may run on (os.sched_getaffinity), whatever
+    OMP_NUM_THREADS a launcher exported (torchrun sets 1).  Returns the team size."""
+    try:
+        n = len(os.sched_getaffinity(0))
+    except AttributeError:
+        n = os.cpu_count() or 1
+    return int(lib().oracle_set_num_threads(n))
 
 
 def half_to_double(h: int) -> float:

@@ -245,6 +245,20 @@ void oracle_softmax(int64_t M, int V, const int32_t* row_ptr, const uint16_t* va
   }
 }
 
+/* Threads of the OpenMP team (the CPU baseline uses every core of the host even when a
+   launcher exported OMP_NUM_THREADS=1); n <= 0 leaves it unchanged.  Returns the team size. */
+int oracle_set_num_threads(int n) {
+#ifdef _OPENMP
+  extern void omp_set_num_threads(int);
+  extern int omp_get_max_threads(void);
+  if (n > 0) omp_set_num_threads(n);
+  return omp_get_max_threads();
+#else
+  (void)n;
+  return 1;
+#endif
+}
+
 int oracle_num_threads(void) {
 #ifdef _OPENMP
   extern int omp_get_max_threads(void);
