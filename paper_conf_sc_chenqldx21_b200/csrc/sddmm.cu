@@ -26,6 +26,10 @@
 namespace vs {
 
 constexpr int kSddmmWarps = 4;
+// K % 128 == 0 (KC = 2 body) and K == 64 (pair body): unpredicated loads (load_seg2_fast)
+#ifndef VS_SDDMM_FAST
+#define VS_SDDMM_FAST 1
+#endif
 // resident CTAs per SM the register allocation is sized for (tools/tune.py over the DLMC batch:
 // 4 -> 551 us, 5 -> 516 us (12 B of spills), 6 -> 644 us, 8 -> 782 us: spills in the loop)
 #ifndef VS_SDDMM_MINB
@@ -51,6 +55,17 @@ __device__ __forceinline__ void load_seg2(const uint16_t* __restrict__ row, int6
     s1 = make_uint4(pack_h2(h[8], h[9]), pack_h2(h[10], h[11]), pack_h2(h[12], h[13]),
                     pack_h2(h[14], h[15]));
   }
+}
+
+// K % 64 == 0 fast path: no bounds predicates and no zero fill.  Slots past the window end and
+// MMA rows >= V read a valid dummy row (row 0) instead: they only feed accumulator rows / columns
+// that store_chunk never writes (rows >= M are written as +0 there), so every stored output is the
+// same sum in the same MMA order as the guarded path -> the same bits, with ~6 fewer instructions
+// per 16-byte load (the predicates, CS2R zeroing and branch of the guarded loads).
+__device__ __forceinline__ void load_seg2_fast(const uint16_t* __restrict__ row, int64_t k, uint4& s0,
+                                               uint4& s1) {
+  s0 = ldg128(row + k);
+  s1 = ldg128(row + k + 32);
 }
 
 __device__ __forceinline__ uint32_t wordj(const uint4& v, int j) {
@@ -90,7 +105,7 @@ __device__ __forceinline__ void store_chunk(const float (&acc)[4], int64_t v0, i
 // (The previous design -- contiguous 16-vector slices straddling windows, one 64-wide chunk
 // in flight -- paid a round trip per chunk on the A row and per window of a straddling
 // slice: 7 us for a 98%-sparse 512 x 512 mask at K = 256; this one takes 3.3 us.)
-template <int V, bool VEC, int KC, bool ARES>
+template <int V, bool VEC, int KC, bool ARES, int FAST = 0>
 __device__ __forceinline__ void sddmm_window(int64_t M, int64_t K,
                                              const int32_t* __restrict__ row_ptr,
                                              const int32_t* __restrict__ col_idx,
@@ -107,14 +122,17 @@ __device__ __forceinline__ void sddmm_window(int64_t M, int64_t K,
   if (v0 >= pe) return;
   const int64_t arow = w * V + g;
   const bool ok_row = (g < V) && (arow < M);
-  const uint16_t* rowA = A + arow * K;
+  const uint16_t* rowA = A + (FAST != 0 && !ok_row ? 0 : arow) * K;
   const bool one_block = K <= 64 * KC;
   int ca = (v0 + g < pe) ? ldg32i(col_idx + v0 + g) : 0;
   int cb = (v0 + g + 8 < pe) ? ldg32i(col_idx + v0 + g + 8) : 0;
   uint4 xx0[KC], xx1[KC];  // A rows of the window, K block
   if (one_block) {
 #pragma unroll
-    for (int c = 0; c < KC; ++c) load_seg2<VEC>(rowA, K, 64 * c + kt, ok_row, xx0[c], xx1[c]);
+    for (int c = 0; c < KC; ++c) {
+      if (FAST != 0) load_seg2_fast(rowA, 64 * c + kt, xx0[c], xx1[c]);
+      else load_seg2<VEC>(rowA, K, 64 * c + kt, ok_row, xx0[c], xx1[c]);
+    }
   }
   for (; v0 < pe; v0 += 16 * q) {
     const bool oka = v0 + g < pe, okb = v0 + g + 8 < pe;
@@ -129,9 +147,17 @@ __device__ __forceinline__ void sddmm_window(int64_t M, int64_t K,
 #pragma unroll
       for (int c = 0; c < KC; ++c) {
         const int64_t k = kb + 64 * c + kt;
-        load_seg2<VEC>(rowa, K, k, oka, xa0[c], xa1[c]);
-        load_seg2<VEC>(rowb, K, k, okb, xb0[c], xb1[c]);
-        if (!one_block) load_seg2<VEC>(rowA, K, k, ok_row, xx0[c], xx1[c]);
+        // FAST 1: every chunk unpredicated (slots past the window end read row 0); FAST 2: only
+        // full chunks (warp-uniform test), the tail chunk keeps the guarded loads
+        if (FAST == 1 || (FAST == 2 && v0 + 16 <= pe)) {
+          load_seg2_fast(rowa, k, xa0[c], xa1[c]);
+          load_seg2_fast(rowb, k, xb0[c], xb1[c]);
+          if (!one_block) load_seg2_fast(rowA, k, xx0[c], xx1[c]);
+        } else {
+          load_seg2<VEC>(rowa, K, k, oka, xa0[c], xa1[c]);
+          load_seg2<VEC>(rowb, K, k, okb, xb0[c], xb1[c]);
+          if (!one_block) load_seg2<VEC>(rowA, K, k, ok_row, xx0[c], xx1[c]);
+        }
       }
 #pragma unroll
       for (int c = 0; c < KC; ++c)
@@ -150,7 +176,7 @@ __device__ __forceinline__ void sddmm_window(int64_t M, int64_t K,
 // 8 LDG.128 per thread before the first MMA instead of 4, so a warp keeps twice the gather
 // bytes in flight at the same occupancy (register cost = the KC = 2 body's).  Each chunk's
 // accumulation order is the KC = 1 body's, so the bits are identical.
-template <int V>
+template <int V, int FAST = 0>
 __device__ __forceinline__ void sddmm_window_pair(int64_t M, int64_t K,
                                                   const int32_t* __restrict__ row_ptr,
                                                   const int32_t* __restrict__ col_idx,
@@ -169,16 +195,26 @@ __device__ __forceinline__ void sddmm_window_pair(int64_t M, int64_t K,
   const int64_t sq = 16 * q;
   auto col = [&](int64_t v) { return (v < pe) ? ldg32i(col_idx + v) : 0; };
   int c0a = col(v0 + g), c0b = col(v0 + g + 8), c1a = col(v0 + sq + g), c1b = col(v0 + sq + g + 8);
+  // K == 64: see load_seg2_fast (absent slots read row 0, never stored); FAST 2 only for pairs
+  // of full chunks
   uint4 xx0, xx1;
-  load_seg2<true>(A + arow * K, K, kt, ok_row, xx0, xx1);
+  if (FAST != 0) load_seg2_fast(A + (ok_row ? arow : 0) * K, kt, xx0, xx1);
+  else load_seg2<true>(A + arow * K, K, kt, ok_row, xx0, xx1);
   for (; v0 < pe; v0 += 2 * sq) {
     const int64_t v1 = v0 + sq, n0 = v0 + 2 * sq, n1 = n0 + sq;
     const int n0a = col(n0 + g), n0b = col(n0 + g + 8), n1a = col(n1 + g), n1b = col(n1 + g + 8);
     uint4 a0[2], a1[2], b0[2], b1[2];
-    load_seg2<true>(Bt + (int64_t)c0a * K, K, kt, v0 + g < pe, a0[0], a1[0]);
-    load_seg2<true>(Bt + (int64_t)c0b * K, K, kt, v0 + g + 8 < pe, b0[0], b1[0]);
-    load_seg2<true>(Bt + (int64_t)c1a * K, K, kt, v1 + g < pe, a0[1], a1[1]);
-    load_seg2<true>(Bt + (int64_t)c1b * K, K, kt, v1 + g + 8 < pe, b0[1], b1[1]);
+    if (FAST == 1 || (FAST == 2 && v1 + 16 <= pe)) {
+      load_seg2_fast(Bt + (int64_t)c0a * K, kt, a0[0], a1[0]);
+      load_seg2_fast(Bt + (int64_t)c0b * K, kt, b0[0], b1[0]);
+      load_seg2_fast(Bt + (int64_t)c1a * K, kt, a0[1], a1[1]);
+      load_seg2_fast(Bt + (int64_t)c1b * K, kt, b0[1], b1[1]);
+    } else {
+      load_seg2<true>(Bt + (int64_t)c0a * K, K, kt, v0 + g < pe, a0[0], a1[0]);
+      load_seg2<true>(Bt + (int64_t)c0b * K, K, kt, v0 + g + 8 < pe, b0[0], b1[0]);
+      load_seg2<true>(Bt + (int64_t)c1a * K, K, kt, v1 + g < pe, a0[1], a1[1]);
+      load_seg2<true>(Bt + (int64_t)c1b * K, K, kt, v1 + g + 8 < pe, b0[1], b1[1]);
+    }
     float acc0[4] = {0.f, 0.f, 0.f, 0.f}, acc1[4] = {0.f, 0.f, 0.f, 0.f};
 #pragma unroll
     for (int j = 0; j < 4; ++j)
@@ -197,7 +233,7 @@ __device__ __forceinline__ void sddmm_window_pair(int64_t M, int64_t K,
 // ARES slot = "mixed K blocks": one kernel serves both K <= 64 (KC = 1 body) and K > 64
 // (KC = 2 body), chosen per problem at run time, so a batch needs one launch per V instead of
 // one per (V, KC) group (no tail between the two launches).  Same bodies, same bits.
-template <int V, bool VEC, int KC, bool ARES>
+template <int V, bool VEC, int KC, bool ARES, int FAST = 0>
 __device__ __forceinline__ void sddmm_window_any(int64_t M, int64_t K,
                                                  const int32_t* __restrict__ row_ptr,
                                                  const int32_t* __restrict__ col_idx,
@@ -205,7 +241,14 @@ __device__ __forceinline__ void sddmm_window_any(int64_t M, int64_t K,
                                                  const uint16_t* __restrict__ Bt,
                                                  uint16_t* __restrict__ out, bool out4, int64_t w,
                                                  int64_t j0, int64_t q, bool pair) {
-  if constexpr (ARES && VEC) {
+  if constexpr (ARES && VEC && FAST != 0) {
+    // only K == 64 or K % 128 == 0 problems reach this instantiation (sddmm_fast_ok)
+    (void)pair;
+    if (K <= 64)
+      sddmm_window_pair<V, FAST>(M, K, row_ptr, col_idx, A, Bt, out, out4, w, j0, q);
+    else
+      sddmm_window<V, VEC, 2, false, FAST>(M, K, row_ptr, col_idx, A, Bt, out, out4, w, j0, q);
+  } else if constexpr (ARES && VEC) {
     if (K <= 64 && pair)
       sddmm_window_pair<V>(M, K, row_ptr, col_idx, A, Bt, out, out4, w, j0, q);
     else if (K <= 64)
@@ -239,7 +282,7 @@ __device__ __forceinline__ int64_t sddmm_q(int64_t chunks, int64_t W, int64_t pe
   return q < 1 ? 1 : (q > 64 ? 64 : q);
 }
 
-template <int V, bool VEC, int KC, bool ARES>
+template <int V, bool VEC, int KC, bool ARES, bool FAST = false>
 __global__ void __launch_bounds__(kSddmmWarps * 32, VS_SDDMM_MINB)
     sddmm_kernel(int64_t M, int64_t K, int64_t W, const int32_t* __restrict__ row_ptr,
                  const int32_t* __restrict__ col_idx, const uint16_t* __restrict__ A,
@@ -255,8 +298,9 @@ __global__ void __launch_bounds__(kSddmmWarps * 32, VS_SDDMM_MINB)
     const int64_t w = it / q;
     const int64_t qq = sddmm_gather_q(dense_ok, N, V, W, row_ptr, col_idx, w, it - w * q, q);
     if (qq == 0) continue;
-    sddmm_window_any<V, VEC, KC, ARES>(M, K, row_ptr, col_idx, A, Bt, out, out4, w,
-                                       qq == q ? it - w * q : 0, qq, pair);
+    // single-problem kernel: FAST mode 1 (measured best per call, profiles/r02_sddmm_variants.md)
+    sddmm_window_any<V, VEC, KC, ARES, FAST ? 1 : 0>(M, K, row_ptr, col_idx, A, Bt, out, out4, w,
+                                                     qq == q ? it - w * q : 0, qq, pair);
   }
 }
 
@@ -282,7 +326,7 @@ struct SddmmBatch {
   SddmmDesc d[kSddmmMaxBatch];
 };
 
-template <int V, bool VEC, int KC, bool ARES>
+template <int V, bool VEC, int KC, bool ARES, bool FAST = false>
 __global__ void __launch_bounds__(kSddmmWarps * 32, VS_SDDMM_MINB)
     sddmm_batched_kernel(const __grid_constant__ SddmmBatch b) {
   __shared__ int64_t pre[kSddmmMaxBatch + 1];  // prefix of work items
@@ -338,8 +382,10 @@ __global__ void __launch_bounds__(kSddmmWarps * 32, VS_SDDMM_MINB)
     const int64_t w = loc / q;
     const int64_t qq = sddmm_gather_q(d.dense_ok != 0, d.N, V, d.W, d.row_ptr, d.col_idx, w, loc - w * q, q);
     if (qq == 0) continue;
-    sddmm_window_any<V, VEC, KC, ARES>(d.M, d.K, d.row_ptr, d.col_idx, d.A, d.Bt, d.out,
-                                       d.out4 != 0, w, qq == q ? loc - w * q : 0, qq, b.pair != 0);
+    // batched kernel: FAST mode 2 (full chunks only: many short windows in a batch)
+    sddmm_window_any<V, VEC, KC, ARES, FAST ? 2 : 0>(d.M, d.K, d.row_ptr, d.col_idx, d.A, d.Bt, d.out,
+                                                     d.out4 != 0, w, qq == q ? loc - w * q : 0, qq,
+                                                     b.pair != 0);
   }
 }
 
@@ -373,8 +419,9 @@ static int sddmm_variant(int64_t K, bool vec) {
   constexpr int cap = VS_SDDMM_KC >= 2 ? 2 : 1;
   int kc = (!vec || K <= 64) ? 1 : 2;
   if (kc > cap) kc = cap;
-  // vector-path problems of any K share the mixed kernel
-  if (vec && VS_SDDMM_MIX && cap == 2) return 2 * 2 + 1;
+  // vector-path problems of any K share the mixed kernel; K == 64 and K % 128 == 0 take its
+  // unpredicated-load instantiation (code 6)
+  if (vec && VS_SDDMM_MIX && cap == 2) return (VS_SDDMM_FAST && K > 0 && (K == 64 || K % 128 == 0)) ? 6 : 2 * 2 + 1;
   return kc * 2;
 }
 
@@ -382,25 +429,25 @@ static int sddmm_variant(int64_t K, bool vec) {
 // (sddmm_window_pair); VS_SDDMM_PAIR=0 selects the one-chunk body.  Same bits either way.
 static constexpr bool sddmm_pair_on() { return VS_SDDMM_PAIR != 0; }
 
-template <int V, bool VEC, int KC, bool ARES>
+template <int V, bool VEC, int KC, bool ARES, bool FAST = false>
 static int sddmm_ctas_per_sm() {
-  static const int n = ctas_per_sm(sddmm_kernel<V, VEC, KC, ARES>);
+  static const int n = ctas_per_sm(sddmm_kernel<V, VEC, KC, ARES, FAST>);
   return n;
 }
-template <int V, bool VEC, int KC, bool ARES>
+template <int V, bool VEC, int KC, bool ARES, bool FAST = false>
 static int sddmm_batched_ctas_per_sm() {
-  static const int n = ctas_per_sm(sddmm_batched_kernel<V, VEC, KC, ARES>);
+  static const int n = ctas_per_sm(sddmm_batched_kernel<V, VEC, KC, ARES, FAST>);
   return n;
 }
 
-template <int V, bool VEC, int KC, bool ARES>
+template <int V, bool VEC, int KC, bool ARES, bool FAST = false>
 static void launch_sddmm_one(int64_t M, int64_t K, const int32_t* row_ptr, const int32_t* col_idx,
                              const uint16_t* A, const uint16_t* Bt, uint16_t* out, int num_sms,
                              cudaStream_t s, int64_t N, bool dense_ok) {
   const int64_t W = ceil_div64(M, V);
   const bool out4 = (reinterpret_cast<uintptr_t>(out) & 3) == 0;
-  dim3 grid((unsigned)(num_sms * sddmm_ctas_per_sm<V, VEC, KC, ARES>()));
-  sddmm_kernel<V, VEC, KC, ARES><<<grid, kSddmmWarps * 32, 0, s>>>(M, K, W, row_ptr, col_idx, A,
+  dim3 grid((unsigned)(num_sms * sddmm_ctas_per_sm<V, VEC, KC, ARES, FAST>()));
+  sddmm_kernel<V, VEC, KC, ARES, FAST><<<grid, kSddmmWarps * 32, 0, s>>>(M, K, W, row_ptr, col_idx, A,
                                                                    Bt, out, out4, sddmm_pair_on(),
                                                                    N, dense_ok);
 }
@@ -431,6 +478,7 @@ static cudaError_t launch_sddmm_v(int64_t M, int64_t N, int64_t K, const int32_t
     case 8 + 3: launch_sddmm_one<V, true, 1, true>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok); break;
     case 8 + 4: launch_sddmm_one<V, true, 2, false>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok); break;
     case 8 + 5: launch_sddmm_one<V, true, 2, true>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok); break;
+    case 8 + 6: launch_sddmm_one<V, true, 2, true, true>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok); break;
     case 3: launch_sddmm_one<V, false, 1, true>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok); break;
     default: launch_sddmm_one<V, false, 1, false>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok); break;
   }
@@ -442,7 +490,7 @@ static cudaError_t launch_sddmm_v(int64_t M, int64_t N, int64_t K, const int32_t
   return launch_sddmm_dense(1, &M, &N, &K, &V_, &row_ptr, &col_idx, &a, &bt, &o, num_sms, s);
 }
 
-template <int V, bool VEC, int KC, bool ARES>
+template <int V, bool VEC, int KC, bool ARES, bool FAST = false>
 static void launch_sddmm_batch(const SddmmBatch& b, int num_sms, cudaStream_t s) {
   // VS_SDDMM_OVERSUB (build time): grid = that many times the resident CTAs.  2 is 5% faster
   // for the SDDMM batch alone but 2% slower for the bench step, where the oversubscribed grid
@@ -451,8 +499,8 @@ static void launch_sddmm_batch(const SddmmBatch& b, int num_sms, cudaStream_t s)
 #define VS_SDDMM_OVERSUB 1
 #endif
   constexpr int over = VS_SDDMM_OVERSUB < 1 ? 1 : VS_SDDMM_OVERSUB;
-  dim3 grid((unsigned)(num_sms * sddmm_batched_ctas_per_sm<V, VEC, KC, ARES>() * over));
-  sddmm_batched_kernel<V, VEC, KC, ARES><<<grid, kSddmmWarps * 32, 0, s>>>(b);
+  dim3 grid((unsigned)(num_sms * sddmm_batched_ctas_per_sm<V, VEC, KC, ARES, FAST>() * over));
+  sddmm_batched_kernel<V, VEC, KC, ARES, FAST><<<grid, kSddmmWarps * 32, 0, s>>>(b);
 }
 
 template <int V>
@@ -462,6 +510,7 @@ static void launch_sddmm_batch_v(const SddmmBatch& b, int code, int num_sms, cud
     case 8 + 3: return launch_sddmm_batch<V, true, 1, true>(b, num_sms, s);
     case 8 + 4: return launch_sddmm_batch<V, true, 2, false>(b, num_sms, s);
     case 8 + 5: return launch_sddmm_batch<V, true, 2, true>(b, num_sms, s);
+    case 8 + 6: return launch_sddmm_batch<V, true, 2, true, true>(b, num_sms, s);
     case 3: return launch_sddmm_batch<V, false, 1, true>(b, num_sms, s);
     default: return launch_sddmm_batch<V, false, 1, false>(b, num_sms, s);
   }
