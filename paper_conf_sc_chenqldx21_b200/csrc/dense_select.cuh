@@ -18,13 +18,16 @@
 
 #include "common.cuh"
 
-// VS_DENSE_CF = 0 (the shipped library): the dense-tile kernels are not built and never
-// launched; every row block stays with the gather kernels.  Measured on B200 (DESIGN.md §7.8,
-// profiles/r02_dense_tile.md): with the current dense-tile kernels a 32-row unit costs ~9-13 us
-// of pipeline latency, so over the DLMC set they beat the gather kernels only for the largest
-// 50%-sparse SDDMM problems; an opt-in build (-DVS_DENSE_CF=<flop per byte>) enables them.
-#ifndef VS_DENSE_CF
-#define VS_DENSE_CF 0
+// Build-time cost-model constants (flop per gathered byte), one per op; 0 = the dense-tile
+// kernel of that op is not built and never launched (every row block stays with the gather
+// kernel).  VS_SDDMM_DENSE_CF: the 128 x 128-unit SDDMM kernel (dense_tile.cu), tuned on B200
+// over the DLMC batch.  VS_SPMM_DENSE_CF: the dense-tile SpMM, measured slower
+// than the gather kernel at DLMC sizes (profiles/r02_dense_tile.md) -> 0 in the shipped library.
+#ifndef VS_SDDMM_DENSE_CF
+#define VS_SDDMM_DENSE_CF 64
+#endif
+#ifndef VS_SPMM_DENSE_CF
+#define VS_SPMM_DENSE_CF 0
 #endif
 
 namespace vs {
@@ -38,27 +41,41 @@ __host__ __device__ __forceinline__ void rb_windows(int64_t rb, int V, int64_t W
   if (w1 > W) w1 = W;
 }
 
-// dense iff nnz_v(rb) * CF > 128 * Lc (Lc padded to the dense tile granularity)
+// dense iff nnz_v(rb) * cf > 128 * Lc (Lc padded to the dense tile granularity)
 __device__ __forceinline__ bool rb_is_dense(const int32_t* __restrict__ row_ptr, int64_t W, int V,
-                                            int64_t rb, int64_t Lc_padded) {
+                                            int64_t rb, int64_t Lc_padded, int64_t cf) {
   int64_t w0, w1;
   rb_windows(rb, V, W, w0, w1);
   const int64_t nnz = (int64_t)__ldg(row_ptr + w1) - (int64_t)__ldg(row_ptr + w0);
-  return nnz * (int64_t)VS_DENSE_CF > (int64_t)kDenseRows * Lc_padded;
+  return nnz * cf > (int64_t)kDenseRows * Lc_padded;
+}
+// SDDMM [M x N mask]: Lc = the mask columns padded to the 128-column tiles of the dense kernel
+__device__ __forceinline__ bool sddmm_rb_dense(const int32_t* __restrict__ row_ptr, int64_t W, int V,
+                                               int64_t rb, int64_t N) {
+  return rb_is_dense(row_ptr, W, V, rb, ceil_div64(N, 128) * 128, (int64_t)VS_SDDMM_DENSE_CF);
 }
 
-// warp-uniform: col_idx[pb, pe) strictly ascending (every lane returns the same answer)
-__device__ __forceinline__ bool window_sorted(const int32_t* __restrict__ col_idx, int64_t pb, int64_t pe) {
+// warp-uniform: col_idx[pb, pe) strictly ascending (every lane returns the same answer).
+// 128 entries per round trip (4 coalesced loads per lane in flight).
+static __device__ __noinline__ bool window_sorted(const int32_t* __restrict__ col_idx, int64_t pb, int64_t pe) {
   const int lane = lane_id();
-  int prev_last = -1;  // last entry of the previous batch (entries are >= 0)
-  for (int64_t base = pb; base < pe; base += 32) {
-    const int64_t p = base + lane;
-    const int c = p < pe ? __ldg(col_idx + p) : 0x7fffffff;
-    int prev = __shfl_up_sync(0xffffffffu, c, 1);
-    if (lane == 0) prev = prev_last;
-    const bool bad = (p < pe) && (c <= prev);
+  int prev_last = -1;  // last entry of the previous row of 32 (entries are >= 0)
+  for (int64_t base = pb; base < pe; base += 128) {
+    int c[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int64_t p = base + 32 * j + lane;
+      c[j] = p < pe ? __ldg(col_idx + p) : 0x7fffffff;
+    }
+    bool bad = false;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      int prev = __shfl_up_sync(0xffffffffu, c[j], 1);
+      if (lane == 0) prev = prev_last;
+      bad |= (base + 32 * j + lane < pe) && (c[j] <= prev);
+      prev_last = __shfl_sync(0xffffffffu, c[j], 31);
+    }
     if (__any_sync(0xffffffffu, bad)) return false;
-    prev_last = __shfl_sync(0xffffffffu, c, 31);
   }
   return true;
 }

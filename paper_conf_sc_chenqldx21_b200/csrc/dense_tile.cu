@@ -4,27 +4,27 @@
 // Why: a stored V x 1 vector gives the gather kernels V flop per gathered byte
 // (AL1), and B200 moves ~8-20 TB/s of random rows from L2 into the SMs against
 // ~1.5-2 PFLOP/s of dense fp16 tensor throughput.  Where a 128-row block holds more than
-// 128 * Lc / VS_DENSE_CF stored vectors, computing its whole dense tile on the tensor cores
-// costs less than gathering its vectors.  The results are the same sums (fp32 accumulate,
-// fp16 round-to-nearest-even output); absent vectors only add exact zero products (SpMM) or
-// are not stored (SDDMM).
+// 128 * Lc / CF stored vectors, computing its whole dense tile on the tensor cores costs less
+// than gathering its vectors.  The results are the same sums (fp32 accumulate, fp16
+// round-to-nearest-even output); absent vectors only add exact zero products (SpMM) or are not
+// stored (SDDMM).
 //
 // SDDMM  out[p*V + r] = sum_k A[wV+r][k] * Bt[col_idx[p]][k]   (§6)
-//   Unit = (problem, 32-row block of A = rows [i0, i0+32), range of <= 1024 mask columns).
-//   Per column tile c0 (128 mask columns): D[128 mask cols x 32 A rows] (fp32, TMEM) =
-//   Bt[c0:c0+128, :] * A[i0:i0+32, :]^T, tcgen05.mma M = 128, N = 32, K = 16 (operand switch
-//   of P:1059-1063: mask columns on the MMA M side); both operands are K-contiguous rows loaded
-//   by TMA 2-D tile copies (SWIZZLE_128B = the canonical K-major layout); the A rows of the unit
-//   (K <= 256) stay resident in shared memory.  Each finished tile is drained TMEM -> fp16 (RN)
-//   into a shared [32 rows x 1024 columns] tile, so the whole column range of the unit is on
-//   chip; then ONE flat pass over the unit's stored vectors (contiguous in col_idx: the windows
-//   of the 32 rows) writes out[p*V .. p*V+V) for every vector whose column is in the range --
-//   any col_idx order, duplicates included, coalesced 2V-byte stores.
-//   Warp roles: warp 0 TMA producer, warp 1 MMA issuer (one elected lane) + TMEM owner,
-//   warps 2-9 epilogue (TMEM lane quarter = warp % 4, column half = (warp - 2) / 4).  Two TMEM
-//   accumulators: the drain of tile t overlaps the MMAs of tile t + 1.
+//   Unit = (problem, 128-row block rb of A, 128-column tile ct of the mask): one CTA of 4 warps,
+//   non-persistent (3 resident per SM, so one CTA's loads overlap another's MMAs / epilogue).
+//   D[128 mask cols x 128 A rows] (fp32, TMEM, 128 columns) = Bt[c0:c0+128, :] * A[r0:r0+128, :]^T
+//   with tcgen05.mma M = 128, N = 128, K = 16 (the operand switch of P:1059-1063: mask columns on
+//   the MMA M side), both operands K-contiguous rows loaded by TMA 2-D tile copies (SWIZZLE_128B
+//   = the canonical K-major layout), a 2-stage ring of 64-wide K slabs (any inner K).  Warp 0
+//   lane 0 issues the TMA copies, warp 1 lane 0 the MMAs; then every warp drains its TMEM lane
+//   quarter (thread = mask column c) into a shared tile Tt[c][r] (fp16 RN, rows >= M are +0;
+//   each c a 256-byte row, 16-byte chunks XOR-swizzled by c), so the V rows of a window at
+//   column c are 2V contiguous bytes.  Sampling: warp j takes windows j, j+4, ... of the row
+//   block and walks each window's col_idx (16-byte loads); every stored vector whose column
+//   falls in the tile gets one 2V-byte shared load and one 2V-byte global store -- any col_idx
+//   order, duplicates included.
 //
-// SpMM  C[i][n] = sum_p vals[p*V + i%V] * B[col_idx[p]][n]   (§5)
+// SpMM  C[i][n] = sum_p vals[p*V + i%V] * B[col_idx[p]][n]   (§5)  [opt-in build]
 //   Unit = (problem, 32-row block of A / C).  The unit's stored vectors (contiguous: the
 //   windows of the 32 rows) are decoded once into a dense [32 rows x K] fp16 tile in shared
 //   memory (K-major, 128-byte swizzle; K <= 2048), then for every 128-column panel of B:
@@ -45,32 +45,42 @@
 #include "dense_select.cuh"
 #include "tc_common.cuh"
 
-#if VS_DENSE_CF > 0  // opt-in build only (dense_select.cuh)
+#if VS_SDDMM_DENSE_CF > 0 || VS_SPMM_DENSE_CF > 0
 namespace vs {
 namespace dt {
 
-constexpr int kCtPerUnit = 8;   // column tiles of 128 per SDDMM unit (1024 columns)
-constexpr int kMaxProb = 32;    // problems per launch (tensor maps travel as kernel parameters)
-constexpr int kSdRows = 32;     // A rows per SDDMM unit (MMA N)
-constexpr int kSdThreads = 320; // 10 warps
-constexpr int kSdEpi = 256;     // epilogue threads (warps 2-9)
-constexpr int kBtTile = 128 * 128;        // 128 mask columns x 64 k fp16 (16 KB)
-constexpr int kATile = kSdRows * 128;     // 32 rows x 64 k fp16 (4 KB)
-constexpr int kSdKbMax = 4;               // K <= 256 (A resident)
-constexpr int kSdStages = 8;   // 128 KB of Bt tiles in flight per SM (the stream is latency-bound)
-constexpr int kSdDhBytes = kSdRows * kCtPerUnit * 128 * 2;  // 64 KB
-constexpr int kSdSmem = kSdKbMax * kATile + kSdStages * kBtTile + kSdDhBytes + 1024;
-constexpr uint32_t kIdescSd = tc::idesc_f16(128, kSdRows, 0, 0);
+constexpr int kMaxProb = 32;  // problems per launch (tensor maps travel as kernel parameters)
+
+static PFN_cuTensorMapEncodeTiled_v12000 tmap_encoder();
+static bool make_kmajor_map(CUtensorMap* m, const void* base, int64_t rows, int64_t K, int box_rows);
+static bool make_mnmajor_map(CUtensorMap* m, const void* base, int64_t K, int64_t N);
+
+}  // namespace dt
+}  // namespace vs
+#endif
+
+#if VS_SDDMM_DENSE_CF > 0
+namespace vs {
+namespace dt {
+
+// ================================================================================ SDDMM
+constexpr int kSdThreads = 128;              // 4 warps = the 4 TMEM lane quarters
+constexpr int kSdSlab = 128 * 128;           // bytes: 128 rows x 64 k fp16 (16 KB)
+constexpr int kSdStage = 2 * kSdSlab;        // Bt slab + A slab
+constexpr int kSdStages = 2;
+constexpr int kSdSmem = kSdStages * kSdStage + 1024;  // + 1024-byte alignment slack (SWIZZLE_128B)
+constexpr int kSdCtasPerSm = 3;
+constexpr uint32_t kIdescSd = tc::idesc_f16(128, 128, 0, 0);
+static_assert(128 * 256 <= kSdStages * kSdStage, "Tt tile reuses the stage ring");
 
 struct alignas(64) SdDesc {
-  CUtensorMap tmA;   // A [M x K] fp16, box {64, 32}, SWIZZLE_128B
+  CUtensorMap tmA;   // A [M x K] fp16, box {64, 128}, SWIZZLE_128B
   CUtensorMap tmBt;  // Bt [N x K] fp16, box {64, 128}, SWIZZLE_128B
-  int64_t M, N, K, W, n_cr, n_rb;
+  int64_t M, N, K, W, n_ct;
   const int32_t* row_ptr;
   const int32_t* col_idx;
   uint16_t* out;
-  int64_t nnz_total;  // (not known on the host: unused)
-  int32_t V, out_vec;  // out_vec: out is 2V-byte aligned (one store per vector)
+  int32_t V, out_vec;  // out_vec: out is 2V-byte aligned
 };
 struct SdBatch {
   int count;
@@ -78,55 +88,151 @@ struct SdBatch {
   SdDesc d[kMaxProb];
 };
 
-// unit -> (problem, 32-row block, column-tile range); problems in ascending unit order
-struct UnitIt {
-  int p;
-  __device__ __forceinline__ void locate(const SdBatch& b, int64_t u, int64_t& rb, int64_t& ct0,
-                                         int64_t& ct1) {
-    while (b.first_unit[p + 1] <= u) ++p;
-    const SdDesc& d = b.d[p];
-    const int64_t loc = u - b.first_unit[p];
-    rb = loc / d.n_cr;
-    const int64_t cr = loc - rb * d.n_cr;
-    const int64_t nct = ceil_div64(d.N, 128);
-    ct0 = cr * kCtPerUnit;
-    ct1 = ct0 + kCtPerUnit < nct ? ct0 + kCtPerUnit : nct;
+template <int V>
+__device__ __forceinline__ void sd_sample_store(uint32_t a, uint16_t* dst, bool vec) {
+  if (V == 8) {
+    const uint4 t = lds128_u32(a);
+    if (vec) {
+      *reinterpret_cast<uint4*>(dst) = t;
+    } else {
+      const uint32_t w[4] = {t.x, t.y, t.z, t.w};
+#pragma unroll
+      for (int r = 0; r < 8; ++r) dst[r] = (uint16_t)(w[r >> 1] >> (16 * (r & 1)));
+    }
+  } else if (V == 4) {
+    uint32_t x, y;
+    asm volatile("ld.shared.v2.u32 {%0,%1}, [%2];" : "=r"(x), "=r"(y) : "r"(a));
+    if (vec) {
+      *reinterpret_cast<uint2*>(dst) = make_uint2(x, y);
+    } else {
+      dst[0] = (uint16_t)x; dst[1] = (uint16_t)(x >> 16); dst[2] = (uint16_t)y; dst[3] = (uint16_t)(y >> 16);
+    }
+  } else if (V == 2) {
+    uint32_t x;
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(x) : "r"(a));
+    if (vec) {
+      *reinterpret_cast<uint32_t*>(dst) = x;
+    } else {
+      dst[0] = (uint16_t)x; dst[1] = (uint16_t)(x >> 16);
+    }
+  } else {
+    dst[0] = lds16(a);
   }
-};
-
-// the 32-row block rb32 belongs to the 128-row block of the dense/gather decision
-__device__ __forceinline__ bool sd_unit_dense(const SdDesc& d, int64_t rb32) {
-  return rb_is_dense(d.row_ptr, d.W, d.V, rb32 / (kDenseRows / kSdRows), ceil_div64(d.N, 128) * 128);
 }
 
-__global__ void __launch_bounds__(kSdThreads, 1) sddmm_dense_kernel(const __grid_constant__ SdBatch b) {
-  extern __shared__ uint8_t smem_raw[];
-  __shared__ __align__(8) uint64_t full_bar[kSdStages], empty_bar[kSdStages];
-  __shared__ __align__(8) uint64_t tfull_bar[2], tempty_bar[2], afull_bar, aempty_bar;
-  __shared__ uint32_t tmem_base_sh;
-  __shared__ int32_t wptr[kSdRows + 1];  // row_ptr of the unit's windows (relative to nothing)
-  const uint32_t smem = (smem_u32(smem_raw) + 1023u) & ~1023u;
-  const uint32_t s_ares = smem;                            // A tiles of the unit (kSdKbMax x 4 KB)
-  const uint32_t s_stage = smem + kSdKbMax * kATile;       // Bt stage ring
-  const uint32_t s_dh = s_stage + kSdStages * kBtTile;     // Dh [32 rows][2048 cols] fp16
-  const int warp = threadIdx.x >> 5, lane = lane_id();
-  const int64_t total = b.first_unit[b.count];
+// Smallest i in [lo, hi] with a[i] >= x, for two targets at once (a[lo, hi) ascending, a[hi]
+// taken as +inf): 9-ary search, 8 independent probes per target per round trip (a 1024-entry
+// window takes 3 rounds + one of <= 8 loads), so the latency of one thread's search is ~4 L2
+// round trips.  On a window that is not ascending the result is some index in [lo, hi].
+__device__ __forceinline__ void kary_lower_bound2(const int32_t* __restrict__ a, int lo, int hi, int x1, int x2,
+                                                  int& r1, int& r2) {
+  int l1 = lo, h1 = hi, l2 = lo, h2 = hi;
+  while (h1 - l1 > 8 || h2 - l2 > 8) {
+    const int s1 = (h1 - l1) / 9, s2 = (h2 - l2) / 9;
+    int c1 = 0, c2 = 0;
+#pragma unroll
+    for (int i = 1; i <= 8; ++i) {
+      c1 += (s1 > 0 && __ldg(a + l1 + s1 * i) < x1) ? 1 : 0;
+      c2 += (s2 > 0 && __ldg(a + l2 + s2 * i) < x2) ? 1 : 0;
+    }
+    if (s1 > 0) {
+      const int nh = c1 < 8 ? l1 + s1 * (c1 + 1) : h1;
+      l1 = c1 > 0 ? l1 + s1 * c1 + 1 : l1;
+      h1 = nh;
+    }
+    if (s2 > 0) {
+      const int nh = c2 < 8 ? l2 + s2 * (c2 + 1) : h2;
+      l2 = c2 > 0 ? l2 + s2 * c2 + 1 : l2;
+      h2 = nh;
+    }
+  }
+  int c1 = 0, c2 = 0;
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    c1 += (l1 + i < h1 && __ldg(a + l1 + i) < x1) ? 1 : 0;
+    c2 += (l2 + i < h2 && __ldg(a + l2 + i) < x2) ? 1 : 0;
+  }
+  r1 = l1 + c1;
+  r2 = l2 + c2;
+}
 
+// Store pass of one unit: warp j takes windows j, j + 4, ... of the block, four windows per
+// round with their first 64 vectors' col_idx loads in flight together (lane = vector: coalesced
+// loads, 2V-byte shared load + 2V-byte global store each); the window's vectors in the tile's
+// column range are [lo, hi) (searched before the drain).  A vector whose column is outside the
+// range (possible only in a window that is not ascending) is not stored.
+template <int V>
+__device__ __forceinline__ void sd_store1(const SdDesc& d, uint32_t tt, uint32_t rofs, int e, int col, int c0,
+                                          bool vec) {
+  const uint32_t c = (uint32_t)(col - c0);
+  if (col >= 0 && c < 128u)
+    sd_sample_store<V>(tt + c * 256 + (((rofs >> 3) ^ (c & 15)) << 4) + (rofs & 7) * 2, d.out + (int64_t)e * V, vec);
+}
+template <int V>
+__device__ __forceinline__ void sd_store(const SdDesc& d, uint32_t tt, const int32_t* lo_s, const int32_t* hi_s,
+                                         int nwin, int c0, int warp, int lane) {
+  const bool vec = d.out_vec != 0;
+  const int32_t* __restrict__ ci = d.col_idx;
+  for (int wb = warp; wb < nwin; wb += 16) {
+    int lo[4], hi[4], ca[4], cb[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const int wl = wb + 4 * u;
+      lo[u] = wl < nwin ? lo_s[wl] : 0;
+      hi[u] = wl < nwin ? hi_s[wl] : 0;
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      ca[u] = lo[u] + lane < hi[u] ? __ldg(ci + lo[u] + lane) : -1;
+      cb[u] = lo[u] + 32 + lane < hi[u] ? __ldg(ci + lo[u] + 32 + lane) : -1;
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const uint32_t rofs = (uint32_t)((wb + 4 * u) * V);
+      sd_store1<V>(d, tt, rofs, lo[u] + lane, ca[u], c0, vec);
+      sd_store1<V>(d, tt, rofs, lo[u] + 32 + lane, cb[u], c0, vec);
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {  // windows with more than 64 vectors in the tile (dense ones)
+      const uint32_t rofs = (uint32_t)((wb + 4 * u) * V);
+      for (int e0 = lo[u] + 64; e0 < hi[u]; e0 += 64) {
+        const int e1 = e0 + lane, e2 = e0 + 32 + lane;
+        const int c1 = e1 < hi[u] ? __ldg(ci + e1) : -1;
+        const int c2 = e2 < hi[u] ? __ldg(ci + e2) : -1;
+        sd_store1<V>(d, tt, rofs, e1, c1, c0, vec);
+        sd_store1<V>(d, tt, rofs, e2, c2, c0, vec);
+      }
+    }
+  }
+}
+
+__global__ void __launch_bounds__(kSdThreads, kSdCtasPerSm) sddmm_dense_kernel(const __grid_constant__ SdBatch b) {
+  extern __shared__ uint8_t smem_raw[];
+  __shared__ __align__(8) uint64_t full_bar[kSdStages], empty_bar[kSdStages], done_bar;
+  __shared__ uint32_t tmem_base_sh;
+  __shared__ int32_t lo_s[128], hi_s[128];  // per window: its vectors in the tile's column range
+  const int64_t u = blockIdx.x;
+  const int p = first_problem(b.first_unit, b.count, u);
+  const SdDesc& d = b.d[p];
+  const int loc = (int)(u - b.first_unit[p]);  // < 2^31: units = ceil(M/128) * ceil(N/128), both < 2^24
+  const int n_ct = (int)d.n_ct;
+  const int rb = loc / n_ct, ct = loc - rb * n_ct;
+  if (!sddmm_rb_dense(d.row_ptr, d.W, d.V, rb, d.N)) return;  // CTA-uniform: the gather kernel's block
+
+  const uint32_t smem = (smem_u32(smem_raw) + 1023u) & ~1023u;
+  const int warp = threadIdx.x >> 5, lane = lane_id();
+  const int64_t w0 = rb * (128 / d.V);
+  const int nwin = (int)((w0 + 128 / d.V < d.W ? w0 + 128 / d.V : d.W) - w0);
   if (threadIdx.x == 0) {
     for (int s = 0; s < kSdStages; ++s) {
       tc::mbar_init(smem_u32(&full_bar[s]), 1);
       tc::mbar_init(smem_u32(&empty_bar[s]), 1);
     }
-    for (int a = 0; a < 2; ++a) {
-      tc::mbar_init(smem_u32(&tfull_bar[a]), 1);
-      tc::mbar_init(smem_u32(&tempty_bar[a]), 8);  // one arrive per epilogue warp
-    }
-    tc::mbar_init(smem_u32(&afull_bar), 1);
-    tc::mbar_init(smem_u32(&aempty_bar), 1);
+    tc::mbar_init(smem_u32(&done_bar), 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  if (warp == 1) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 64;" ::"r"(
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 128;" ::"r"(
         smem_u32(&tmem_base_sh)));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
   }
@@ -134,186 +240,172 @@ __global__ void __launch_bounds__(kSdThreads, 1) sddmm_dense_kernel(const __grid
   __syncthreads();
   tc::fence_after();
   const uint32_t tmem = tmem_base_sh;
+  const int KB = (int)ceil_div64(d.K, 64);
+  const int r0 = (int)(rb * 128), c0 = (int)(ct * 128);
 
-  UnitIt it{0};
   if (warp == 0) {
-    // ================================ TMA producer ================================
-    uint32_t s = 0, ph = 0, au = 0;
-    for (int64_t u = blockIdx.x; u < total; u += gridDim.x) {
-      int64_t rb, ct0, ct1;
-      it.locate(b, u, rb, ct0, ct1);
-      const SdDesc& d = b.d[it.p];
-      if (!sd_unit_dense(d, rb)) continue;
-      const int KB = (int)ceil_div64(d.K, 64);
-      // the unit's first kSdStages Bt stages go out while the previous unit's MMAs finish;
-      // its A tiles as soon as those MMAs released the resident A buffer
-      const int64_t nslots = (ct1 - ct0) * KB;
-      int64_t j = 0;
-      auto load_a = [&]() {
-        tc::mbar_wait(smem_u32(&aempty_bar), (au & 1) ^ 1);
-        if (lane == 0) {
-          tc::mbar_expect_tx(smem_u32(&afull_bar), KB * kATile);
-          for (int kb = 0; kb < KB; ++kb)
-            tc::tma_load_2d(s_ares + kb * kATile, &d.tmA, kb * 64, (int)(rb * kSdRows), smem_u32(&afull_bar));
-        }
-        __syncwarp();
-        ++au;
-      };
-      for (int64_t ct = ct0; ct < ct1; ++ct) {
-        for (int kb = 0; kb < KB; ++kb, ++j) {
-          if (j == (nslots - 1 < kSdStages ? nslots - 1 : kSdStages)) load_a();
-          tc::mbar_wait(smem_u32(&empty_bar[s]), ph ^ 1);
-          if (lane == 0) {
-            tc::mbar_expect_tx(smem_u32(&full_bar[s]), kBtTile);
-            tc::tma_load_2d(s_stage + s * kBtTile, &d.tmBt, kb * 64, (int)(ct * 128), smem_u32(&full_bar[s]));
-          }
-          __syncwarp();
-          if (++s == kSdStages) { s = 0; ph ^= 1; }
-        }
+    // ---- TMA producer: slab kb -> stage kb & 1 (Bt slab, then A slab)
+    if (lane == 0) {
+      for (int kb = 0; kb < KB; ++kb) {
+        const int s = kb & 1;
+        if (kb >= 2) tc::mbar_wait(smem_u32(&empty_bar[s]), ((kb >> 1) - 1) & 1);
+        const uint32_t st = smem + s * kSdStage;
+        tc::mbar_expect_tx(smem_u32(&full_bar[s]), kSdStage);
+        tc::tma_load_2d(st, &d.tmBt, kb * 64, c0, smem_u32(&full_bar[s]));
+        tc::tma_load_2d(st + kSdSlab, &d.tmA, kb * 64, r0, smem_u32(&full_bar[s]));
       }
     }
+    __syncwarp();
   } else if (warp == 1) {
-    // ================================ MMA issuer ================================
-    uint32_t s = 0, ph = 0, au = 0, tile = 0;
-    for (int64_t u = blockIdx.x; u < total; u += gridDim.x) {
-      int64_t rb, ct0, ct1;
-      it.locate(b, u, rb, ct0, ct1);
-      const SdDesc& d = b.d[it.p];
-      if (!sd_unit_dense(d, rb)) continue;
-      const int KB = (int)ceil_div64(d.K, 64);
-      tc::mbar_wait(smem_u32(&afull_bar), au & 1);
-      tc::fence_after();
-      for (int64_t ct = ct0; ct < ct1; ++ct) {
-        const uint32_t acc = tile & 1;
-        tc::mbar_wait(smem_u32(&tempty_bar[acc]), ((tile >> 1) & 1) ^ 1);
+    // ---- MMA issuer
+    if (lane == 0) {
+      for (int kb = 0; kb < KB; ++kb) {
+        const int s = kb & 1;
+        tc::mbar_wait(smem_u32(&full_bar[s]), (kb >> 1) & 1);
         tc::fence_after();
-        for (int kb = 0; kb < KB; ++kb) {
-          tc::mbar_wait(smem_u32(&full_bar[s]), ph);
-          tc::fence_after();
-          if (lane == 0) {
-            const uint32_t st = s_stage + s * kBtTile;
-            const uint32_t at = s_ares + kb * kATile;
+        const uint32_t st = smem + s * kSdStage;
 #pragma unroll
-            for (int k = 0; k < 4; ++k)
-              tc::mma(tmem + acc * kSdRows, tc::sdesc(st + 32 * k, 16, 1024), tc::sdesc(at + 32 * k, 16, 1024),
-                      kIdescSd, (kb > 0 || k > 0) ? 1u : 0u);
-            tc::commit(smem_u32(&empty_bar[s]));
-          }
-          __syncwarp();
-          if (++s == kSdStages) { s = 0; ph ^= 1; }
-        }
-        if (lane == 0) tc::commit(smem_u32(&tfull_bar[acc]));
-        __syncwarp();
-        ++tile;
+        for (int k = 0; k < 4; ++k)
+          tc::mma(tmem, tc::sdesc(st + 32 * k, 16, 1024), tc::sdesc(st + kSdSlab + 32 * k, 16, 1024), kIdescSd,
+                  (kb > 0 || k > 0) ? 1u : 0u);
+        tc::commit(smem_u32(&empty_bar[s]));
       }
-      if (lane == 0) tc::commit(smem_u32(&aempty_bar));
-      __syncwarp();
-      ++au;
+      tc::commit(smem_u32(&done_bar));
     }
+    __syncwarp();
   } else {
-    // ================================ epilogue ================================
-    const int et = threadIdx.x - 64;   // 0..255
-    const int q = warp & 3;            // TMEM lane quarter (tcgen05.ld restriction: warp % 4)
-    const int h = (warp - 2) >> 2;     // column half of the accumulator: rows 16h .. 16h+15
-    uint32_t tile = 0;
-    for (int64_t u = blockIdx.x; u < total; u += gridDim.x) {
-      int64_t rb, ct0, ct1;
-      it.locate(b, u, rb, ct0, ct1);
-      const SdDesc& d = b.d[it.p];
-      if (!sd_unit_dense(d, rb)) continue;
-      const int V = d.V;
-      const int64_t i0 = rb * kSdRows;
-      const int64_t w0 = i0 / V;
-      const int64_t w1 = (i0 + kSdRows) / V < d.W ? (i0 + kSdRows) / V : d.W;
-      const int nwin = (int)(w1 - w0);
-      // ---- drain every column tile of the range into Dh (fp16 RN; rows >= M are +0)
-      for (int64_t ct = ct0; ct < ct1; ++ct) {
-        const uint32_t acc = tile & 1;
-        tc::mbar_wait(smem_u32(&tfull_bar[acc]), (tile >> 1) & 1);
-        tc::fence_after();
-        uint32_t v[16];
-        asm volatile(
-            "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
-            : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
-              "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]),
-              "=r"(v[15])
-            : "r"(tmem + ((uint32_t)(32 * q) << 16) + acc * kSdRows + 16 * h));
-        tc::ld_wait();
-        tc::fence_before();
-        __syncwarp();
-        if (lane == 0) tc::mbar_arrive(smem_u32(&tempty_bar[acc]));
-        const int col = (int)(ct - ct0) * 128 + 32 * q + lane;  // column within the range
-#pragma unroll
-        for (int x = 0; x < 16; ++x) {
-          const int r = 16 * h + x;
-          const float f = (i0 + r < d.M) ? __uint_as_float(v[x]) : 0.f;
-          asm volatile("st.shared.u16 [%0], %1;" ::"r"(s_dh + (uint32_t)((r * (kCtPerUnit * 128) + col) * 2)),
-                       "h"(f_to_h(f))
-                       : "memory");
-        }
-        ++tile;
-      }
-      if (et <= nwin) wptr[et] = __ldg(d.row_ptr + w0 + et);
-      tc::named_bar(1, kSdEpi);  // Dh and wptr complete
-      // ---- one flat pass over the unit's stored vectors [P0, P1)
-      const int64_t P0 = wptr[0], P1 = wptr[nwin];
-      const int64_t cbeg = ct0 * 128, cend = ct1 * 128;
-      // groups of 4 entries at 16-byte aligned addresses of col_idx (any base alignment)
-      const int64_t off = (int64_t)((reinterpret_cast<uintptr_t>(d.col_idx) >> 2) & 3);
-      const int64_t Pa = ((P0 + off) & ~(int64_t)3) - off;
-      for (int64_t base = Pa + 4 * et; base < P1; base += 4 * kSdEpi) {
-        int c4[4];
-        if (base >= P0 && base + 3 < P1) {
-          const int4 t = __ldg(reinterpret_cast<const int4*>(d.col_idx + base));
-          c4[0] = t.x; c4[1] = t.y; c4[2] = t.z; c4[3] = t.w;
-        } else {
-#pragma unroll
-          for (int j = 0; j < 4; ++j) c4[j] = (base + j >= P0 && base + j < P1) ? __ldg(d.col_idx + base + j) : -1;
-        }
-        // window of the first entry (binary search), then advance
-        const int64_t pf = base < P0 ? P0 : base;
-        int lo = 0, hi = nwin - 1;
-        while (lo < hi) {
-          const int mid = (lo + hi + 1) >> 1;
-          if (wptr[mid] <= pf) lo = mid; else hi = mid - 1;
-        }
-        int wl = lo;
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-          const int64_t p = base + j;
-          if (p < P0 || p >= P1) continue;
-          while (wptr[wl + 1] <= p) ++wl;
-          const int64_t c = c4[j];
-          if (c < cbeg || c >= cend) continue;
-          const uint32_t a = s_dh + (uint32_t)(((int64_t)(wl * V) * (kCtPerUnit * 128) + (c - cbeg)) * 2);
-          uint16_t hv[8];
-#pragma unroll
-          for (int r = 0; r < 8; ++r) hv[r] = r < V ? lds16(a + (uint32_t)(r * kCtPerUnit * 128 * 2)) : (uint16_t)0;
-          uint16_t* dst = d.out + p * V;
-          if (d.out_vec) {
-            if (V == 8) *reinterpret_cast<uint4*>(dst) = make_uint4(pack_h2(hv[0], hv[1]), pack_h2(hv[2], hv[3]),
-                                                                   pack_h2(hv[4], hv[5]), pack_h2(hv[6], hv[7]));
-            else if (V == 4) *reinterpret_cast<uint2*>(dst) = make_uint2(pack_h2(hv[0], hv[1]), pack_h2(hv[2], hv[3]));
-            else *reinterpret_cast<uint32_t*>(dst) = pack_h2(hv[0], hv[1]);
-          } else {
-            for (int r = 0; r < V; ++r) dst[r] = hv[r];
-          }
-        }
-      }
-      tc::named_bar(1, kSdEpi);  // Dh / wptr reads done before the next unit's drain
+    // ---- warps 2-3, while the TMA / MMA run: per window (thread = window), its vectors with a
+    // column in [c0, c0 + 128) are the range [lo, hi) of its (ascending) col_idx
+    for (int i = threadIdx.x - 64; i < nwin; i += kSdThreads - 64) {
+      const int pb = __ldg(d.row_ptr + w0 + i), pe = __ldg(d.row_ptr + w0 + i + 1);
+      int lo, hi;
+      kary_lower_bound2(d.col_idx, pb, pe, c0, c0 + 128, lo, hi);
+      lo_s[i] = lo;
+      hi_s[i] = hi > lo ? hi : lo;
     }
   }
 
+  // ---- drain: thread = mask column c = TMEM lane 32 * warp + lane; Tt[c][r] fp16 over the ring
+  tc::mbar_wait(smem_u32(&done_bar), 0);
+  tc::fence_after();
+  const int c = 32 * warp + lane;
+  const uint32_t trow = smem + (uint32_t)c * 256;
+  const int64_t rows_valid = d.M - r0;  // rows >= M are stored as +0
+#pragma unroll 1
+  for (int j = 0; j < 4; ++j) {
+    uint32_t v[32];
+    tc::ld32(tmem + ((uint32_t)(32 * warp) << 16) + 32 * j, v);
+    tc::ld_wait();
+    uint32_t h[16];
+#pragma unroll
+    for (int x = 0; x < 16; ++x) {
+      const int r = 32 * j + 2 * x;
+      const float f0 = r < rows_valid ? __uint_as_float(v[2 * x]) : 0.f;
+      const float f1 = r + 1 < rows_valid ? __uint_as_float(v[2 * x + 1]) : 0.f;
+      h[x] = f2_to_h2(f0, f1);
+    }
+#pragma unroll
+    for (int m = 0; m < 4; ++m)
+      asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(trow + ((((uint32_t)(4 * j + m)) ^ (c & 15)) << 4)),
+                   "r"(h[4 * m]), "r"(h[4 * m + 1]), "r"(h[4 * m + 2]), "r"(h[4 * m + 3])
+                   : "memory");
+  }
   tc::fence_before();
-  __syncthreads();
-  if (warp == 1) {
+  __syncthreads();  // Tt complete, TMEM drained
+  if (warp == 0) {
     tc::fence_after();
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 64;" ::"r"(tmem));
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 128;" ::"r"(tmem));
+  }
+  switch (d.V) {
+    case 1: sd_store<1>(d, smem, lo_s, hi_s, nwin, c0, warp, lane); break;
+    case 2: sd_store<2>(d, smem, lo_s, hi_s, nwin, c0, warp, lane); break;
+    case 4: sd_store<4>(d, smem, lo_s, hi_s, nwin, c0, warp, lane); break;
+    default: sd_store<8>(d, smem, lo_s, hi_s, nwin, c0, warp, lane); break;
   }
 }
 
+static cudaError_t launch_sd(const SdBatch& b, cudaStream_t s) {
+  static std::once_flag once[64];
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev >= 0 && dev < 64)
+    std::call_once(once[dev], [] {
+      cudaFuncSetAttribute(sddmm_dense_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kSdSmem);
+    });
+  const int64_t units = b.first_unit[b.count];
+  if (units > 0) sddmm_dense_kernel<<<(unsigned)units, kSdThreads, kSdSmem, s>>>(b);
+  return cudaGetLastError();
+}
+
+}  // namespace dt
+
+// Problems the dense SDDMM path can take at all (the per-row-block choice is made on the
+// device): 0 < K with K % 8 == 0 (16-byte TMA row stride), 16-byte aligned A and Bt, row and
+// column counts that fit the int32 TMA coordinates.
+bool sddmm_dense_eligible(int64_t M, int64_t N, int64_t K, int V, const void* A, const void* Bt) {
+  return M > 0 && N > 0 && K > 0 && V >= 1 && V <= 8 && K % 8 == 0 &&
+         ((reinterpret_cast<uintptr_t>(A) & 15) == 0) && ((reinterpret_cast<uintptr_t>(Bt) & 15) == 0) &&
+         N < (int64_t(1) << 31) && M < (int64_t(1) << 31) && K < (int64_t(1) << 31) &&
+         ceil_div64(M, 128) * ceil_div64(N, 128) < (int64_t(1) << 31);
+}
+
+// Launches the dense-tile SDDMM over the eligible problems (units of row blocks the cost
+// model leaves to the gather kernel exit at once on the device).
+cudaError_t launch_sddmm_dense(int64_t count, const int64_t* M, const int64_t* N, const int64_t* K,
+                               const int* V, const int32_t* const* row_ptr, const int32_t* const* col_idx,
+                               const void* const* A, const void* const* Bt, void* const* out, int num_sms,
+                               cudaStream_t s) {
+  using namespace dt;
+  (void)num_sms;
+  SdBatch batch;
+  batch.count = 0;
+  batch.first_unit[0] = 0;
+  auto flush = [&]() -> cudaError_t {
+    if (batch.count == 0) return cudaSuccess;
+    const cudaError_t e = launch_sd(batch, s);
+    batch.count = 0;
+    batch.first_unit[0] = 0;
+    return e;
+  };
+  for (int64_t i = 0; i < count; ++i) {
+    if (!sddmm_dense_eligible(M[i], N[i], K[i], V[i], A[i], Bt[i])) continue;
+    if (batch.first_unit[batch.count] + ceil_div64(M[i], 128) * ceil_div64(N[i], 128) >= (int64_t(1) << 31)) {
+      const cudaError_t e = flush();  // one launch's grid stays below 2^31 CTAs
+      if (e != cudaSuccess) return e;
+    }
+    SdDesc& d = batch.d[batch.count];
+    if (!make_kmajor_map(&d.tmA, A[i], M[i], K[i], 128) || !make_kmajor_map(&d.tmBt, Bt[i], N[i], K[i], 128))
+      return cudaErrorInvalidValue;
+    d.M = M[i];
+    d.N = N[i];
+    d.K = K[i];
+    d.V = V[i];
+    d.W = ceil_div64(M[i], V[i]);
+    d.n_ct = ceil_div64(N[i], 128);
+    d.row_ptr = row_ptr[i];
+    d.col_idx = col_idx[i];
+    d.out = static_cast<uint16_t*>(out[i]);
+    d.out_vec = (reinterpret_cast<uintptr_t>(out[i]) & (uintptr_t)(2 * V[i] - 1)) == 0 ? 1 : 0;
+    batch.first_unit[batch.count + 1] = batch.first_unit[batch.count] + ceil_div64(M[i], 128) * d.n_ct;
+    ++batch.count;
+    if (batch.count == kMaxProb) {
+      const cudaError_t e = flush();
+      if (e != cudaSuccess) return e;
+    }
+  }
+  return flush();
+}
+
+}  // namespace vs
+#endif  // VS_SDDMM_DENSE_CF > 0
+
+#if VS_SPMM_DENSE_CF > 0  // opt-in build only (dense_select.cuh)
+namespace vs {
+namespace dt {
+
 // ================================================================================ SpMM
 constexpr int kSpRows = 32;            // A / C rows per unit (MMA N)
+constexpr int kATile = kSpRows * 128;  // 32 rows x 64 k fp16 (4 KB)
 constexpr int kSpThreads = 320;        // 10 warps
 constexpr int kSpEpi = 256;            // decode / epilogue threads (warps 2-9)
 constexpr int kSpKbMax = 32;           // K <= 2048: the decoded A tile stays resident
@@ -340,7 +432,8 @@ struct SpBatch {
 };
 
 __device__ __forceinline__ bool sp_unit_dense(const SpDesc& d, int64_t rb32) {
-  return rb_is_dense(d.row_ptr, d.W, d.V, rb32 / (kDenseRows / kSpRows), ceil_div64(d.K, 64) * 64);
+  return rb_is_dense(d.row_ptr, d.W, d.V, rb32 / (kDenseRows / kSpRows), ceil_div64(d.K, 64) * 64,
+                     (int64_t)VS_SPMM_DENSE_CF);
 }
 
 // byte offset of element (row, k) in the decoded K-major 128-byte-swizzled A tile
@@ -564,46 +657,6 @@ __global__ void __launch_bounds__(kSpThreads, 1) spmm_dense_kernel(const __grid_
   }
 }
 
-// ------------------------------------------------------------------------------ host side
-
-static PFN_cuTensorMapEncodeTiled_v12000 tmap_encoder() {
-  static PFN_cuTensorMapEncodeTiled_v12000 fn = [] {
-    void* p = nullptr;
-    cudaDriverEntryPointQueryResult q;
-    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) != cudaSuccess ||
-        q != cudaDriverEntryPointSuccess)
-      p = nullptr;
-    return reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
-  }();
-  return fn;
-}
-
-// K-major fp16 [rows x K] operand, box {64, box_rows}, 128-byte swizzle, OOB -> zero
-static bool make_kmajor_map(CUtensorMap* m, const void* base, int64_t rows, int64_t K, int box_rows) {
-  auto enc = tmap_encoder();
-  if (enc == nullptr) return false;
-  cuuint64_t gdim[2] = {(cuuint64_t)K, (cuuint64_t)rows};
-  cuuint64_t gstride[1] = {(cuuint64_t)K * 2};
-  cuuint32_t box[2] = {64, (cuuint32_t)box_rows};
-  cuuint32_t estr[2] = {1, 1};
-  return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, const_cast<void*>(base), gdim, gstride, box, estr,
-             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
-             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
-}
-
-// MN-major fp16 B [K x N] (N contiguous), box {64 n, 64 k}, 128-byte swizzle, OOB -> zero
-static bool make_mnmajor_map(CUtensorMap* m, const void* base, int64_t K, int64_t N) {
-  auto enc = tmap_encoder();
-  if (enc == nullptr) return false;
-  cuuint64_t gdim[2] = {(cuuint64_t)N, (cuuint64_t)K};
-  cuuint64_t gstride[1] = {(cuuint64_t)N * 2};
-  cuuint32_t box[2] = {64, 64};
-  cuuint32_t estr[2] = {1, 1};
-  return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, const_cast<void*>(base), gdim, gstride, box, estr,
-             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
-             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
-}
-
 static cudaError_t launch_sp(const SpBatch& b, int num_sms, cudaStream_t s) {
   static std::once_flag once[64];
   int dev = 0;
@@ -618,75 +671,7 @@ static cudaError_t launch_sp(const SpBatch& b, int num_sms, cudaStream_t s) {
   return cudaGetLastError();
 }
 
-static cudaError_t launch_sd(const SdBatch& b, int num_sms, cudaStream_t s) {
-  static std::once_flag once[64];
-  int dev = 0;
-  cudaGetDevice(&dev);
-  if (dev >= 0 && dev < 64)
-    std::call_once(once[dev], [] {
-      cudaFuncSetAttribute(sddmm_dense_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kSdSmem);
-    });
-  const int64_t units = b.first_unit[b.count];
-  const int grid = (int)std::min<int64_t>(num_sms, units);
-  if (grid > 0) sddmm_dense_kernel<<<grid, kSdThreads, kSdSmem, s>>>(b);
-  return cudaGetLastError();
-}
-
 }  // namespace dt
-
-// Problems the dense SDDMM path can take at all (the per-row-block choice is made on the
-// device): V >= 2, 0 < K <= 256 with K % 8 == 0 (A tiles resident, 16-byte TMA row stride),
-// 16-byte aligned A and Bt.
-bool sddmm_dense_eligible(int64_t M, int64_t N, int64_t K, int V, const void* A, const void* Bt) {
-  return M > 0 && N > 0 && K > 0 && K <= 64 * dt::kSdKbMax && V >= 2 && K % 8 == 0 &&
-         ((reinterpret_cast<uintptr_t>(A) & 15) == 0) && ((reinterpret_cast<uintptr_t>(Bt) & 15) == 0) &&
-         N < (int64_t(1) << 31) && M < (int64_t(1) << 31);
-}
-
-// Launches the dense-tile SDDMM over the eligible problems (units of row blocks the cost
-// model leaves to the gather kernel are skipped on the device).
-cudaError_t launch_sddmm_dense(int64_t count, const int64_t* M, const int64_t* N, const int64_t* K,
-                               const int* V, const int32_t* const* row_ptr, const int32_t* const* col_idx,
-                               const void* const* A, const void* const* Bt, void* const* out, int num_sms,
-                               cudaStream_t s) {
-  using namespace dt;
-  SdBatch batch;
-  batch.count = 0;
-  batch.first_unit[0] = 0;
-  auto flush = [&]() -> cudaError_t {
-    if (batch.count == 0) return cudaSuccess;
-    const cudaError_t e = launch_sd(batch, num_sms, s);
-    batch.count = 0;
-    batch.first_unit[0] = 0;
-    return e;
-  };
-  for (int64_t i = 0; i < count; ++i) {
-    if (!sddmm_dense_eligible(M[i], N[i], K[i], V[i], A[i], Bt[i])) continue;
-    SdDesc& d = batch.d[batch.count];
-    if (!make_kmajor_map(&d.tmA, A[i], M[i], K[i], kSdRows) ||
-        !make_kmajor_map(&d.tmBt, Bt[i], N[i], K[i], 128))
-      return cudaErrorInvalidValue;
-    d.M = M[i];
-    d.N = N[i];
-    d.K = K[i];
-    d.V = V[i];
-    d.W = ceil_div64(M[i], V[i]);
-    d.n_cr = ceil_div64(ceil_div64(N[i], 128), kCtPerUnit);
-    d.n_rb = ceil_div64(M[i], kSdRows);
-    d.row_ptr = row_ptr[i];
-    d.col_idx = col_idx[i];
-    d.out = static_cast<uint16_t*>(out[i]);
-    d.nnz_total = 0;
-    d.out_vec = (reinterpret_cast<uintptr_t>(out[i]) & (uintptr_t)(2 * V[i] - 1)) == 0 ? 1 : 0;
-    batch.first_unit[batch.count + 1] = batch.first_unit[batch.count] + d.n_rb * d.n_cr;
-    ++batch.count;
-    if (batch.count == kMaxProb) {
-      const cudaError_t e = flush();
-      if (e != cudaSuccess) return e;
-    }
-  }
-  return flush();
-}
 
 // Problems the dense SpMM path can take at all (the per-row-block choice is made on the
 // device): V >= 2, 0 < K <= 2048 (decoded A tile resident), N % 8 == 0 and 16-byte aligned B
@@ -741,4 +726,50 @@ cudaError_t launch_spmm_dense(int64_t count, const int64_t* M, const int64_t* K,
 }
 
 }  // namespace vs
-#endif  // VS_DENSE_CF > 0
+#endif  // VS_SPMM_DENSE_CF > 0
+
+#if VS_SDDMM_DENSE_CF > 0 || VS_SPMM_DENSE_CF > 0
+namespace vs {
+namespace dt {
+
+static PFN_cuTensorMapEncodeTiled_v12000 tmap_encoder() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = [] {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+      p = nullptr;
+    return reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+  }();
+  return fn;
+}
+
+// K-major fp16 [rows x K] operand, box {64, box_rows}, 128-byte swizzle, OOB -> zero
+static bool make_kmajor_map(CUtensorMap* m, const void* base, int64_t rows, int64_t K, int box_rows) {
+  auto enc = tmap_encoder();
+  if (enc == nullptr) return false;
+  cuuint64_t gdim[2] = {(cuuint64_t)K, (cuuint64_t)rows};
+  cuuint64_t gstride[1] = {(cuuint64_t)K * 2};
+  cuuint32_t box[2] = {64, (cuuint32_t)box_rows};
+  cuuint32_t estr[2] = {1, 1};
+  return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, const_cast<void*>(base), gdim, gstride, box, estr,
+             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+// MN-major fp16 B [K x N] (N contiguous), box {64 n, 64 k}, 128-byte swizzle, OOB -> zero
+static bool make_mnmajor_map(CUtensorMap* m, const void* base, int64_t K, int64_t N) {
+  auto enc = tmap_encoder();
+  if (enc == nullptr) return false;
+  cuuint64_t gdim[2] = {(cuuint64_t)N, (cuuint64_t)K};
+  cuuint64_t gstride[1] = {(cuuint64_t)N * 2};
+  cuuint32_t box[2] = {64, 64};
+  cuuint32_t estr[2] = {1, 1};
+  return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, const_cast<void*>(base), gdim, gstride, box, estr,
+             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+}  // namespace dt
+}  // namespace vs
+#endif

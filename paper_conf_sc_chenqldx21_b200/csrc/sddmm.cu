@@ -260,18 +260,21 @@ __device__ __forceinline__ void sddmm_window_any(int64_t M, int64_t K,
   }
 }
 
-// Row blocks the dense-tile kernel takes (dense_select.cuh) are skipped here: the dense kernel
-// computes every stored vector of them, in any col_idx order.  Returns the q to use for the
-// item, or 0 to skip it.
+// Row blocks the dense-tile kernel takes (dense_select.cuh) are skipped here, except windows
+// whose col_idx is not strictly ascending: the dense kernel finds a window's vectors of each
+// column tile by a search that assumes ascending order, so such a window (rare: the encoder
+// emits ascending windows) is computed here in full by the warp of its first item, after the
+// dense kernel (same stream, launched first), whose writes for it this one overwrites.
+// Returns the q to use for the item, or 0 to skip it.
 __device__ __forceinline__ int64_t sddmm_gather_q(bool dense_ok, int64_t N, int V, int64_t W,
                                                   const int32_t* __restrict__ row_ptr,
                                                   const int32_t* __restrict__ col_idx, int64_t w,
                                                   int64_t j0, int64_t q) {
-  (void)col_idx;
-  (void)j0;
   if (!dense_ok) return q;
   const int64_t rb = (w * V) / kDenseRows;
-  return rb_is_dense(row_ptr, W, V, rb, ceil_div64(N, 128) * 128) ? 0 : q;
+  if (!sddmm_rb_dense(row_ptr, W, V, rb, N)) return q;
+  if (j0 != 0) return 0;
+  return window_sorted(col_idx, __ldg(row_ptr + w), __ldg(row_ptr + w + 1)) ? 0 : 1;
 }
 
 // Work items of one problem: W windows x q warps per window (warp j of window w takes the
@@ -452,7 +455,7 @@ static void launch_sddmm_one(int64_t M, int64_t K, const int32_t* row_ptr, const
                                                                    N, dense_ok);
 }
 
-#if VS_DENSE_CF > 0
+#if VS_SDDMM_DENSE_CF > 0
 bool sddmm_dense_eligible(int64_t M, int64_t N, int64_t K, int V, const void* A, const void* Bt);
 cudaError_t launch_sddmm_dense(int64_t count, const int64_t* M, const int64_t* N, const int64_t* K,
                                const int* V, const int32_t* const* row_ptr, const int32_t* const* col_idx,
@@ -473,6 +476,15 @@ static cudaError_t launch_sddmm_v(int64_t M, int64_t N, int64_t K, const int32_t
                                   uint16_t* out, bool vec, int num_sms, cudaStream_t s) {
   const int V_ = V;
   const bool dok = sddmm_dense_eligible(M, N, K, V, A, Bt);
+  if (dok) {
+    // dense row blocks first (short non-persistent CTAs); the persistent gather grid then
+    // takes the remaining row blocks
+    const void* a = A;
+    const void* bt = Bt;
+    void* o = out;
+    const cudaError_t de = launch_sddmm_dense(1, &M, &N, &K, &V_, &row_ptr, &col_idx, &a, &bt, &o, num_sms, s);
+    if (de != cudaSuccess) return de;
+  }
   switch ((vec ? 8 : 0) + sddmm_variant(K, vec)) {
     case 8 + 2: launch_sddmm_one<V, true, 1, false>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok); break;
     case 8 + 3: launch_sddmm_one<V, true, 1, true>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok); break;
@@ -482,12 +494,7 @@ static cudaError_t launch_sddmm_v(int64_t M, int64_t N, int64_t K, const int32_t
     case 3: launch_sddmm_one<V, false, 1, true>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok); break;
     default: launch_sddmm_one<V, false, 1, false>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok); break;
   }
-  cudaError_t e = cudaGetLastError();
-  if (e != cudaSuccess || !dok) return e;
-  const void* a = A;
-  const void* bt = Bt;
-  void* o = out;
-  return launch_sddmm_dense(1, &M, &N, &K, &V_, &row_ptr, &col_idx, &a, &bt, &o, num_sms, s);
+  return cudaGetLastError();
 }
 
 template <int V, bool VEC, int KC, bool ARES, bool FAST = false>
@@ -555,10 +562,12 @@ cudaError_t launch_sddmm_batched(int64_t count, const int64_t* M, const int64_t*
                                  const void* const* Bt, void* const* out, int num_sms,
                                  cudaStream_t s) {
   if (!sddmm_tc_on()) {
-    // gather kernels (skipping the dense row blocks), then the dense-tile kernel (taking them)
-    const cudaError_t e = launch_sddmm_mma_batched(count, M, N, K, V, row_ptr, col_idx, A, Bt, out, num_sms, s);
-    if (e != cudaSuccess || VS_DENSE_CF == 0) return e;
-    return launch_sddmm_dense(count, M, N, K, V, row_ptr, col_idx, A, Bt, out, num_sms, s);
+    // the dense-tile kernel (taking the dense row blocks), then the gather kernels (skipping them)
+    if (VS_SDDMM_DENSE_CF != 0) {
+      const cudaError_t e = launch_sddmm_dense(count, M, N, K, V, row_ptr, col_idx, A, Bt, out, num_sms, s);
+      if (e != cudaSuccess) return e;
+    }
+    return launch_sddmm_mma_batched(count, M, N, K, V, row_ptr, col_idx, A, Bt, out, num_sms, s);
   }
   std::vector<int64_t> sel[2];
   for (int64_t i = 0; i < count; ++i) sel[sddmm_tc_eligible(K[i], A[i], Bt[i], out[i]) ? 1 : 0].push_back(i);

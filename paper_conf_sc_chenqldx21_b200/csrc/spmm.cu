@@ -85,7 +85,7 @@ __device__ __forceinline__ bool spmm_skip_window(int64_t dkp, int V, int64_t W, 
                                                  const int32_t* __restrict__ row_ptr,
                                                  const int32_t* __restrict__ col_idx, int pb, int pe) {
   if (dkp == 0 || w >= W) return false;
-  if (!rb_is_dense(row_ptr, W, V, (w * V) / kDenseRows, dkp)) return false;
+  if (!rb_is_dense(row_ptr, W, V, (w * V) / kDenseRows, dkp, (int64_t)VS_SPMM_DENSE_CF)) return false;
   return window_sorted(col_idx, pb, pe);
 }
 
@@ -840,7 +840,7 @@ static int64_t spmm_blocks(const SpmmKernels& k, const SpmmCfg& c, int64_t M, in
   return ceil_div64(N, 64 * c.NC) * nwg;
 }
 
-#if VS_DENSE_CF > 0
+#if VS_SPMM_DENSE_CF > 0
 bool spmm_dense_eligible(int64_t M, int64_t K, int64_t N, int V, const void* vals, const void* B);
 cudaError_t launch_spmm_dense(int64_t count, const int64_t* M, const int64_t* K, const int64_t* N,
                               const int* V, const int32_t* const* row_ptr, const int32_t* const* col_idx,
@@ -1032,7 +1032,7 @@ cudaError_t launch_spmm_batched(int64_t count, const int64_t* M, const int64_t* 
     if (e != cudaSuccess) return e;
   }
   // the dense-tile kernel takes the row blocks the gather launches above skipped
-  if (VS_DENSE_CF == 0) return cudaSuccess;
+  if (VS_SPMM_DENSE_CF == 0) return cudaSuccess;
   std::vector<void* const*> dsts(count);
   std::vector<int> ones(count, 1);
   for (int64_t i = 0; i < count; ++i) dsts[i] = &C[i];
