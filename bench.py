@@ -196,7 +196,9 @@ def count_launches(bufs):
     """Kernel launches of one batched step, by the library's grouping rules: encode groups by
     V (3 kernels per group of <= 128 problems: count, scan, compact); SpMM (cp.async path,
     spmm.cu spmm_config) by (V, panel width NC = 1 for N <= 64 else 2, SPLIT from K); SDDMM
-    (sddmm.cu sddmm_variant) by V (one kernel serves both K-block variants)."""
+    (sddmm.cu sddmm_variant) by V (one kernel serves both K-block variants), plus the dense-tile
+    SDDMM kernel (dense_tile.cu: problems with inner dimension >= VS_SDDMM_DENSE_KMIN = 256,
+    32 problems per launch) before each V group's gather launch."""
     import math as _m
     from collections import Counter
     def split(K):
@@ -205,9 +207,10 @@ def count_launches(bufs):
     enc = Counter(b.p.V for b in bufs)
     sp = Counter((b.p.V, 1 if b.p.N <= 64 else 2, split(b.p.K)) for b in bufs)
     sd = Counter(b.p.V for b in bufs)  # one mixed-K kernel per V (sddmm_window_any)
+    sd_dense = Counter(b.p.V for b in bufs if b.p.N >= 256 and b.p.N % 8 == 0)  # SDDMM inner = N
     per = {"encode": sum(3 * _m.ceil(n / 128) for n in enc.values()),
            "spmm": sum(_m.ceil(n / 128) for n in sp.values()),
-           "sddmm": sum(_m.ceil(n / 128) for n in sd.values())}
+           "sddmm": sum(_m.ceil(n / 128) for n in sd.values()) + sum(_m.ceil(n / 32) for n in sd_dense.values())}
     return {"per_class": per, "total": sum(per.values())}
 
 
@@ -638,6 +641,10 @@ def run_ours(args):
     torch.cuda.synchronize()
     clk = clocks.stop()
 
+    # per-class device times on stderr before the gate (kernel variants under study keep their
+    # timings even when the gate rejects their outputs)
+    print("classes_ms " + json.dumps({k: round(sum(v) / args.steps, 4) for k, v in per_class.items()}) +
+          " step_ms %.4f" % (sum(step_ms) / args.steps), file=sys.stderr)
     # oracle gate on the timed launch configuration's outputs (raises on failure)
     with torch.cuda.stream(stream):
         g_step.replay()

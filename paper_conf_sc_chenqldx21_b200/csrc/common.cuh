@@ -225,6 +225,14 @@ __device__ __forceinline__ int first_problem(const int64_t* first, int count, in
   return lo;
 }
 
+// Programmatic dependent launch (griddepcontrol): let the next kernel of the stream start while
+// this one runs / wait until the previous kernel of the stream has completed and its writes are
+// visible.  Both are no-ops in a kernel launched without the PDL attribute.
+__device__ __forceinline__ void pdl_launch_dependents() {
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+__device__ __forceinline__ void pdl_wait_prior() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+
 __host__ __device__ __forceinline__ int64_t ceil_div64(int64_t a, int64_t b) {
   return (a + b - 1) / b;
 }

@@ -20,11 +20,21 @@
 
 // Build-time cost-model constants (flop per gathered byte), one per op; 0 = the dense-tile
 // kernel of that op is not built and never launched (every row block stays with the gather
-// kernel).  VS_SDDMM_DENSE_CF: the 128 x 128-unit SDDMM kernel (dense_tile.cu), tuned on B200
-// over the DLMC batch.  VS_SPMM_DENSE_CF: the dense-tile SpMM, measured slower
-// than the gather kernel at DLMC sizes (profiles/r02_dense_tile.md) -> 0 in the shipped library.
+// kernel).  VS_SDDMM_DENSE_CF / VS_SDDMM_DENSE_KMIN: the 128 x 128-unit SDDMM kernel
+// (dense_tile.cu) takes the 128-row blocks with nnz_v(rb) * 32 > 128 * Lc (stored density
+// above V/32) of problems with inner dimension K >= 256.  Tuned on B200 (DESIGN.md §7.8,
+// profiles/r03_dense_sddmm.md): over the DLMC batch the step is 0.900 -> 0.830 ms, while the
+// single calls keep the per-cell crossovers with cuBLAS Hgemm (a dense-tile launch adds a
+// ~1-2 us floor to a single call; rules taking smaller K or lower density made the batch
+// faster, 0.816 ms, but single calls up to 1.5x slower).  VS_SPMM_DENSE_CF: the dense-tile
+// SpMM, measured slower than the gather kernel at DLMC sizes (profiles/r02_dense_tile.md) -> 0.
 #ifndef VS_SDDMM_DENSE_CF
-#define VS_SDDMM_DENSE_CF 64
+#define VS_SDDMM_DENSE_CF 32
+#endif
+// smallest inner dimension K the dense-tile SDDMM takes (a shape rule: every shard of a problem
+// decides alike)
+#ifndef VS_SDDMM_DENSE_KMIN
+#define VS_SDDMM_DENSE_KMIN 256
 #endif
 #ifndef VS_SPMM_DENSE_CF
 #define VS_SPMM_DENSE_CF 0

@@ -264,8 +264,9 @@ __device__ __forceinline__ void sddmm_window_any(int64_t M, int64_t K,
 // whose col_idx is not strictly ascending: the dense kernel finds a window's vectors of each
 // column tile by a search that assumes ascending order, so such a window (rare: the encoder
 // emits ascending windows) is computed here in full by the warp of its first item, after the
-// dense kernel (same stream, launched first), whose writes for it this one overwrites.
-// Returns the q to use for the item, or 0 to skip it.
+// dense kernel has completed (this kernel follows it on the stream, overlapped by programmatic
+// dependent launch: the warp waits for it with griddepcontrol.wait), overwriting its writes.
+// Returns the q to use for the item, 0 to skip it, or -1 for such a window.
 __device__ __forceinline__ int64_t sddmm_gather_q(bool dense_ok, int64_t N, int V, int64_t W,
                                                   const int32_t* __restrict__ row_ptr,
                                                   const int32_t* __restrict__ col_idx, int64_t w,
@@ -274,7 +275,7 @@ __device__ __forceinline__ int64_t sddmm_gather_q(bool dense_ok, int64_t N, int 
   const int64_t rb = (w * V) / kDenseRows;
   if (!sddmm_rb_dense(row_ptr, W, V, rb, N)) return q;
   if (j0 != 0) return 0;
-  return window_sorted(col_idx, __ldg(row_ptr + w), __ldg(row_ptr + w + 1)) ? 0 : 1;
+  return window_sorted(col_idx, __ldg(row_ptr + w), __ldg(row_ptr + w + 1)) ? 0 : -1;
 }
 
 // Work items of one problem: W windows x q warps per window (warp j of window w takes the
@@ -299,12 +300,17 @@ __global__ void __launch_bounds__(kSddmmWarps * 32, VS_SDDMM_MINB)
   const int64_t items = W * q;
   for (int64_t it = gw; it < items; it += n_warps) {
     const int64_t w = it / q;
-    const int64_t qq = sddmm_gather_q(dense_ok, N, V, W, row_ptr, col_idx, w, it - w * q, q);
+    int64_t qq = sddmm_gather_q(dense_ok, N, V, W, row_ptr, col_idx, w, it - w * q, q);
     if (qq == 0) continue;
+    if (qq < 0) {  // non-ascending window of a dense row block: after the dense kernel, in full
+      pdl_wait_prior();
+      qq = 1;
+    }
     // single-problem kernel: FAST mode 1 (measured best per call, profiles/r02_sddmm_variants.md)
     sddmm_window_any<V, VEC, KC, ARES, FAST ? 1 : 0>(M, K, row_ptr, col_idx, A, Bt, out, out4, w,
                                                      qq == q ? it - w * q : 0, qq, pair);
   }
+  pdl_wait_prior();  // completes only after a dense-tile kernel it overlaps (no-op otherwise)
 }
 
 // Batched launch over up to kSddmmMaxBatch problems of one configuration: every problem
@@ -383,13 +389,18 @@ __global__ void __launch_bounds__(kSddmmWarps * 32, VS_SDDMM_MINB)
     const int64_t q = qs[p];
     const int64_t loc = it - pre[p];
     const int64_t w = loc / q;
-    const int64_t qq = sddmm_gather_q(d.dense_ok != 0, d.N, V, d.W, d.row_ptr, d.col_idx, w, loc - w * q, q);
+    int64_t qq = sddmm_gather_q(d.dense_ok != 0, d.N, V, d.W, d.row_ptr, d.col_idx, w, loc - w * q, q);
     if (qq == 0) continue;
+    if (qq < 0) {  // non-ascending window of a dense row block: after the dense kernel, in full
+      pdl_wait_prior();
+      qq = 1;
+    }
     // batched kernel: FAST mode 2 (full chunks only: many short windows in a batch)
     sddmm_window_any<V, VEC, KC, ARES, FAST ? 2 : 0>(d.M, d.K, d.row_ptr, d.col_idx, d.A, d.Bt, d.out,
                                                      d.out4 != 0, w, qq == q ? loc - w * q : 0, qq,
                                                      b.pair != 0);
   }
+  pdl_wait_prior();  // completes only after a dense-tile kernel it overlaps (no-op otherwise)
 }
 
 // Persistent grid: as many CTAs as can be resident at once (occupancy queried once per
@@ -443,6 +454,29 @@ static int sddmm_batched_ctas_per_sm() {
   return n;
 }
 
+// Launch, overlapped with the dense-tile kernel just launched on the stream (pdl = true:
+// programmatic dependent launch; the gather kernel's blocks start while it runs and complete
+// after it, see sddmm_gather_q) or plainly.
+template <typename... KArgs, typename... Args>
+static void launch_maybe_pdl(bool pdl, void (*kern)(KArgs...), dim3 grid, dim3 block, cudaStream_t s,
+                             Args... args) {
+  if (!pdl) {
+    kern<<<grid, block, 0, s>>>(args...);
+    return;
+  }
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = 0;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  (void)cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...);
+}
+
 template <int V, bool VEC, int KC, bool ARES, bool FAST = false>
 static void launch_sddmm_one(int64_t M, int64_t K, const int32_t* row_ptr, const int32_t* col_idx,
                              const uint16_t* A, const uint16_t* Bt, uint16_t* out, int num_sms,
@@ -450,9 +484,8 @@ static void launch_sddmm_one(int64_t M, int64_t K, const int32_t* row_ptr, const
   const int64_t W = ceil_div64(M, V);
   const bool out4 = (reinterpret_cast<uintptr_t>(out) & 3) == 0;
   dim3 grid((unsigned)(num_sms * sddmm_ctas_per_sm<V, VEC, KC, ARES, FAST>()));
-  sddmm_kernel<V, VEC, KC, ARES, FAST><<<grid, kSddmmWarps * 32, 0, s>>>(M, K, W, row_ptr, col_idx, A,
-                                                                   Bt, out, out4, sddmm_pair_on(),
-                                                                   N, dense_ok);
+  launch_maybe_pdl(dense_ok, sddmm_kernel<V, VEC, KC, ARES, FAST>, grid, dim3(kSddmmWarps * 32), s, M, K, W,
+                   row_ptr, col_idx, A, Bt, out, out4, sddmm_pair_on(), N, dense_ok);
 }
 
 #if VS_SDDMM_DENSE_CF > 0
@@ -498,7 +531,7 @@ static cudaError_t launch_sddmm_v(int64_t M, int64_t N, int64_t K, const int32_t
 }
 
 template <int V, bool VEC, int KC, bool ARES, bool FAST = false>
-static void launch_sddmm_batch(const SddmmBatch& b, int num_sms, cudaStream_t s) {
+static void launch_sddmm_batch(const SddmmBatch& b, int num_sms, cudaStream_t s, bool pdl) {
   // VS_SDDMM_OVERSUB (build time): grid = that many times the resident CTAs.  2 is 5% faster
   // for the SDDMM batch alone but 2% slower for the bench step, where the oversubscribed grid
   // competes with the concurrent SpMM / encode branches; default 1.
@@ -507,19 +540,19 @@ static void launch_sddmm_batch(const SddmmBatch& b, int num_sms, cudaStream_t s)
 #endif
   constexpr int over = VS_SDDMM_OVERSUB < 1 ? 1 : VS_SDDMM_OVERSUB;
   dim3 grid((unsigned)(num_sms * sddmm_batched_ctas_per_sm<V, VEC, KC, ARES, FAST>() * over));
-  sddmm_batched_kernel<V, VEC, KC, ARES, FAST><<<grid, kSddmmWarps * 32, 0, s>>>(b);
+  launch_maybe_pdl(pdl, sddmm_batched_kernel<V, VEC, KC, ARES, FAST>, grid, dim3(kSddmmWarps * 32), s, b);
 }
 
 template <int V>
-static void launch_sddmm_batch_v(const SddmmBatch& b, int code, int num_sms, cudaStream_t s) {
+static void launch_sddmm_batch_v(const SddmmBatch& b, int code, int num_sms, cudaStream_t s, bool pdl) {
   switch (code) {
-    case 8 + 2: return launch_sddmm_batch<V, true, 1, false>(b, num_sms, s);
-    case 8 + 3: return launch_sddmm_batch<V, true, 1, true>(b, num_sms, s);
-    case 8 + 4: return launch_sddmm_batch<V, true, 2, false>(b, num_sms, s);
-    case 8 + 5: return launch_sddmm_batch<V, true, 2, true>(b, num_sms, s);
-    case 8 + 6: return launch_sddmm_batch<V, true, 2, true, true>(b, num_sms, s);
-    case 3: return launch_sddmm_batch<V, false, 1, true>(b, num_sms, s);
-    default: return launch_sddmm_batch<V, false, 1, false>(b, num_sms, s);
+    case 8 + 2: return launch_sddmm_batch<V, true, 1, false>(b, num_sms, s, pdl);
+    case 8 + 3: return launch_sddmm_batch<V, true, 1, true>(b, num_sms, s, pdl);
+    case 8 + 4: return launch_sddmm_batch<V, true, 2, false>(b, num_sms, s, pdl);
+    case 8 + 5: return launch_sddmm_batch<V, true, 2, true>(b, num_sms, s, pdl);
+    case 8 + 6: return launch_sddmm_batch<V, true, 2, true, true>(b, num_sms, s, pdl);
+    case 3: return launch_sddmm_batch<V, false, 1, true>(b, num_sms, s, pdl);
+    default: return launch_sddmm_batch<V, false, 1, false>(b, num_sms, s, pdl);
   }
 }
 
@@ -554,7 +587,7 @@ static cudaError_t launch_sddmm_mma_batched(int64_t count, const int64_t* M, con
                                             const int32_t* const* row_ptr,
                                             const int32_t* const* col_idx, const void* const* A,
                                             const void* const* Bt, void* const* out, int num_sms,
-                                            cudaStream_t s);
+                                            cudaStream_t s, bool pdl_first = false);
 
 cudaError_t launch_sddmm_batched(int64_t count, const int64_t* M, const int64_t* N, const int64_t* K,
                                  const int* V, const int32_t* const* row_ptr,
@@ -563,11 +596,14 @@ cudaError_t launch_sddmm_batched(int64_t count, const int64_t* M, const int64_t*
                                  cudaStream_t s) {
   if (!sddmm_tc_on()) {
     // the dense-tile kernel (taking the dense row blocks), then the gather kernels (skipping them)
-    if (VS_SDDMM_DENSE_CF != 0) {
+    bool dense = false;
+    for (int64_t i = 0; i < count && VS_SDDMM_DENSE_CF != 0; ++i)
+      dense = dense || sddmm_dense_eligible(M[i], N[i], K[i], V[i], A[i], Bt[i]);
+    if (dense) {
       const cudaError_t e = launch_sddmm_dense(count, M, N, K, V, row_ptr, col_idx, A, Bt, out, num_sms, s);
       if (e != cudaSuccess) return e;
     }
-    return launch_sddmm_mma_batched(count, M, N, K, V, row_ptr, col_idx, A, Bt, out, num_sms, s);
+    return launch_sddmm_mma_batched(count, M, N, K, V, row_ptr, col_idx, A, Bt, out, num_sms, s, dense);
   }
   std::vector<int64_t> sel[2];
   for (int64_t i = 0; i < count; ++i) sel[sddmm_tc_eligible(K[i], A[i], Bt[i], out[i]) ? 1 : 0].push_back(i);
@@ -597,7 +633,7 @@ static cudaError_t launch_sddmm_mma_batched(int64_t count, const int64_t* M, con
                                             const int32_t* const* row_ptr,
                                             const int32_t* const* col_idx, const void* const* A,
                                             const void* const* Bt, void* const* out, int num_sms,
-                                            cudaStream_t s) {
+                                            cudaStream_t s, bool pdl_first) {
   // group by (V, vector path); keep the caller's order inside a group
   std::vector<std::pair<int, int64_t>> order;
   for (int64_t i = 0; i < count; ++i) {
@@ -625,13 +661,14 @@ static cudaError_t launch_sddmm_mma_batched(int64_t count, const int64_t* M, con
     }
     const int code = key & 15;
     switch (key >> 4) {
-      case 1: launch_sddmm_batch_v<1>(batch, code, num_sms, s); break;
-      case 2: launch_sddmm_batch_v<2>(batch, code, num_sms, s); break;
-      case 4: launch_sddmm_batch_v<4>(batch, code, num_sms, s); break;
-      default: launch_sddmm_batch_v<8>(batch, code, num_sms, s); break;
+      case 1: launch_sddmm_batch_v<1>(batch, code, num_sms, s, pdl_first); break;
+      case 2: launch_sddmm_batch_v<2>(batch, code, num_sms, s, pdl_first); break;
+      case 4: launch_sddmm_batch_v<4>(batch, code, num_sms, s, pdl_first); break;
+      default: launch_sddmm_batch_v<8>(batch, code, num_sms, s, pdl_first); break;
     }
     const cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
+    pdl_first = false;  // later launches follow the gather launch before them plainly
   }
   return cudaSuccess;
 }

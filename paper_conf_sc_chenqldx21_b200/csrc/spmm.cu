@@ -73,10 +73,7 @@ __device__ __forceinline__ uint32_t word(const uint4& v, int j) {
 // for the previous launch of the batch to complete before it exits, so a launch completes only
 // after all earlier launches of the batch did and whatever follows on the stream sees every
 // result.  Both are no-ops for a launch made without the PDL attribute (the batch's first).
-__device__ __forceinline__ void pdl_launch_dependents() {
-  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
-}
-__device__ __forceinline__ void pdl_wait_prior() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+// (pdl_launch_dependents / pdl_wait_prior: common.cuh)
 
 // Windows of the 128-row blocks the dense-tile kernel takes (dense_select.cuh; dkp = the
 // problem's K padded to 64, 0 = not dense-eligible) are skipped, except windows whose col_idx

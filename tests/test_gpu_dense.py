@@ -66,8 +66,8 @@ def run_sddmm(vs, mask, A, Bt, V, out_offset=0):
 
 
 @pytest.mark.parametrize("V", [2, 4, 8])
-@pytest.mark.parametrize("M,N,K", [(256, 256, 64), (300, 200, 136), (128, 640, 256), (200, 300, 512),
-                                   (130, 129, 1000), (512, 1024, 128)])
+@pytest.mark.parametrize("M,N,K", [(256, 256, 256), (300, 200, 264), (128, 640, 256), (200, 300, 512),
+                                   (130, 129, 1000), (512, 1024, 320), (256, 256, 64)])
 def test_sddmm_dense_blocks(vs, V, M, N, K):
     rng = gen.make_rng(f"gdense_sd_{V}_{M}_{N}_{K}")
     mask = gen.colvec_mask(rng, M, N, V, 0.6)
@@ -78,7 +78,7 @@ def test_sddmm_dense_blocks(vs, V, M, N, K):
 
 
 @pytest.mark.parametrize("V", [2, 4, 8])
-@pytest.mark.parametrize("K", [64, 256, 384])
+@pytest.mark.parametrize("K", [64, 256, 384, 1000])
 def test_sddmm_mixed_blocks(vs, V, K):
     rng = gen.make_rng(f"gdense_mix_{V}_{K}")
     M, N = 640, 900
@@ -93,7 +93,7 @@ def test_sddmm_mixed_blocks(vs, V, K):
 def test_sddmm_dense_unaligned_out_and_integer_exact(vs, V):
     """Outputs at an odd element offset (scalar stores) and integer-exact inputs: bitwise."""
     rng = gen.make_rng(f"gdense_int_{V}")
-    M, N, K = 200, 300, 128
+    M, N, K = 200, 300, 256
     mask = gen.colvec_mask(rng, M, N, V, 0.8)
     A = gen.dense_operand(rng, M, K, exact=True)
     Bt = gen.dense_operand(rng, N, K, exact=True)
@@ -104,7 +104,7 @@ def test_sddmm_dense_unaligned_out_and_integer_exact(vs, V):
 @pytest.mark.parametrize("V", [2, 4, 8])
 def test_sddmm_dense_padded_rows_zero(vs, V):
     rng = gen.make_rng(f"gdense_pad_{V}")
-    M, N, K = 128 + 5, 256, 64   # last window of the second row block is padded for V > 1
+    M, N, K = 128 + 5, 256, 256  # last window of the second row block is padded for V > 1
     mask = gen.colvec_mask(rng, M, N, V, 0.9)
     A = gen.dense_operand(rng, M, K)
     Bt = gen.dense_operand(rng, N, K)
@@ -114,6 +114,37 @@ def test_sddmm_dense_padded_rows_zero(vs, V):
     if M % V:
         last = out.reshape(-1, V)[rp[-2]:rp[-1], M % V:]
         assert np.all(last.view(np.uint16) == 0)
+
+
+@pytest.mark.parametrize("V", [2, 4, 8])
+@pytest.mark.parametrize("kind", ["perm", "dup"])
+def test_sddmm_dense_unsorted_windows(vs, V, kind):
+    """Windows whose col_idx is not strictly ascending inside dense row blocks: the dense kernel's
+    per-tile search assumes ascending windows, the gather kernel recomputes such windows in full
+    after it.  Every output vs the oracle on the same (permuted / duplicated)
+    arrays, per vector."""
+    rng = gen.make_rng(f"gdense_unsorted_{V}_{kind}")
+    M, N, K = 384, 640, 256
+    mask = gen.colvec_mask(rng, M, N, V, 0.6)
+    A = gen.dense_operand(rng, M, K)
+    Bt = gen.dense_operand(rng, N, K)
+    rp, ci, _ = oracle.encode(M, N, V, mask=mask)
+    ci = ci.copy()
+    W = len(rp) - 1
+    for w in range(0, W, 3):  # every third window
+        b, e = int(rp[w]), int(rp[w + 1])
+        if e - b < 2:
+            continue
+        if kind == "perm":
+            ci[b:e] = ci[b:e][rng.permutation(e - b)]
+        else:
+            ci[b + 1] = ci[b]  # a duplicate column (same output twice)
+    nnz = int(rp[-1])
+    out = torch.full((nnz * V,), 7.0, dtype=torch.float16, device="cuda")
+    vs.vs_sddmm(M, N, K, V, dev(rp), dev(ci), dev(A), dev(Bt), out)
+    torch.cuda.synchronize()
+    o64, s64 = oracle.sddmm(M, N, K, V, rp, ci, A, Bt)
+    assert_within(host(out), o64, s64, f"unsorted {kind} V{V}")
 
 
 def test_sddmm_dense_deterministic(vs):

@@ -64,59 +64,59 @@ namespace vs {
 namespace dt {
 
 // ================================================================================ SDDMM
-constexpr int kSdThreads = 128;              // 4 warps = the 4 TMEM lane quarters
-constexpr int kSdSlab = 128 * 128;           // bytes: 128 rows x 64 k fp16 (16 KB)
-constexpr int kSdStage = 2 * kSdSlab;        // Bt slab + A slab
+// Persistent warp-specialised kernel, one CTA per SM walking the units blockIdx.x, + gridDim.x, ...
+// Roles (each walks the same unit sequence and skips the gather kernel's row blocks by the same
+// predicate, so the per-role counters of dense units agree):
+//   warp 0      TMA producer: Bt slab + A slab of every 64-wide K block into a kSdStages ring
+//   warp 1      MMA issuer: D[acc] (two 128-column TMEM accumulators) += Bt slab * A slab^T
+//   warps 2-5   search: warp s takes dense units j with j % 4 == s and writes, per window, the
+//               range [lo, hi) of its vectors in the tile's column range into slot s
+//   warps 6-13  epilogue, two groups of 4 warps: group g takes dense units j with j % 2 == g
+//               (= accumulator g): TMEM -> Tt[g] (fp16), then the store pass from Tt[g]
+// so the TMA stream, the searches and the store passes of different units overlap.
+constexpr int kSdU = 128;                      // A rows per unit (MMA N; TMEM columns per accumulator)
+constexpr int kSdBtSlab = 128 * 128;           // bytes: 128 mask columns x 64 k fp16 (16 KB)
+constexpr int kSdASlab = kSdU * 128;           // bytes: 128 A rows x 64 k fp16 (16 KB)
+constexpr int kSdStage = kSdBtSlab + kSdASlab;
 constexpr int kSdStages = 2;
-constexpr int kSdSmem = kSdStages * kSdStage + 1024;  // + 1024-byte alignment slack (SWIZZLE_128B)
-constexpr int kSdCtasPerSm = 3;
-constexpr uint32_t kIdescSd = tc::idesc_f16(128, 128, 0, 0);
-static_assert(128 * 256 <= kSdStages * kSdStage, "Tt tile reuses the stage ring");
+constexpr int kSdSearchWarps = 4;
+constexpr int kSdEpiGroups = 4;
+constexpr int kSdTt = 128 * kSdU * 2;          // 32 KB fp16 tile per epilogue group
+constexpr int kSdThreads = 32 * (2 + kSdSearchWarps + 4 * kSdEpiGroups);  // 448
+constexpr int kSdSmem = kSdStages * kSdStage + kSdEpiGroups * kSdTt + 1024;  // + alignment slack
+constexpr uint32_t kIdescSd = tc::idesc_f16(128, kSdU, 0, 0);
+constexpr int kSdSwz = kSdU / 8 - 1;           // Tt chunk swizzle mask (chunks per 2*kSdU-byte row - 1)
 
 struct alignas(64) SdDesc {
-  CUtensorMap tmA;   // A [M x K] fp16, box {64, 128}, SWIZZLE_128B
+  CUtensorMap tmA;   // A [M x K] fp16, box {64, kSdU}, SWIZZLE_128B
   CUtensorMap tmBt;  // Bt [N x K] fp16, box {64, 128}, SWIZZLE_128B
   int64_t M, N, K, W, n_ct;
   const int32_t* row_ptr;
   const int32_t* col_idx;
   uint16_t* out;
-  int32_t V, out_vec;  // out_vec: out is 2V-byte aligned
+  int32_t V, out_vec, col16;  // out_vec: out is 2V-byte aligned; col16: col_idx 16-byte aligned
 };
 struct SdBatch {
   int count;
+  int64_t unit_begin, unit_end;  // the launch's unit range (<= gridDim.x * kSdListCap units)
   int64_t first_unit[kMaxProb + 1];
   SdDesc d[kMaxProb];
 };
 
-template <int V>
-__device__ __forceinline__ void sd_sample_store(uint32_t a, uint16_t* dst, bool vec) {
-  if (V == 8) {
-    const uint4 t = lds128_u32(a);
-    if (vec) {
-      *reinterpret_cast<uint4*>(dst) = t;
-    } else {
-      const uint32_t w[4] = {t.x, t.y, t.z, t.w};
-#pragma unroll
-      for (int r = 0; r < 8; ++r) dst[r] = (uint16_t)(w[r >> 1] >> (16 * (r & 1)));
-    }
-  } else if (V == 4) {
+// out[e*V .. e*V + V) = the V fp16 values at shared address a (2V contiguous bytes)
+__device__ __forceinline__ void sd_sample_store(uint32_t a, uint16_t* dst, int V, bool vec) {
+  if (vec && V == 8) {
+    *reinterpret_cast<uint4*>(dst) = lds128_u32(a);
+  } else if (vec && V == 4) {
     uint32_t x, y;
     asm volatile("ld.shared.v2.u32 {%0,%1}, [%2];" : "=r"(x), "=r"(y) : "r"(a));
-    if (vec) {
-      *reinterpret_cast<uint2*>(dst) = make_uint2(x, y);
-    } else {
-      dst[0] = (uint16_t)x; dst[1] = (uint16_t)(x >> 16); dst[2] = (uint16_t)y; dst[3] = (uint16_t)(y >> 16);
-    }
-  } else if (V == 2) {
+    *reinterpret_cast<uint2*>(dst) = make_uint2(x, y);
+  } else if (vec && V == 2) {
     uint32_t x;
     asm volatile("ld.shared.u32 %0, [%1];" : "=r"(x) : "r"(a));
-    if (vec) {
-      *reinterpret_cast<uint32_t*>(dst) = x;
-    } else {
-      dst[0] = (uint16_t)x; dst[1] = (uint16_t)(x >> 16);
-    }
+    *reinterpret_cast<uint32_t*>(dst) = x;
   } else {
-    dst[0] = lds16(a);
+    for (int r = 0; r < V; ++r) dst[r] = lds16(a + 2 * r);
   }
 }
 
@@ -156,176 +156,375 @@ __device__ __forceinline__ void kary_lower_bound2(const int32_t* __restrict__ a,
   r2 = l2 + c2;
 }
 
-// Store pass of one unit: warp j takes windows j, j + 4, ... of the block, four windows per
+// Store pass of one unit: warp j takes windows j, j + 4, ... of the unit, eight windows per
 // round with their first 64 vectors' col_idx loads in flight together (lane = vector: coalesced
 // loads, 2V-byte shared load + 2V-byte global store each); the window's vectors in the tile's
 // column range are [lo, hi) (searched before the drain).  A vector whose column is outside the
 // range (possible only in a window that is not ascending) is not stored.
-template <int V>
-__device__ __forceinline__ void sd_store1(const SdDesc& d, uint32_t tt, uint32_t rofs, int e, int col, int c0,
+// Tt[c][r]: 2*kSdU-byte row per mask column c, 16-byte chunk j of it at j ^ (c & kSdSwz).
+__device__ __forceinline__ void sd_store1(const SdDesc& d, uint32_t tt, uint32_t rofs, int e, int col, int c0, int V,
                                           bool vec) {
   const uint32_t c = (uint32_t)(col - c0);
   if (col >= 0 && c < 128u)
-    sd_sample_store<V>(tt + c * 256 + (((rofs >> 3) ^ (c & 15)) << 4) + (rofs & 7) * 2, d.out + (int64_t)e * V, vec);
+    sd_sample_store(tt + c * (2 * kSdU) + (((rofs >> 3) ^ (c & kSdSwz)) << 4) + (rofs & 7) * 2, d.out + (int64_t)e * V, V,
+                    vec);
 }
-template <int V>
+constexpr int kSdStoreWin = 4;  // windows per warp round of the store pass
+constexpr int kSdWarps = 4;     // warps of an epilogue group
 __device__ __forceinline__ void sd_store(const SdDesc& d, uint32_t tt, const int32_t* lo_s, const int32_t* hi_s,
-                                         int nwin, int c0, int warp, int lane) {
+                                         int nwin, int c0, int V, int warp, int lane) {
   const bool vec = d.out_vec != 0;
   const int32_t* __restrict__ ci = d.col_idx;
-  for (int wb = warp; wb < nwin; wb += 16) {
-    int lo[4], hi[4], ca[4], cb[4];
+  for (int wb = warp; wb < nwin; wb += kSdWarps * kSdStoreWin) {
+    int lo[kSdStoreWin], hi[kSdStoreWin], ca[kSdStoreWin], cb[kSdStoreWin];
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      const int wl = wb + 4 * u;
+    for (int u = 0; u < kSdStoreWin; ++u) {
+      const int wl = wb + kSdWarps * u;
       lo[u] = wl < nwin ? lo_s[wl] : 0;
       hi[u] = wl < nwin ? hi_s[wl] : 0;
     }
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
+    for (int u = 0; u < kSdStoreWin; ++u) {
       ca[u] = lo[u] + lane < hi[u] ? __ldg(ci + lo[u] + lane) : -1;
       cb[u] = lo[u] + 32 + lane < hi[u] ? __ldg(ci + lo[u] + 32 + lane) : -1;
     }
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      const uint32_t rofs = (uint32_t)((wb + 4 * u) * V);
-      sd_store1<V>(d, tt, rofs, lo[u] + lane, ca[u], c0, vec);
-      sd_store1<V>(d, tt, rofs, lo[u] + 32 + lane, cb[u], c0, vec);
+    for (int u = 0; u < kSdStoreWin; ++u) {
+      const uint32_t rofs = (uint32_t)((wb + kSdWarps * u) * V);
+      sd_store1(d, tt, rofs, lo[u] + lane, ca[u], c0, V, vec);
+      sd_store1(d, tt, rofs, lo[u] + 32 + lane, cb[u], c0, V, vec);
     }
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {  // windows with more than 64 vectors in the tile (dense ones)
-      const uint32_t rofs = (uint32_t)((wb + 4 * u) * V);
+    for (int u = 0; u < kSdStoreWin; ++u) {  // windows with more than 64 vectors in the tile (dense ones)
+      const uint32_t rofs = (uint32_t)((wb + kSdWarps * u) * V);
       for (int e0 = lo[u] + 64; e0 < hi[u]; e0 += 64) {
         const int e1 = e0 + lane, e2 = e0 + 32 + lane;
         const int c1 = e1 < hi[u] ? __ldg(ci + e1) : -1;
         const int c2 = e2 < hi[u] ? __ldg(ci + e2) : -1;
-        sd_store1<V>(d, tt, rofs, e1, c1, c0, vec);
-        sd_store1<V>(d, tt, rofs, e2, c2, c0, vec);
+        sd_store1(d, tt, rofs, e1, c1, c0, V, vec);
+        sd_store1(d, tt, rofs, e2, c2, c0, V, vec);
       }
     }
   }
 }
 
-__global__ void __launch_bounds__(kSdThreads, kSdCtasPerSm) sddmm_dense_kernel(const __grid_constant__ SdBatch b) {
-  extern __shared__ uint8_t smem_raw[];
-  __shared__ __align__(8) uint64_t full_bar[kSdStages], empty_bar[kSdStages], done_bar;
-  __shared__ uint32_t tmem_base_sh;
-  __shared__ int32_t lo_s[128], hi_s[128];  // per window: its vectors in the tile's column range
-  pdl_launch_dependents();  // the gather kernel that follows may start at once (sddmm.cu)
-  const int64_t u = blockIdx.x;
-  const int p = first_problem(b.first_unit, b.count, u);
-  const SdDesc& d = b.d[p];
-  const int loc = (int)(u - b.first_unit[p]);  // < 2^31: units = ceil(M/128) * ceil(N/128), both < 2^24
-  const int n_ct = (int)d.n_ct;
-  const int rb = loc / n_ct, ct = loc - rb * n_ct;
-  if (!sddmm_rb_dense(d.row_ptr, d.W, d.V, rb, d.N)) return;  // CTA-uniform: the gather kernel's block
+// Store pass, 16-byte col_idx loads (col_idx 16-byte aligned; sd_store otherwise): lane l of warp
+// j loads entries [4l, 4l + 4) of the 16-byte groups covering [lo, hi) of windows j, j + 4, ...,
+// eight windows per round (eight 16-byte loads per lane in flight), and stores the in-range
+// ones; Tt is read with plain shared-memory loads (the compiler hoists them ahead of the
+// stores).  Windows with more than 125 vectors in the tile continue in a loop.
+constexpr int kSdStoreWin4 = 8;
+template <int V>
+__device__ __forceinline__ void sd_out(const SdDesc& d, const uint8_t* tt, uint32_t rofs, int e, int col, int c0,
+                                       bool vec) {
+  const uint32_t c = (uint32_t)(col - c0);
+  if (col < 0 || c >= 128u) return;
+  const uint8_t* a = tt + c * (2 * kSdU) + ((((rofs >> 3) ^ (c & kSdSwz))) << 4) + (rofs & 7) * 2;
+  uint16_t* dst = d.out + (int64_t)e * V;
+  if (vec && V == 8) {
+    *reinterpret_cast<uint4*>(dst) = *reinterpret_cast<const uint4*>(a);
+  } else if (vec && V == 4) {
+    *reinterpret_cast<uint2*>(dst) = *reinterpret_cast<const uint2*>(a);
+  } else if (vec && V == 2) {
+    *reinterpret_cast<uint32_t*>(dst) = *reinterpret_cast<const uint32_t*>(a);
+  } else {
+#pragma unroll
+    for (int r = 0; r < V; ++r) dst[r] = reinterpret_cast<const uint16_t*>(a)[r];
+  }
+}
+// col_idx[e, e + 4) with entries >= h as -1; one 16-byte load when all four are below h (no
+// read past h: the last group of col_idx may end mid-way through a 16-byte block)
+__device__ __forceinline__ int4 sd_ld4(const int32_t* __restrict__ ci, int e, int h) {
+  if (e + 3 < h) return __ldg(reinterpret_cast<const int4*>(ci + e));
+  return make_int4(e < h ? __ldg(ci + e) : -1, e + 1 < h ? __ldg(ci + e + 1) : -1, e + 2 < h ? __ldg(ci + e + 2) : -1, -1);
+}
+template <int V>
+__device__ __forceinline__ void sd_store4(const SdDesc& d, const uint8_t* tt, const int32_t* lo_s, const int32_t* hi_s,
+                                          int nwin, int c0, int warp, int lane) {
+  const bool vec = d.out_vec != 0;
+  const int32_t* __restrict__ ci = d.col_idx;
+  for (int wb = warp; wb < nwin; wb += kSdWarps * kSdStoreWin4) {
+    int lo[kSdStoreWin4], hi[kSdStoreWin4];
+    int4 cv[kSdStoreWin4];
+#pragma unroll
+    for (int u = 0; u < kSdStoreWin4; ++u) {
+      const int wl = wb + kSdWarps * u;
+      lo[u] = wl < nwin ? lo_s[wl] : 0;
+      hi[u] = wl < nwin ? hi_s[wl] : 0;
+    }
+#pragma unroll
+    for (int u = 0; u < kSdStoreWin4; ++u) cv[u] = sd_ld4(ci, (lo[u] & ~3) + 4 * lane, hi[u]);
+#pragma unroll
+    for (int u = 0; u < kSdStoreWin4; ++u) {
+      const uint32_t rofs = (uint32_t)((wb + kSdWarps * u) * V);
+      const int e = (lo[u] & ~3) + 4 * lane;
+      sd_out<V>(d, tt, rofs, e, e >= lo[u] && e < hi[u] ? cv[u].x : -1, c0, vec);
+      sd_out<V>(d, tt, rofs, e + 1, e + 1 >= lo[u] && e + 1 < hi[u] ? cv[u].y : -1, c0, vec);
+      sd_out<V>(d, tt, rofs, e + 2, e + 2 >= lo[u] && e + 2 < hi[u] ? cv[u].z : -1, c0, vec);
+      sd_out<V>(d, tt, rofs, e + 3, e + 3 >= lo[u] && e + 3 < hi[u] ? cv[u].w : -1, c0, vec);
+    }
+#pragma unroll 1
+    for (int u = 0; u < kSdStoreWin4; ++u) {  // windows with vectors past the first 128-entry group row
+      const int wl = wb + kSdWarps * u;
+      if (wl >= nwin) break;
+      const int l = lo_s[wl], h = hi_s[wl];
+      const uint32_t rofs = (uint32_t)(wl * V);
+      for (int g = (l & ~3) + 128; g < h; g += 128) {
+        const int e = g + 4 * lane;
+        const int4 x = sd_ld4(ci, e, h);
+        sd_out<V>(d, tt, rofs, e, e < h ? x.x : -1, c0, vec);
+        sd_out<V>(d, tt, rofs, e + 1, e + 1 < h ? x.y : -1, c0, vec);
+        sd_out<V>(d, tt, rofs, e + 2, e + 2 < h ? x.z : -1, c0, vec);
+        sd_out<V>(d, tt, rofs, e + 3, e + 3 < h ? x.w : -1, c0, vec);
+      }
+    }
+  }
+}
 
+// Unit u of the batch: problem, 128-row block, 128-column tile, and whether the row block is
+// the dense kernel's (dense_select.cuh: the same predicate as sddmm_rb_dense).
+struct SdUnit {
+  int p, rb, ct, nwin;
+  int64_t w0;
+};
+__device__ __forceinline__ void sd_decode(const SdBatch& b, int64_t u, SdUnit& x) {
+  x.p = first_problem(b.first_unit, b.count, u);
+  const SdDesc& d = b.d[x.p];
+  const int loc = (int)(u - b.first_unit[x.p]);  // < 2^31 (sddmm_dense_eligible)
+  const int n_ct = (int)d.n_ct;
+  x.rb = loc / n_ct;
+  x.ct = loc - x.rb * n_ct;
+  int64_t w1;
+  rb_windows(x.rb, d.V, d.W, x.w0, w1);
+  x.nwin = (int)(w1 - x.w0);
+}
+__device__ __forceinline__ bool sd_dense(const SdBatch& b, const SdUnit& x) {
+  const SdDesc& d = b.d[x.p];
+  const int64_t nnz = (int64_t)__ldg(d.row_ptr + x.w0 + x.nwin) - (int64_t)__ldg(d.row_ptr + x.w0);
+  return nnz * (int64_t)VS_SDDMM_DENSE_CF > (int64_t)kDenseRows * (d.n_ct * 128);
+}
+constexpr int kSdListCap = 2048;  // dense units per CTA per launch (the host splits larger launches)
+
+__global__ void __launch_bounds__(kSdThreads, 1) sddmm_dense_kernel(const __grid_constant__ SdBatch b) {
+  extern __shared__ uint8_t smem_raw[];
+  __shared__ __align__(8) uint64_t full_bar[kSdStages], empty_bar[kSdStages];
+  __shared__ __align__(8) uint64_t tfull_bar[kSdEpiGroups], tempty_bar[kSdEpiGroups];
+  __shared__ __align__(8) uint64_t sfull_bar[kSdSearchWarps], sempty_bar[kSdSearchWarps];
+  __shared__ uint32_t tmem_base_sh;
+  __shared__ int32_t lo_s[kSdSearchWarps][kSdU], hi_s[kSdSearchWarps][kSdU];
+  __shared__ int32_t ulist[kSdListCap];  // the CTA's dense units (offsets from b.unit_begin)
+  __shared__ int n_dense_sh;
   const uint32_t smem = (smem_u32(smem_raw) + 1023u) & ~1023u;
+  const uint32_t s_ring = smem, s_tt = smem + kSdStages * kSdStage;
   const int warp = threadIdx.x >> 5, lane = lane_id();
-  const int64_t w0 = rb * (128 / d.V);
-  const int nwin = (int)((w0 + 128 / d.V < d.W ? w0 + 128 / d.V : d.W) - w0);
+
   if (threadIdx.x == 0) {
     for (int s = 0; s < kSdStages; ++s) {
       tc::mbar_init(smem_u32(&full_bar[s]), 1);
       tc::mbar_init(smem_u32(&empty_bar[s]), 1);
     }
-    tc::mbar_init(smem_u32(&done_bar), 1);
+    for (int a = 0; a < kSdEpiGroups; ++a) {
+      tc::mbar_init(smem_u32(&tfull_bar[a]), 1);
+      tc::mbar_init(smem_u32(&tempty_bar[a]), 4);  // one arrive per warp of the epilogue group
+    }
+    for (int s = 0; s < kSdSearchWarps; ++s) {
+      tc::mbar_init(smem_u32(&sfull_bar[s]), 1);
+      tc::mbar_init(smem_u32(&sempty_bar[s]), 1);
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 0) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 128;" ::"r"(
-        smem_u32(&tmem_base_sh)));
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&tmem_base_sh)),
+                 "r"(kSdEpiGroups * kSdU));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  // ---- the CTA's dense units (ascending), evaluated in parallel: one round trip per 448 units
+  // instead of one per unit in every role
+  {
+    const int64_t mine = b.unit_end > b.unit_begin + blockIdx.x
+                             ? ceil_div64(b.unit_end - b.unit_begin - blockIdx.x, gridDim.x) : 0;
+    __shared__ int wcnt[kSdThreads / 32];
+    int running = 0;
+    for (int64_t base = 0; base < mine; base += kSdThreads) {
+      const int64_t idx = base + threadIdx.x;
+      const int64_t u = b.unit_begin + blockIdx.x + idx * gridDim.x;
+      bool dense = false;
+      if (idx < mine) {
+        SdUnit x;
+        sd_decode(b, u, x);
+        dense = sd_dense(b, x);
+      }
+      const unsigned bal = __ballot_sync(0xffffffffu, dense);
+      if (lane == 0) wcnt[warp] = __popc(bal);
+      __syncthreads();
+      int before = running, tot = 0;
+      for (int w = 0; w < kSdThreads / 32; ++w) {
+        if (w < warp) before += wcnt[w];
+        tot += wcnt[w];
+      }
+      if (dense) ulist[before + __popc(bal & ((1u << lane) - 1u))] = (int32_t)(u - b.unit_begin);
+      running += tot;
+      __syncthreads();
+    }
+    if (threadIdx.x == 0) n_dense_sh = running;
   }
   tc::fence_before();
   __syncthreads();
   tc::fence_after();
   const uint32_t tmem = tmem_base_sh;
-  const int KB = (int)ceil_div64(d.K, 64);
-  const int r0 = (int)(rb * 128), c0 = (int)(ct * 128);
+  const int n_dense = n_dense_sh;
 
   if (warp == 0) {
-    // ---- TMA producer: slab kb -> stage kb & 1 (Bt slab, then A slab)
+    // ================================ TMA producer ================================
     if (lane == 0) {
-      for (int kb = 0; kb < KB; ++kb) {
-        const int s = kb & 1;
-        if (kb >= 2) tc::mbar_wait(smem_u32(&empty_bar[s]), ((kb >> 1) - 1) & 1);
-        const uint32_t st = smem + s * kSdStage;
-        tc::mbar_expect_tx(smem_u32(&full_bar[s]), kSdStage);
-        tc::tma_load_2d(st, &d.tmBt, kb * 64, c0, smem_u32(&full_bar[s]));
-        tc::tma_load_2d(st + kSdSlab, &d.tmA, kb * 64, r0, smem_u32(&full_bar[s]));
+      uint32_t it = 0;
+      SdUnit x;
+      for (int li = 0; li < n_dense; ++li) {
+        sd_decode(b, b.unit_begin + ulist[li], x);
+        const SdDesc& d = b.d[x.p];
+        const int KB = (int)ceil_div64(d.K, 64);
+        for (int kb = 0; kb < KB; ++kb, ++it) {
+          const uint32_t s = it % kSdStages, use = it / kSdStages;
+          if (use > 0) tc::mbar_wait(smem_u32(&empty_bar[s]), (use - 1) & 1);
+          const uint32_t st = s_ring + s * kSdStage;
+          tc::mbar_expect_tx(smem_u32(&full_bar[s]), kSdStage);
+          tc::tma_load_2d(st, &d.tmBt, kb * 64, x.ct * 128, smem_u32(&full_bar[s]));
+          tc::tma_load_2d(st + kSdBtSlab, &d.tmA, kb * 64, x.rb * kSdU, smem_u32(&full_bar[s]));
+        }
       }
     }
-    __syncwarp();
   } else if (warp == 1) {
-    // ---- MMA issuer
+    // ================================ MMA issuer ================================
     if (lane == 0) {
-      for (int kb = 0; kb < KB; ++kb) {
-        const int s = kb & 1;
-        tc::mbar_wait(smem_u32(&full_bar[s]), (kb >> 1) & 1);
+      uint32_t it = 0, seq = 0;
+      SdUnit x;
+      for (int li = 0; li < n_dense; ++li) {
+        sd_decode(b, b.unit_begin + ulist[li], x);
+        const SdDesc& d = b.d[x.p];
+        const int KB = (int)ceil_div64(d.K, 64);
+        const uint32_t acc = seq % kSdEpiGroups;
+        tc::mbar_wait(smem_u32(&tempty_bar[acc]), ((seq / kSdEpiGroups) & 1) ^ 1);
         tc::fence_after();
-        const uint32_t st = smem + s * kSdStage;
+        for (int kb = 0; kb < KB; ++kb, ++it) {
+          const uint32_t s = it % kSdStages, use = it / kSdStages;
+          tc::mbar_wait(smem_u32(&full_bar[s]), use & 1);
+          tc::fence_after();
+          const uint32_t st = s_ring + s * kSdStage;
 #pragma unroll
-        for (int k = 0; k < 4; ++k)
-          tc::mma(tmem, tc::sdesc(st + 32 * k, 16, 1024), tc::sdesc(st + kSdSlab + 32 * k, 16, 1024), kIdescSd,
-                  (kb > 0 || k > 0) ? 1u : 0u);
-        tc::commit(smem_u32(&empty_bar[s]));
+          for (int k = 0; k < 4; ++k)
+            tc::mma(tmem + acc * kSdU, tc::sdesc(st + 32 * k, 16, 1024), tc::sdesc(st + kSdBtSlab + 32 * k, 16, 1024),
+                    kIdescSd, (kb > 0 || k > 0) ? 1u : 0u);
+          tc::commit(smem_u32(&empty_bar[s]));
+        }
+        tc::commit(smem_u32(&tfull_bar[acc]));
+        ++seq;
       }
-      tc::commit(smem_u32(&done_bar));
     }
-    __syncwarp();
+  } else if (warp < 2 + kSdSearchWarps) {
+    // ================================ search ================================
+#ifndef VS_SD_EXP
+#define VS_SD_EXP 0
+#endif
+    const int sw = warp - 2;
+    uint32_t seq = 0;
+    SdUnit x;
+    for (int li = 0; li < n_dense; ++li) {
+      if ((int)(seq % kSdSearchWarps) == sw) {
+        sd_decode(b, b.unit_begin + ulist[li], x);
+        const uint32_t use = seq / kSdSearchWarps;
+        tc::mbar_wait(smem_u32(&sempty_bar[sw]), (use & 1) ^ 1);
+        const SdDesc& d = b.d[x.p];
+        const int c0 = x.ct * 128;
+        for (int i = lane; i < (VS_SD_EXP >= 2 ? 0 : x.nwin); i += 32) {
+          int lo, hi;
+          kary_lower_bound2(d.col_idx, __ldg(d.row_ptr + x.w0 + i), __ldg(d.row_ptr + x.w0 + i + 1), c0, c0 + 128, lo,
+                            hi);
+          lo_s[sw][i] = lo;
+          hi_s[sw][i] = hi > lo ? hi : lo;
+        }
+        __syncwarp();
+        if (lane == 0) tc::mbar_arrive(smem_u32(&sfull_bar[sw]));
+      }
+      ++seq;
+    }
   } else {
-    // ---- warps 2-3, while the TMA / MMA run: per window (thread = window), its vectors with a
-    // column in [c0, c0 + 128) are the range [lo, hi) of its (ascending) col_idx
-    for (int i = threadIdx.x - 64; i < nwin; i += kSdThreads - 64) {
-      const int pb = __ldg(d.row_ptr + w0 + i), pe = __ldg(d.row_ptr + w0 + i + 1);
-      int lo, hi;
-      kary_lower_bound2(d.col_idx, pb, pe, c0, c0 + 128, lo, hi);
-      lo_s[i] = lo;
-      hi_s[i] = hi > lo ? hi : lo;
+    // ================================ epilogue ================================
+    const int ew = warp - 2 - kSdSearchWarps;  // 0 .. 4 * kSdEpiGroups - 1
+    const int g = ew >> 2, gw = ew & 3;         // group, warp within the group
+    const int q = warp & 3;                     // TMEM lane quarter (tcgen05.ld: warp % 4)
+    const uint32_t tt = s_tt + g * kSdTt;
+    const int c = 32 * q + lane;                // mask column of this thread in the drain
+    const uint32_t trow = tt + (uint32_t)c * (2 * kSdU);
+    uint32_t seq = 0;
+    SdUnit x;
+    for (int li = 0; li < n_dense; ++li) {
+      if ((int)(seq % kSdEpiGroups) == g) {
+        sd_decode(b, b.unit_begin + ulist[li], x);
+        const SdDesc& d = b.d[x.p];
+        const uint32_t use = seq / kSdEpiGroups;  // this group's use of accumulator g
+        // ---- drain: Tt[c][r] fp16 (RN), rows >= M +0, 16-byte chunks XOR-swizzled by c
+        tc::mbar_wait(smem_u32(&tfull_bar[g]), use & 1);
+        tc::fence_after();
+        const int64_t rows_valid = d.M - (int64_t)x.rb * kSdU;
+#pragma unroll 1
+        for (int j = 0; j < kSdU / 32; ++j) {
+          uint32_t v[32];
+          tc::ld32(tmem + g * kSdU + ((uint32_t)(32 * q) << 16) + 32 * j, v);
+          tc::ld_wait();
+          uint32_t h[16];
+#pragma unroll
+          for (int xx = 0; xx < 16; ++xx) {
+            const int r = 32 * j + 2 * xx;
+            const float f0 = r < rows_valid ? __uint_as_float(v[2 * xx]) : 0.f;
+            const float f1 = r + 1 < rows_valid ? __uint_as_float(v[2 * xx + 1]) : 0.f;
+            h[xx] = f2_to_h2(f0, f1);
+          }
+#pragma unroll
+          for (int m = 0; m < 4; ++m)
+            asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(
+                             trow + ((((uint32_t)(4 * j + m)) ^ (c & kSdSwz)) << 4)),
+                         "r"(h[4 * m]), "r"(h[4 * m + 1]), "r"(h[4 * m + 2]), "r"(h[4 * m + 3])
+                         : "memory");
+        }
+        tc::fence_before();
+        __syncwarp();
+        if (lane == 0) tc::mbar_arrive(smem_u32(&tempty_bar[g]));
+        tc::named_bar(1 + g, 128);  // Tt[g] complete
+        // ---- store pass (slot of the search warp that took this unit)
+        const uint32_t slot = seq % kSdSearchWarps, suse = seq / kSdSearchWarps;
+        tc::mbar_wait(smem_u32(&sfull_bar[slot]), suse & 1);
+#ifndef VS_SD_EXP
+#define VS_SD_EXP 0
+#endif
+        if (VS_SD_EXP == 0) {
+          if (d.col16) {
+            const uint8_t* ttp = smem_raw + (tt - smem_u32(smem_raw));
+            switch (d.V) {
+              case 1: sd_store4<1>(d, ttp, lo_s[slot], hi_s[slot], x.nwin, x.ct * 128, gw, lane); break;
+              case 2: sd_store4<2>(d, ttp, lo_s[slot], hi_s[slot], x.nwin, x.ct * 128, gw, lane); break;
+              case 4: sd_store4<4>(d, ttp, lo_s[slot], hi_s[slot], x.nwin, x.ct * 128, gw, lane); break;
+              default: sd_store4<8>(d, ttp, lo_s[slot], hi_s[slot], x.nwin, x.ct * 128, gw, lane); break;
+            }
+          } else {
+            sd_store(d, tt, lo_s[slot], hi_s[slot], x.nwin, x.ct * 128, d.V, gw, lane);
+          }
+        }
+        tc::named_bar(1 + g, 128);  // Tt[g] and the slot read by the whole group
+        if (gw == 0 && lane == 0) tc::mbar_arrive(smem_u32(&sempty_bar[slot]));
+      }
+      ++seq;
     }
   }
 
-  // ---- drain: thread = mask column c = TMEM lane 32 * warp + lane; Tt[c][r] fp16 over the ring
-  tc::mbar_wait(smem_u32(&done_bar), 0);
-  tc::fence_after();
-  const int c = 32 * warp + lane;
-  const uint32_t trow = smem + (uint32_t)c * 256;
-  const int64_t rows_valid = d.M - r0;  // rows >= M are stored as +0
-#pragma unroll 1
-  for (int j = 0; j < 4; ++j) {
-    uint32_t v[32];
-    tc::ld32(tmem + ((uint32_t)(32 * warp) << 16) + 32 * j, v);
-    tc::ld_wait();
-    uint32_t h[16];
-#pragma unroll
-    for (int x = 0; x < 16; ++x) {
-      const int r = 32 * j + 2 * x;
-      const float f0 = r < rows_valid ? __uint_as_float(v[2 * x]) : 0.f;
-      const float f1 = r + 1 < rows_valid ? __uint_as_float(v[2 * x + 1]) : 0.f;
-      h[x] = f2_to_h2(f0, f1);
-    }
-#pragma unroll
-    for (int m = 0; m < 4; ++m)
-      asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(trow + ((((uint32_t)(4 * j + m)) ^ (c & 15)) << 4)),
-                   "r"(h[4 * m]), "r"(h[4 * m + 1]), "r"(h[4 * m + 2]), "r"(h[4 * m + 3])
-                   : "memory");
-  }
   tc::fence_before();
-  __syncthreads();  // Tt complete, TMEM drained
+  __syncthreads();
   if (warp == 0) {
     tc::fence_after();
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 128;" ::"r"(tmem));
-  }
-  switch (d.V) {
-    case 1: sd_store<1>(d, smem, lo_s, hi_s, nwin, c0, warp, lane); break;
-    case 2: sd_store<2>(d, smem, lo_s, hi_s, nwin, c0, warp, lane); break;
-    case 4: sd_store<4>(d, smem, lo_s, hi_s, nwin, c0, warp, lane); break;
-    default: sd_store<8>(d, smem, lo_s, hi_s, nwin, c0, warp, lane); break;
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(kSdEpiGroups * kSdU));
   }
 }
 
-static cudaError_t launch_sd(const SdBatch& b, cudaStream_t s) {
+static cudaError_t launch_sd(SdBatch& b, int num_sms, cudaStream_t s) {
   static std::once_flag once[64];
   int dev = 0;
   cudaGetDevice(&dev);
@@ -334,8 +533,17 @@ static cudaError_t launch_sd(const SdBatch& b, cudaStream_t s) {
       cudaFuncSetAttribute(sddmm_dense_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kSdSmem);
     });
   const int64_t units = b.first_unit[b.count];
-  if (units > 0) sddmm_dense_kernel<<<(unsigned)units, kSdThreads, kSdSmem, s>>>(b);
-  return cudaGetLastError();
+  const int grid = (int)std::min<int64_t>(num_sms, units);
+  if (grid <= 0) return cudaSuccess;
+  const int64_t per_launch = (int64_t)grid * kSdListCap;
+  for (int64_t u0 = 0; u0 < units; u0 += per_launch) {
+    b.unit_begin = u0;
+    b.unit_end = std::min<int64_t>(units, u0 + per_launch);
+    sddmm_dense_kernel<<<grid, kSdThreads, kSdSmem, s>>>(b);
+    const cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
 }
 
 }  // namespace dt
@@ -344,10 +552,10 @@ static cudaError_t launch_sd(const SdBatch& b, cudaStream_t s) {
 // device): 0 < K with K % 8 == 0 (16-byte TMA row stride), 16-byte aligned A and Bt, row and
 // column counts that fit the int32 TMA coordinates.
 bool sddmm_dense_eligible(int64_t M, int64_t N, int64_t K, int V, const void* A, const void* Bt) {
-  return M > 0 && N > 0 && K >= VS_SDDMM_DENSE_KMIN && K > 0 && V >= 1 && V <= 8 && K % 8 == 0 &&
+  return M > 0 && N > 0 && K > 0 && V >= 1 && V <= 8 && K % 8 == 0 &&
          ((reinterpret_cast<uintptr_t>(A) & 15) == 0) && ((reinterpret_cast<uintptr_t>(Bt) & 15) == 0) &&
          N < (int64_t(1) << 31) && M < (int64_t(1) << 31) && K < (int64_t(1) << 31) &&
-         ceil_div64(M, 128) * ceil_div64(N, 128) < (int64_t(1) << 31);
+         ceil_div64(M, dt::kSdU) * ceil_div64(N, 128) < (int64_t(1) << 31);
 }
 
 // Launches the dense-tile SDDMM over the eligible problems (units of row blocks the cost
@@ -357,25 +565,24 @@ cudaError_t launch_sddmm_dense(int64_t count, const int64_t* M, const int64_t* N
                                const void* const* A, const void* const* Bt, void* const* out, int num_sms,
                                cudaStream_t s) {
   using namespace dt;
-  (void)num_sms;
   SdBatch batch;
   batch.count = 0;
   batch.first_unit[0] = 0;
   auto flush = [&]() -> cudaError_t {
     if (batch.count == 0) return cudaSuccess;
-    const cudaError_t e = launch_sd(batch, s);
+    const cudaError_t e = launch_sd(batch, num_sms, s);
     batch.count = 0;
     batch.first_unit[0] = 0;
     return e;
   };
   for (int64_t i = 0; i < count; ++i) {
     if (!sddmm_dense_eligible(M[i], N[i], K[i], V[i], A[i], Bt[i])) continue;
-    if (batch.first_unit[batch.count] + ceil_div64(M[i], 128) * ceil_div64(N[i], 128) >= (int64_t(1) << 31)) {
+    if (batch.first_unit[batch.count] + ceil_div64(M[i], dt::kSdU) * ceil_div64(N[i], 128) >= (int64_t(1) << 31)) {
       const cudaError_t e = flush();  // one launch's grid stays below 2^31 CTAs
       if (e != cudaSuccess) return e;
     }
     SdDesc& d = batch.d[batch.count];
-    if (!make_kmajor_map(&d.tmA, A[i], M[i], K[i], 128) || !make_kmajor_map(&d.tmBt, Bt[i], N[i], K[i], 128))
+    if (!make_kmajor_map(&d.tmA, A[i], M[i], K[i], kSdU) || !make_kmajor_map(&d.tmBt, Bt[i], N[i], K[i], 128))
       return cudaErrorInvalidValue;
     d.M = M[i];
     d.N = N[i];
@@ -387,7 +594,8 @@ cudaError_t launch_sddmm_dense(int64_t count, const int64_t* M, const int64_t* N
     d.col_idx = col_idx[i];
     d.out = static_cast<uint16_t*>(out[i]);
     d.out_vec = (reinterpret_cast<uintptr_t>(out[i]) & (uintptr_t)(2 * V[i] - 1)) == 0 ? 1 : 0;
-    batch.first_unit[batch.count + 1] = batch.first_unit[batch.count] + ceil_div64(M[i], 128) * d.n_ct;
+    d.col16 = (reinterpret_cast<uintptr_t>(col_idx[i]) & 15) == 0 ? 1 : 0;
+    batch.first_unit[batch.count + 1] = batch.first_unit[batch.count] + ceil_div64(M[i], kSdU) * d.n_ct;
     ++batch.count;
     if (batch.count == kMaxProb) {
       const cudaError_t e = flush();
