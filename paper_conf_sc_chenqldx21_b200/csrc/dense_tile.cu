@@ -400,31 +400,46 @@ cudaError_t launch_sddmm_dense(int64_t count, const int64_t* M, const int64_t* N
 }  // namespace vs
 #endif  // VS_SDDMM_DENSE_CF > 0
 
-#if VS_SPMM_DENSE_CF > 0  // opt-in build only (dense_select.cuh)
+#if VS_SPMM_DENSE_CF > 0
 namespace vs {
 namespace dt {
 
 // ================================================================================ SpMM
-constexpr int kSpRows = 32;            // A / C rows per unit (MMA N)
-constexpr int kATile = kSpRows * 128;  // 32 rows x 64 k fp16 (4 KB)
-constexpr int kSpThreads = 320;        // 10 warps
-constexpr int kSpEpi = 256;            // decode / epilogue threads (warps 2-9)
-constexpr int kSpKbMax = 32;           // K <= 2048: the decoded A tile stays resident
-constexpr int kSpStages = 4;
-constexpr int kBPanel = 64 * 128 * 2;  // B tile: 64 k x 128 n fp16 = 2 slabs of 64 n (16 KB)
-constexpr int kSpSmem = kSpKbMax * kATile + kSpStages * kBPanel + 1024;
-constexpr uint32_t kIdescSp = tc::idesc_f16(128, kSpRows, 1, 0);
+// Unit = (problem, 128-row block): one CTA of 8 warps, one per SM (193 KB of shared memory).
+//  1. decode: the block's stored vectors [P0, P1) (contiguous in col_idx: the windows of the
+//     block) are streamed by all 256 threads (coalesced col_idx / vals loads, a per-thread window
+//     cursor over the block's row_ptr) and scattered into a zeroed dense A tile [128 rows x K]
+//     in shared memory, K-major SWIZZLE_128B (K <= 512: the tile stays resident); a window whose
+//     col_idx is not strictly ascending is flagged (the gather kernel computes it: duplicates
+//     sum there, spmm_skip_window);
+//  2. per N panel of <= 256 columns: D[128 rows x Np] (fp32, TMEM) = A tile * B panel with
+//     tcgen05.mma M = 128, N = Np, K = 16, B MN-major straight from TMA boxes {64 n, 64 k}
+//     (2-stage ring), warp 0 lane 0 issuing the copies, warp 1 lane 0 the MMAs;
+//  3. epilogue: warp w drains TMEM lane quarter w % 4 (thread = row), column half w / 4, fp16
+//     (RN), 16-byte stores of the row into every destination (vs_spmm_scatter), rows >= M and
+//     rows of flagged windows skipped.
+constexpr int kSpU = 128;
+constexpr int kSpKMax = 512;
+constexpr int kSpASlab = kSpU * 128;        // 128 rows x 64 k fp16 (16 KB)
+constexpr int kSpNP = 256;                  // N panel (MMA N, TMEM columns)
+constexpr int kSpBBox = 64 * 128;           // one TMA box: 64 k x 64 n fp16 (8 KB)
+constexpr int kSpBStage = (kSpNP / 64) * kSpBBox;
+constexpr int kSpStages = 2;
+constexpr int kSpThreads = 256;
+constexpr int kSpSmem = (kSpKMax / 64) * kSpASlab + kSpStages * kSpBStage + 1024;
 constexpr int kMaxDst = 8;
+constexpr int kSpUnroll = 4;
 
 struct alignas(64) SpDesc {
   CUtensorMap tmB;  // B [K x N] fp16 (N contiguous), box {64 n, 64 k}, SWIZZLE_128B
-  int64_t M, K, N, W, n_rb;
+  int64_t M, K, N, W;
   const int32_t* row_ptr;
   const int32_t* col_idx;
   const uint16_t* vals;
   uint16_t* C[kMaxDst];
   int64_t ldc;
-  int32_t V, nC;
+  int32_t V, nC, c16, in16;  // c16: every destination and ldc * 2 bytes 16-byte aligned;
+                              // in16: col_idx and vals 16-byte aligned
 };
 struct SpBatch {
   int count;
@@ -432,233 +447,284 @@ struct SpBatch {
   SpDesc d[kMaxProb];
 };
 
-__device__ __forceinline__ bool sp_unit_dense(const SpDesc& d, int64_t rb32) {
-  return rb_is_dense(d.row_ptr, d.W, d.V, rb32 / (kDenseRows / kSpRows), ceil_div64(d.K, 64) * 64,
-                     (int64_t)VS_SPMM_DENSE_CF);
+// byte offset of element (row, k) in the decoded K-major 128-byte-swizzled A tile
+__device__ __forceinline__ uint32_t sp_adec(int row, int k) {
+  const int kk = k & 63, rr = row & 7;
+  return (uint32_t)((k >> 6) * kSpASlab + (row >> 3) * 1024 + rr * 128 + ((((kk >> 3) ^ rr)) << 4) + (kk & 7) * 2);
 }
 
-// byte offset of element (row, k) in the decoded K-major 128-byte-swizzled A tile
-__device__ __forceinline__ uint32_t adec_off(int row, int k) {
-  const int kb = k >> 6, kk = k & 63, rr = row & 7;
-  return (uint32_t)(kb * kATile + (row >> 3) * 1024 + rr * 128 + ((((kk >> 3) ^ rr)) << 4) + (kk & 7) * 2);
+template <int V>
+__device__ __forceinline__ void sp_decode(const SpDesc& d, uint32_t atile, const int32_t* wptr, int nwin,
+                                          int rows_valid, int* uns) {
+  const int P0 = wptr[0], P1 = wptr[nwin];
+  int wl = -1, wend = P0;
+  for (int base = P0 + (int)threadIdx.x; base < P1; base += kSpThreads * kSpUnroll) {
+    int col[kSpUnroll], prev[kSpUnroll];
+    uint16_t hv[kSpUnroll][V];
+#pragma unroll
+    for (int u = 0; u < kSpUnroll; ++u) {
+      const int e = base + kSpThreads * u;
+      col[u] = e < P1 ? __ldg(d.col_idx + e) : -1;
+      prev[u] = (e < P1 && e > P0) ? __ldg(d.col_idx + e - 1) : -1;
+      const uint16_t* src = d.vals + (int64_t)e * V;
+      if (V == 8) {
+        const uint4 t = e < P1 ? __ldg(reinterpret_cast<const uint4*>(src)) : make_uint4(0, 0, 0, 0);
+        const uint32_t w[4] = {t.x, t.y, t.z, t.w};
+#pragma unroll
+        for (int r = 0; r < V; ++r) hv[u][r] = (uint16_t)(w[r >> 1] >> (16 * (r & 1)));
+      } else if (V == 4) {
+        const uint2 t = e < P1 ? __ldg(reinterpret_cast<const uint2*>(src)) : make_uint2(0, 0);
+        const uint32_t w[2] = {t.x, t.y};
+#pragma unroll
+        for (int r = 0; r < V; ++r) hv[u][r] = (uint16_t)(w[r >> 1] >> (16 * (r & 1)));
+      } else if (V == 2) {
+        const uint32_t t = e < P1 ? __ldg(reinterpret_cast<const unsigned int*>(src)) : 0u;
+        hv[u][0] = (uint16_t)t;
+        hv[u][1] = (uint16_t)(t >> 16);
+      } else {
+        hv[u][0] = e < P1 ? __ldg(src) : (uint16_t)0;
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < kSpUnroll; ++u) {
+      const int e = base + kSpThreads * u;
+      if (e >= P1) continue;
+      while (wend <= e) wend = wptr[++wl + 1];
+      if (e > wptr[wl] && prev[u] >= col[u]) atomicOr(&uns[wl], 1);  // not strictly ascending
+#pragma unroll
+      for (int r = 0; r < V; ++r) {
+        const int row = wl * V + r;
+        if (row < rows_valid)
+          asm volatile("st.shared.u16 [%0], %1;" ::"r"(atile + sp_adec(row, col[u])), "h"(hv[u][r]) : "memory");
+      }
+    }
+  }
+}
+
+// Decode with 16-byte loads (col_idx and vals 16-byte aligned): thread t takes the four
+// consecutive vectors [e0, e0 + 4) at e0 = 4t + 1024u (+ 4096 per round) of the 16-byte groups
+// covering [P0, P1), kSpUnroll groups in flight: one int4 of col_idx and V/2 uint4 of vals per
+// group.  The column before a group (ascending check) is the previous lane's last one (shuffle),
+// or a load for lane 0.
+template <int V>
+__device__ __forceinline__ void sp_decode16(const SpDesc& d, uint32_t atile, const int32_t* wptr, int nwin,
+                                            int rows_valid, int* uns) {
+  const int P0 = wptr[0], P1 = wptr[nwin];
+  const int Pa = P0 & ~3;
+  const int lane = lane_id();
+  int wl = -1, wend = P0;
+  constexpr int NV = (4 * V * 2 + 15) / 16;  // uint4 of vals per group (V = 1: half of one)
+  for (int base = Pa + 4 * (int)threadIdx.x; base - 4 * lane < P1; base += 4 * kSpThreads * kSpUnroll) {
+    int4 cv[kSpUnroll];
+    uint4 vv[kSpUnroll][NV];
+    int pv[kSpUnroll];
+#pragma unroll
+    for (int u = 0; u < kSpUnroll; ++u) {
+      const int e = base + 4 * kSpThreads * u;
+      const bool full = e >= P0 && e + 3 < P1;
+      if (full) {
+        cv[u] = __ldg(reinterpret_cast<const int4*>(d.col_idx + e));
+      } else {
+        cv[u] = make_int4(e >= P0 && e < P1 ? __ldg(d.col_idx + e) : -1,
+                          e + 1 >= P0 && e + 1 < P1 ? __ldg(d.col_idx + e + 1) : -1,
+                          e + 2 >= P0 && e + 2 < P1 ? __ldg(d.col_idx + e + 2) : -1,
+                          e + 3 >= P0 && e + 3 < P1 ? __ldg(d.col_idx + e + 3) : -1);
+      }
+      const uint16_t* src = d.vals + (int64_t)e * V;
+      if (full) {
+#pragma unroll
+        for (int q = 0; q < NV; ++q) {
+          if (V == 1) {
+            const uint2 t = __ldg(reinterpret_cast<const uint2*>(src));
+            vv[u][q] = make_uint4(t.x, t.y, 0, 0);
+          } else {
+            vv[u][q] = __ldg(reinterpret_cast<const uint4*>(src) + q);
+          }
+        }
+      } else {  // a partial group: per-entry loads (no read outside [P0, P1))
+        uint32_t w[4 * NV] = {};
+#pragma unroll
+        for (int j = 0; j < 4; ++j)
+#pragma unroll
+          for (int r = 0; r < V; ++r)
+            if (e + j >= P0 && e + j < P1)
+              w[(j * V + r) >> 1] |= (uint32_t)__ldg(src + j * V + r) << (16 * ((j * V + r) & 1));
+#pragma unroll
+        for (int q = 0; q < NV; ++q) vv[u][q] = make_uint4(w[4 * q], w[4 * q + 1], w[4 * q + 2], w[4 * q + 3]);
+      }
+      const int up = __shfl_up_sync(0xffffffffu, cv[u].w, 1);
+      pv[u] = lane > 0 ? up : (e > P0 && e - 1 < P1 ? __ldg(d.col_idx + e - 1) : -1);
+    }
+#pragma unroll
+    for (int u = 0; u < kSpUnroll; ++u) {
+      const int c[4] = {cv[u].x, cv[u].y, cv[u].z, cv[u].w};
+      uint32_t w[4 * NV];
+#pragma unroll
+      for (int q = 0; q < NV; ++q) {
+        w[4 * q] = vv[u][q].x; w[4 * q + 1] = vv[u][q].y; w[4 * q + 2] = vv[u][q].z; w[4 * q + 3] = vv[u][q].w;
+      }
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int e = base + 4 * kSpThreads * u + j;
+        if (e < P0 || e >= P1) continue;
+        while (wend <= e) wend = wptr[++wl + 1];
+        const int prev = j == 0 ? pv[u] : c[j - 1];
+        if (e > wptr[wl] && prev >= c[j]) atomicOr(&uns[wl], 1);  // not strictly ascending
+#pragma unroll
+        for (int r = 0; r < V; ++r) {
+          const int row = wl * V + r;
+          const int hidx = j * V + r;  // half index within the group's vals
+          const uint16_t hv = (uint16_t)(w[hidx >> 1] >> (16 * (hidx & 1)));
+          if (row < rows_valid)
+            asm volatile("st.shared.u16 [%0], %1;" ::"r"(atile + sp_adec(row, c[j])), "h"(hv) : "memory");
+        }
+      }
+    }
+  }
 }
 
 __global__ void __launch_bounds__(kSpThreads, 1) spmm_dense_kernel(const __grid_constant__ SpBatch b) {
   extern __shared__ uint8_t smem_raw[];
-  __shared__ __align__(8) uint64_t full_bar[kSpStages], empty_bar[kSpStages];
-  __shared__ __align__(8) uint64_t tfull_bar[2], tempty_bar[2], afull_bar, aempty_bar;
+  __shared__ __align__(8) uint64_t full_bar[kSpStages], empty_bar[kSpStages], done_bar;
   __shared__ uint32_t tmem_base_sh;
-  __shared__ int32_t wptr[kSpRows + 1];
-  __shared__ int32_t unsorted[kSpRows];
-  const uint32_t smem = (smem_u32(smem_raw) + 1023u) & ~1023u;
-  const uint32_t s_adec = smem;                          // decoded A tile (kSpKbMax x 4 KB)
-  const uint32_t s_stage = smem + kSpKbMax * kATile;     // B stage ring
+  __shared__ int32_t wptr[kSpU + 1];
+  __shared__ int uns[kSpU];
+  pdl_launch_dependents();  // the gather launch that follows may start at once (spmm.cu)
+  const int64_t u = blockIdx.x;
+  const int p = first_problem(b.first_unit, b.count, u);
+  const SpDesc& d = b.d[p];
+  const int rb = (int)(u - b.first_unit[p]);
+  const int V = d.V;
+  int64_t w0, w1;
+  rb_windows(rb, V, d.W, w0, w1);
+  const int nwin = (int)(w1 - w0);
+  for (int i = threadIdx.x; i <= nwin; i += kSpThreads) wptr[i] = __ldg(d.row_ptr + w0 + i);
+  if (threadIdx.x < kSpU) uns[threadIdx.x] = 0;
   const int warp = threadIdx.x >> 5, lane = lane_id();
-  const int64_t total = b.first_unit[b.count];
-
   if (threadIdx.x == 0) {
     for (int s = 0; s < kSpStages; ++s) {
       tc::mbar_init(smem_u32(&full_bar[s]), 1);
       tc::mbar_init(smem_u32(&empty_bar[s]), 1);
     }
-    for (int a = 0; a < 2; ++a) {
-      tc::mbar_init(smem_u32(&tfull_bar[a]), 1);
-      tc::mbar_init(smem_u32(&tempty_bar[a]), 8);
-    }
-    tc::mbar_init(smem_u32(&afull_bar), 1);   // the decoders (one elected arrive)
-    tc::mbar_init(smem_u32(&aempty_bar), 1);  // MMA commit after the unit's last MMA
+    tc::mbar_init(smem_u32(&done_bar), 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  if (warp == 1) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 64;" ::"r"(
-        smem_u32(&tmem_base_sh)));
+  __syncthreads();
+  const int KB = (int)ceil_div64(d.K, 64);
+  if ((int64_t)(wptr[nwin] - wptr[0]) * (int64_t)VS_SPMM_DENSE_CF <= (int64_t)kDenseRows * (KB * 64))
+    return;  // CTA-uniform: a row block of the gather kernel (spmm_skip_window)
+
+  const uint32_t smem = (smem_u32(smem_raw) + 1023u) & ~1023u;
+  const uint32_t s_a = smem, s_ring = smem + (kSpKMax / 64) * kSpASlab;
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&tmem_base_sh)),
+                 "r"(kSpNP));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
   }
+  // zero the A tile (KB slabs), then decode the block's vectors into it
+  for (int x = threadIdx.x; x < KB * kSpASlab / 16; x += kSpThreads)
+    asm volatile("st.shared.v4.u32 [%0], {%1,%1,%1,%1};" ::"r"(s_a + x * 16), "r"(0) : "memory");
+  __syncthreads();
+  const int r0 = rb * kSpU;
+  const int rows_valid = (int)(d.M - r0 < kSpU ? d.M - r0 : kSpU);
+  if (d.in16) {
+    switch (V) {
+      case 1: sp_decode16<1>(d, s_a, wptr, nwin, rows_valid, uns); break;
+      case 2: sp_decode16<2>(d, s_a, wptr, nwin, rows_valid, uns); break;
+      case 4: sp_decode16<4>(d, s_a, wptr, nwin, rows_valid, uns); break;
+      default: sp_decode16<8>(d, s_a, wptr, nwin, rows_valid, uns); break;
+    }
+  } else {
+    switch (V) {
+      case 1: sp_decode<1>(d, s_a, wptr, nwin, rows_valid, uns); break;
+      case 2: sp_decode<2>(d, s_a, wptr, nwin, rows_valid, uns); break;
+      case 4: sp_decode<4>(d, s_a, wptr, nwin, rows_valid, uns); break;
+      default: sp_decode<8>(d, s_a, wptr, nwin, rows_valid, uns); break;
+    }
+  }
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic stores -> tensor core reads
   tc::fence_before();
   __syncthreads();
   tc::fence_after();
   const uint32_t tmem = tmem_base_sh;
+  const int row = 32 * (warp & 3) + lane;  // epilogue: this thread's row (TMEM lane)
+  const bool row_ok = row < rows_valid && uns[row / V] == 0;
+  const int h = warp >> 2;                 // epilogue: column half of the panel
 
-  int p = 0;  // problem cursor
-  auto locate = [&](int64_t u) -> int64_t {
-    while (b.first_unit[p + 1] <= u) ++p;
-    return u - b.first_unit[p];
-  };
-  if (warp == 0) {
-    // ================================ TMA producer (B tiles) ================================
-    uint32_t s = 0, ph = 0;
-    for (int64_t u = blockIdx.x; u < total; u += gridDim.x) {
-      const int64_t rb = locate(u);
-      const SpDesc& d = b.d[p];
-      if (!sp_unit_dense(d, rb)) continue;
-      const int KB = (int)ceil_div64(d.K, 64);
-      for (int64_t n0 = 0; n0 < d.N; n0 += 128) {
-        for (int kb = 0; kb < KB; ++kb) {
-          tc::mbar_wait(smem_u32(&empty_bar[s]), ph ^ 1);
-          if (lane == 0) {
-            const uint32_t st = s_stage + s * kBPanel;
-            tc::mbar_expect_tx(smem_u32(&full_bar[s]), kBPanel);
-            tc::tma_load_2d(st, &d.tmB, (int)n0, kb * 64, smem_u32(&full_bar[s]));
-            tc::tma_load_2d(st + kBPanel / 2, &d.tmB, (int)n0 + 64, kb * 64, smem_u32(&full_bar[s]));
-          }
-          __syncwarp();
-          if (++s == kSpStages) { s = 0; ph ^= 1; }
+  uint32_t it = 0;
+  int panel = 0;
+  for (int64_t n0 = 0; n0 < d.N; n0 += kSpNP, ++panel) {
+    const int np = (int)(d.N - n0 < kSpNP ? ceil_div64(d.N - n0, 64) * 64 : kSpNP);  // MMA N (64-multiple)
+    if (warp == 0) {
+      if (lane == 0) {
+        uint32_t j = it;
+        for (int kb = 0; kb < KB; ++kb, ++j) {
+          const uint32_t s = j % kSpStages, use = j / kSpStages;
+          if (use > 0) tc::mbar_wait(smem_u32(&empty_bar[s]), (use - 1) & 1);
+          const uint32_t st = s_ring + s * kSpBStage;
+          tc::mbar_expect_tx(smem_u32(&full_bar[s]), (uint32_t)(np / 64) * kSpBBox);
+          for (int q = 0; q < np / 64; ++q)
+            tc::tma_load_2d(st + q * kSpBBox, &d.tmB, (int)n0 + 64 * q, kb * 64, smem_u32(&full_bar[s]));
         }
       }
-    }
-  } else if (warp == 1) {
-    // ================================ MMA issuer ================================
-    uint32_t s = 0, ph = 0, au = 0, tile = 0;
-    for (int64_t u = blockIdx.x; u < total; u += gridDim.x) {
-      const int64_t rb = locate(u);
-      const SpDesc& d = b.d[p];
-      if (!sp_unit_dense(d, rb)) continue;
-      const int KB = (int)ceil_div64(d.K, 64);
-      tc::mbar_wait(smem_u32(&afull_bar), au & 1);  // decoded A tile of this unit
-      tc::fence_after();
-      for (int64_t n0 = 0; n0 < d.N; n0 += 128) {
-        const uint32_t acc = tile & 1;
-        tc::mbar_wait(smem_u32(&tempty_bar[acc]), ((tile >> 1) & 1) ^ 1);
-        tc::fence_after();
-        for (int kb = 0; kb < KB; ++kb) {
-          tc::mbar_wait(smem_u32(&full_bar[s]), ph);
-          tc::fence_after();
-          if (lane == 0) {
-            const uint32_t st = s_stage + s * kBPanel;
-            const uint32_t at = s_adec + kb * kATile;
-#pragma unroll
-            for (int k = 0; k < 4; ++k)
-              tc::mma(tmem + acc * kSpRows, tc::sdesc(st + 2048 * k, kBPanel / 2, 1024),
-                      tc::sdesc(at + 32 * k, 16, 1024), kIdescSp, (kb > 0 || k > 0) ? 1u : 0u);
-            tc::commit(smem_u32(&empty_bar[s]));
-          }
-          __syncwarp();
-          if (++s == kSpStages) { s = 0; ph ^= 1; }
-        }
-        if (lane == 0) tc::commit(smem_u32(&tfull_bar[acc]));
-        __syncwarp();
-        ++tile;
-      }
-      if (lane == 0) tc::commit(smem_u32(&aempty_bar));  // A tile free once these MMAs complete
       __syncwarp();
-      ++au;
-    }
-  } else {
-    // ================================ decode + epilogue ================================
-    const int et = threadIdx.x - 64;  // 0..255
-    const int q = warp & 3, h = (warp - 2) >> 2;
-    uint32_t au = 0, tile = 0;
-    for (int64_t u = blockIdx.x; u < total; u += gridDim.x) {
-      const int64_t rb = locate(u);
-      const SpDesc& d = b.d[p];
-      if (!sp_unit_dense(d, rb)) continue;
-      const int V = d.V;
-      const int KB = (int)ceil_div64(d.K, 64);
-      const int64_t i0 = rb * kSpRows;
-      const int64_t w0 = i0 / V;
-      const int64_t w1 = (i0 + kSpRows) / V < d.W ? (i0 + kSpRows) / V : d.W;
-      const int nwin = (int)(w1 - w0);
-      // ---- wait until the previous unit's MMAs released the A tile, then zero it
-      tc::mbar_wait(smem_u32(&aempty_bar), (au & 1) ^ 1);
-      for (int x = et; x < KB * kATile / 16; x += kSpEpi)
-        asm volatile("st.shared.v4.u32 [%0], {%1,%1,%1,%1};" ::"r"(s_adec + x * 16), "r"(0) : "memory");
-      if (et <= nwin) wptr[et] = __ldg(d.row_ptr + w0 + et);
-      if (et < kSpRows) unsorted[et] = 0;
-      tc::named_bar(1, kSpEpi);
-      // ---- decode: one flat pass over the unit's vectors [P0, P1)
-      const int64_t P0 = wptr[0], P1 = wptr[nwin];
-      const int64_t off = (int64_t)((reinterpret_cast<uintptr_t>(d.col_idx) >> 2) & 3);
-      const int64_t Pa = ((P0 + off) & ~(int64_t)3) - off;
-      for (int64_t base = Pa + 4 * et; base < P1; base += 4 * kSpEpi) {
-        int c4[4];
-        if (base >= P0 && base + 3 < P1) {
-          const int4 t = __ldg(reinterpret_cast<const int4*>(d.col_idx + base));
-          c4[0] = t.x; c4[1] = t.y; c4[2] = t.z; c4[3] = t.w;
-        } else {
+    } else if (warp == 1) {
+      if (lane == 0) {
+        const uint32_t idesc = tc::idesc_f16(128, np, 0, 1);
+        uint32_t j = it;
+        for (int kb = 0; kb < KB; ++kb, ++j) {
+          const uint32_t s = j % kSpStages, use = j / kSpStages;
+          tc::mbar_wait(smem_u32(&full_bar[s]), use & 1);
+          tc::fence_after();
+          const uint32_t st = s_ring + s * kSpBStage;
 #pragma unroll
-          for (int j = 0; j < 4; ++j) c4[j] = (base + j >= P0 && base + j < P1) ? __ldg(d.col_idx + base + j) : -1;
+          for (int k = 0; k < 4; ++k)
+            tc::mma(tmem, tc::sdesc(s_a + kb * kSpASlab + 32 * k, 16, 1024), tc::sdesc(st + 2048 * k, kSpBBox, 1024),
+                    idesc, (kb > 0 || k > 0) ? 1u : 0u);
+          tc::commit(smem_u32(&empty_bar[s]));
         }
-        const int64_t pf = base < P0 ? P0 : base;
-        int lo = 0, hi = nwin - 1;
-        while (lo < hi) {
-          const int mid = (lo + hi + 1) >> 1;
-          if (wptr[mid] <= pf) lo = mid; else hi = mid - 1;
-        }
-        int wl = lo;
-        int prev = (pf > wptr[wl] && pf < P1) ? __ldg(d.col_idx + pf - 1) : -1;
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-          const int64_t pp = base + j;
-          if (pp < P0 || pp >= P1) continue;
-          while (wptr[wl + 1] <= pp) { ++wl; prev = -1; }
-          const int c = c4[j];
-          if (c <= prev) atomicOr(&unsorted[wl], 1);
-          prev = c;
-          const uint16_t* src = d.vals + pp * V;
-          uint16_t hv[8];
-          if (V == 8) {
-            const uint4 t = __ldg(reinterpret_cast<const uint4*>(src));
-            hv[0] = t.x & 0xFFFF; hv[1] = t.x >> 16; hv[2] = t.y & 0xFFFF; hv[3] = t.y >> 16;
-            hv[4] = t.z & 0xFFFF; hv[5] = t.z >> 16; hv[6] = t.w & 0xFFFF; hv[7] = t.w >> 16;
-          } else if (V == 4) {
-            const uint2 t = __ldg(reinterpret_cast<const uint2*>(src));
-            hv[0] = t.x & 0xFFFF; hv[1] = t.x >> 16; hv[2] = t.y & 0xFFFF; hv[3] = t.y >> 16;
-          } else {
-            const uint32_t t = __ldg(reinterpret_cast<const unsigned int*>(src));
-            hv[0] = t & 0xFFFF; hv[1] = t >> 16;
-          }
-#pragma unroll
-          for (int r = 0; r < 8; ++r)
-            if (r < V)
-              asm volatile("st.shared.u16 [%0], %1;" ::"r"(s_adec + adec_off(wl * V + r, c)), "h"(hv[r]) : "memory");
-        }
+        tc::commit(smem_u32(&done_bar));
       }
-      // generic-proxy stores -> visible to the tensor core (async proxy), then hand over
-      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-      tc::named_bar(1, kSpEpi);
-      if (et == 0) tc::mbar_arrive(smem_u32(&afull_bar));
-      ++au;
-      // ---- epilogue per 128-column panel: TMEM -> fp16 (RN) -> C rows (every destination)
-      for (int64_t n0 = 0; n0 < d.N; n0 += 128) {
-        const uint32_t acc = tile & 1;
-        tc::mbar_wait(smem_u32(&tfull_bar[acc]), (tile >> 1) & 1);
-        tc::fence_after();
-        uint32_t v[16];
-        asm volatile(
-            "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
-            : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
-              "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]),
-              "=r"(v[15])
-            : "r"(tmem + ((uint32_t)(32 * q) << 16) + acc * kSpRows + 16 * h));
-        tc::ld_wait();
-        tc::fence_before();
-        __syncwarp();
-        if (lane == 0) tc::mbar_arrive(smem_u32(&tempty_bar[acc]));
-        const int64_t n = n0 + 32 * q + lane;
-        if (n < d.N) {
-#pragma unroll
-          for (int x = 0; x < 16; ++x) {
-            const int r = 16 * h + x;
-            const int64_t i = i0 + r;
-            if (i >= d.M || unsorted[r / V]) continue;
-            const uint16_t hv = f_to_h(__uint_as_float(v[x]));
-            for (int dd = 0; dd < d.nC; ++dd) d.C[dd][i * d.ldc + n] = hv;
-          }
-        }
-        ++tile;
-      }
+      __syncwarp();
     }
-  }
-
-  tc::fence_before();
-  __syncthreads();
-  if (warp == 1) {
+    it += KB;
+    // ---- epilogue of the panel
+    tc::mbar_wait(smem_u32(&done_bar), panel & 1);
     tc::fence_after();
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 64;" ::"r"(tmem));
+    for (int c0 = h * (np / 2); c0 < (h + 1) * (np / 2); c0 += 32) {
+      uint32_t v[32];
+      tc::ld32(tmem + ((uint32_t)(32 * (warp & 3)) << 16) + c0, v);
+      tc::ld_wait();
+      if (!row_ok) continue;
+      uint32_t hh[16];
+#pragma unroll
+      for (int x = 0; x < 16; ++x) hh[x] = f2_to_h2(__uint_as_float(v[2 * x]), __uint_as_float(v[2 * x + 1]));
+      for (int dd = 0; dd < d.nC; ++dd) {
+        uint16_t* dst = d.C[dd] + (int64_t)(r0 + row) * d.ldc + n0 + c0;
+#pragma unroll
+        for (int g = 0; g < 4; ++g) {
+          if (n0 + c0 + 8 * g >= d.N) break;  // N % 8 == 0
+          if (d.c16) {
+            *reinterpret_cast<uint4*>(dst + 8 * g) = make_uint4(hh[4 * g], hh[4 * g + 1], hh[4 * g + 2], hh[4 * g + 3]);
+          } else {
+#pragma unroll
+            for (int x = 0; x < 4; ++x) {
+              dst[8 * g + 2 * x] = (uint16_t)hh[4 * g + x];
+              dst[8 * g + 2 * x + 1] = (uint16_t)(hh[4 * g + x] >> 16);
+            }
+          }
+        }
+      }
+    }
+    tc::fence_before();
+    __syncthreads();  // TMEM drained before the next panel's MMAs
+    tc::fence_after();
   }
+  if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(kSpNP));
 }
 
 static cudaError_t launch_sp(const SpBatch& b, int num_sms, cudaStream_t s) {
+  (void)num_sms;
   static std::once_flag once[64];
   int dev = 0;
   cudaGetDevice(&dev);
@@ -667,18 +733,18 @@ static cudaError_t launch_sp(const SpBatch& b, int num_sms, cudaStream_t s) {
       cudaFuncSetAttribute(spmm_dense_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kSpSmem);
     });
   const int64_t units = b.first_unit[b.count];
-  const int grid = (int)std::min<int64_t>(num_sms, units);
-  if (grid > 0) spmm_dense_kernel<<<grid, kSpThreads, kSpSmem, s>>>(b);
+  if (units > 0) spmm_dense_kernel<<<(unsigned)units, kSpThreads, kSpSmem, s>>>(b);
   return cudaGetLastError();
 }
 
 }  // namespace dt
 
 // Problems the dense SpMM path can take at all (the per-row-block choice is made on the
-// device): V >= 2, 0 < K <= 2048 (decoded A tile resident), N % 8 == 0 and 16-byte aligned B
-// (TMA), vals aligned to 2V bytes (one load per vector).
+// device): 0 < K <= 512 (the decoded A tile stays resident), N % 8 == 0 and 16-byte aligned B
+// (TMA), vals aligned to 2V bytes (one load per vector).  Independent of N's size, so every
+// N-panel shard of a problem decides alike.
 bool spmm_dense_eligible(int64_t M, int64_t K, int64_t N, int V, const void* vals, const void* B) {
-  return M > 0 && N > 0 && K > 0 && K <= 64 * dt::kSpKbMax && V >= 2 && N % 8 == 0 &&
+  return M > 0 && N > 0 && K > 0 && K <= dt::kSpKMax && V >= 2 && V <= 8 && N % 8 == 0 &&
          ((reinterpret_cast<uintptr_t>(B) & 15) == 0) &&
          ((reinterpret_cast<uintptr_t>(vals) & (uintptr_t)(2 * V - 1)) == 0) && N < (int64_t(1) << 31) &&
          M < (int64_t(1) << 31);
@@ -709,14 +775,20 @@ cudaError_t launch_spmm_dense(int64_t count, const int64_t* M, const int64_t* K,
     d.N = N[i];
     d.V = V[i];
     d.W = ceil_div64(M[i], V[i]);
-    d.n_rb = ceil_div64(M[i], kSpRows);
     d.row_ptr = row_ptr[i];
     d.col_idx = col_idx[i];
     d.vals = static_cast<const uint16_t*>(vals[i]);
-    for (int k = 0; k < kMaxDst; ++k) d.C[k] = k < nC[i] ? static_cast<uint16_t*>(C_dst[i][k]) : nullptr;
+    bool c16 = (ldc[i] % 8) == 0;
+    for (int k = 0; k < kMaxDst; ++k) {
+      d.C[k] = k < nC[i] ? static_cast<uint16_t*>(C_dst[i][k]) : nullptr;
+      if (k < nC[i]) c16 = c16 && ((reinterpret_cast<uintptr_t>(C_dst[i][k]) & 15) == 0);
+    }
     d.nC = nC[i];
     d.ldc = ldc[i];
-    batch.first_unit[batch.count + 1] = batch.first_unit[batch.count] + d.n_rb;
+    d.c16 = c16 ? 1 : 0;
+    d.in16 = ((reinterpret_cast<uintptr_t>(col_idx[i]) & 15) == 0 && (reinterpret_cast<uintptr_t>(vals[i]) & 15) == 0)
+                 ? 1 : 0;
+    batch.first_unit[batch.count + 1] = batch.first_unit[batch.count] + ceil_div64(M[i], kSpU);
     ++batch.count;
     if (batch.count == kMaxProb) {
       const cudaError_t e = flush();

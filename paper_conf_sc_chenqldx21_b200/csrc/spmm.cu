@@ -313,6 +313,7 @@ __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32)
                 uint16_t* __restrict__ C, int64_t dkp) {
   const CDst<1> cd = {{C}, 1, N};
   spmm_body<V, NC, VEC, SPLIT, UNROLL, 1>(M, N, W, n_wgroups, blockIdx.x, row_ptr, col_idx, vals, B, cd, dkp);
+  pdl_wait_prior();  // completes after a dense-tile launch it overlaps (no-op otherwise)
 }
 
 // vs_spmm_scatter, register path (unaligned operands or destinations, V = 1)
@@ -324,6 +325,7 @@ __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32)
                         const __grid_constant__ CDst<kMaxScatter> cd, int64_t dkp) {
   spmm_body<V, NC, VEC, SPLIT, 1, kMaxScatter>(M, N, W, n_wgroups, blockIdx.x, row_ptr, col_idx,
                                                vals, B, cd, dkp);
+  pdl_wait_prior();  // completes after a dense-tile launch it overlaps (no-op otherwise)
 }
 
 // Batched launch: one grid over the units of up to kSpmmMaxBatch problems that share a
@@ -615,6 +617,7 @@ __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32, CpMinBlocks<SPLIT
   extern __shared__ __align__(128) unsigned char smem[];
   const CDst<1> cd = {{C}, 1, N};
   spmm_cp_body<V, NC, SPLIT, D, 1>(M, N, W, n_wgroups, blockIdx.x, row_ptr, col_idx, vals, B, cd, smem, dkp);
+  pdl_wait_prior();  // completes after a dense-tile launch it overlaps (no-op otherwise)
 }
 
 // vs_spmm_scatter, cp.async path: the same body, every output tile stored into cd.n destinations
@@ -627,6 +630,7 @@ __global__ void __launch_bounds__(SpmmCta<SPLIT>::kWarps * 32, CpMinBlocks<SPLIT
   extern __shared__ __align__(128) unsigned char smem[];
   spmm_cp_body<V, NC, SPLIT, D, kMaxScatter>(M, N, W, n_wgroups, blockIdx.x, row_ptr, col_idx, vals, B,
                                              cd, smem, dkp);
+  pdl_wait_prior();  // completes after a dense-tile launch it overlaps (no-op otherwise)
 }
 
 template <int V, int NC, int SPLIT, int D>
@@ -879,6 +883,27 @@ static cudaError_t launch_spmm_tc(int64_t, const int64_t*, const int64_t*, const
 }
 #endif
 
+// Launch of a gather kernel overlapped (pdl) with the dense-tile kernel launched just before it.
+template <typename... KArgs, typename... Args>
+static cudaError_t spmm_launch(bool pdl, void (*kern)(KArgs...), unsigned grid, int threads, int smem,
+                               cudaStream_t s, Args... args) {
+  if (!pdl) {
+    kern<<<grid, threads, smem, s>>>(args...);
+    return cudaGetLastError();
+  }
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3((unsigned)threads);
+  cfg.dynamicSmemBytes = (size_t)smem;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...);
+}
+
 cudaError_t launch_spmm(int64_t M, int64_t K, int64_t N, int V, const int32_t* row_ptr,
                         const int32_t* col_idx, const void* vals, const void* B, void* C,
                         int num_sms, cudaStream_t s) {
@@ -895,16 +920,17 @@ cudaError_t launch_spmm(int64_t M, int64_t K, int64_t N, int V, const int32_t* r
   if (grid > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
   if (grid == 0) return cudaSuccess;
   const int64_t dkp = spmm_dkp(M, K, N, V, vals, B);
-  k.single<<<(unsigned)grid, k.threads, k.smem, s>>>(M, N, W, nwg, row_ptr, col_idx,
-                                                     static_cast<const uint16_t*>(vals),
-                                                     static_cast<const uint16_t*>(B),
-                                                     static_cast<uint16_t*>(C), dkp);
-  cudaError_t e = cudaGetLastError();
-  if (e != cudaSuccess || dkp == 0) return e;
-  void* dst[1] = {C};
-  void* const* dsts = dst;
-  const int one = 1;
-  return launch_spmm_dense(1, &M, &K, &N, &V, &row_ptr, &col_idx, &vals, &B, &dsts, &one, &N, num_sms, s);
+  if (dkp != 0) {  // dense row blocks first; the gather launch overlaps it
+    void* dst[1] = {C};
+    void* const* dsts = dst;
+    const int one = 1;
+    const cudaError_t de = launch_spmm_dense(1, &M, &K, &N, &V, &row_ptr, &col_idx, &vals, &B, &dsts, &one, &N,
+                                             num_sms, s);
+    if (de != cudaSuccess) return de;
+  }
+  return spmm_launch(dkp != 0, k.single, (unsigned)grid, k.threads, k.smem, s, M, N, W, nwg, row_ptr, col_idx,
+                     static_cast<const uint16_t*>(vals), static_cast<const uint16_t*>(B), static_cast<uint16_t*>(C),
+                     dkp);
 }
 
 // vs_spmm_scatter: the launch of vs_spmm, every output tile stored into n_dst destinations
@@ -931,13 +957,13 @@ cudaError_t launch_spmm_scatter(int64_t M, int64_t K, int64_t N, int V, const in
   if (grid > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
   if (grid == 0) return cudaSuccess;
   const int64_t dkp = spmm_dkp(M, K, N, V, vals, B);
-  k.scatter<<<(unsigned)grid, k.threads, k.smem, s>>>(M, N, W, nwg, row_ptr, col_idx,
-                                                      static_cast<const uint16_t*>(vals),
-                                                      static_cast<const uint16_t*>(B), cd, dkp);
-  cudaError_t e = cudaGetLastError();
-  if (e != cudaSuccess || dkp == 0) return e;
-  return launch_spmm_dense(1, &M, &K, &N, &V, &row_ptr, &col_idx, &vals, &B, &C_dst, &n_dst, &ldc,
-                           num_sms, s);
+  if (dkp != 0) {  // dense row blocks first; the gather launch overlaps it
+    const cudaError_t de = launch_spmm_dense(1, &M, &K, &N, &V, &row_ptr, &col_idx, &vals, &B, &C_dst, &n_dst, &ldc,
+                                             num_sms, s);
+    if (de != cudaSuccess) return de;
+  }
+  return spmm_launch(dkp != 0, k.scatter, (unsigned)grid, k.threads, k.smem, s, M, N, W, nwg, row_ptr, col_idx,
+                     static_cast<const uint16_t*>(vals), static_cast<const uint16_t*>(B), cd, dkp);
 }
 
 // VS_SPMM_PDL (build-time, default 1): the launches of one batched call after the first use programmatic
@@ -978,9 +1004,25 @@ cudaError_t launch_spmm_batched(int64_t count, const int64_t* M, const int64_t* 
   }
   std::stable_sort(order.begin(), order.end(),
                    [](const auto& a, const auto& b) { return a.first < b.first; });
+  // the dense-tile kernel first (it takes the dense row blocks; the gather launches below skip
+  // them and start while it runs: programmatic dependent launch, disjoint output rows)
+  int launched = 0;
+  if (VS_SPMM_DENSE_CF != 0) {
+    bool any = false;
+    for (const auto& o : order)
+      any = any || spmm_dense_eligible(M[o.second], K[o.second], N[o.second], V[o.second], vals[o.second], B[o.second]);
+    if (any) {
+      std::vector<void* const*> dsts(count);
+      std::vector<int> ones(count, 1);
+      for (int64_t j = 0; j < count; ++j) dsts[j] = &C[j];
+      const cudaError_t e = launch_spmm_dense(count, M, K, N, V, row_ptr, col_idx, vals, B, dsts.data(), ones.data(),
+                                              N, num_sms, s);
+      if (e != cudaSuccess) return e;
+      launched = 1;  // the first gather launch overlaps it
+    }
+  }
   SpmmBatch batch;
   size_t i = 0;
-  int launched = 0;
   while (i < order.size()) {
     const SpmmCfg c = order[i].first;
     const SpmmKernels k = pick(c);
@@ -1028,13 +1070,7 @@ cudaError_t launch_spmm_batched(int64_t count, const int64_t* M, const int64_t* 
     const cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
   }
-  // the dense-tile kernel takes the row blocks the gather launches above skipped
-  if (VS_SPMM_DENSE_CF == 0) return cudaSuccess;
-  std::vector<void* const*> dsts(count);
-  std::vector<int> ones(count, 1);
-  for (int64_t i = 0; i < count; ++i) dsts[i] = &C[i];
-  return launch_spmm_dense(count, M, K, N, V, row_ptr, col_idx, vals, B, dsts.data(), ones.data(), N,
-                           num_sms, s);
+  return cudaSuccess;
 }
 
 }  // namespace vs
