@@ -203,6 +203,16 @@ vs_status_t vs_spmm_scatter(int64_t M, int64_t K, int64_t N, int V,
  *     p in window w and wV+r < M; padded rows (wV+r >= M) get +0.0.
  *   The mask only selects positions: no scaling and no multiplication by mask values.
  *   M == 0, N == 0 or nnz_v == 0: no-op.  K == 0: out_vals zero-filled.
+ *   Kernels (DESIGN.md 7.3 / 7.8): the 128-row blocks of the mask whose stored density is
+ *   above V/32, in problems with K >= 256 (and K % 8 == 0, 16-byte aligned A and Bt), are
+ *   computed as dense 128 x 128 tcgen05 tiles and sampled; the other blocks by the
+ *   column-vector gather kernel.  The choice depends only on the block's vectors and on K and
+ *   N, so it is the same for vs_sddmm_batched and for any 128-row-aligned row-window shard
+ *   (same bits).  A window whose col_idx is not strictly ascending inside a dense block is
+ *   recomputed by the gather kernel after the dense kernel (any order and duplicates are
+ *   supported; each stored vector gets its own output).  The call enqueues two kernels
+ *   (the second overlapped with the first by programmatic dependent launch) and completes
+ *   when both have.
  */
 vs_status_t vs_sddmm(int64_t M, int64_t N, int64_t K, int V,
                      const int32_t* row_ptr, const int32_t* col_idx,
