@@ -11,29 +11,27 @@
 //
 // SDDMM  out[p*V + r] = sum_k A[wV+r][k] * Bt[col_idx[p]][k]   (§6)
 //   Unit = (problem, 128-row block rb of A, 128-column tile ct of the mask): one CTA of 4 warps,
-//   non-persistent (3 resident per SM, so one CTA's loads overlap another's MMAs / epilogue).
+//   non-persistent (4 resident per SM, so one CTA's loads overlap another's MMAs / epilogue).
 //   D[128 mask cols x 128 A rows] (fp32, TMEM, 128 columns) = Bt[c0:c0+128, :] * A[r0:r0+128, :]^T
 //   with tcgen05.mma M = 128, N = 128, K = 16 (the operand switch of P:1059-1063: mask columns on
 //   the MMA M side), both operands K-contiguous rows loaded by TMA 2-D tile copies (SWIZZLE_128B
-//   = the canonical K-major layout), a 2-stage ring of 64-wide K slabs (any inner K).  Warp 0
+//   = the canonical K-major layout), a ring of 64-wide K slabs (any inner K; one stage, 4 CTAs per SM).  Warp 0
 //   lane 0 issues the TMA copies, warp 1 lane 0 the MMAs; then every warp drains its TMEM lane
 //   quarter (thread = mask column c) into a shared tile Tt[c][r] (fp16 RN, rows >= M are +0;
 //   each c a 256-byte row, 16-byte chunks XOR-swizzled by c), so the V rows of a window at
-//   column c are 2V contiguous bytes.  Sampling: warp j takes windows j, j+4, ... of the row
-//   block and walks each window's col_idx (16-byte loads); every stored vector whose column
-//   falls in the tile gets one 2V-byte shared load and one 2V-byte global store -- any col_idx
-//   order, duplicates included.
+//   column c are 2V contiguous bytes.  While the TMA / MMA run, warps 2-3 find per window the
+//   range [lo, hi) of its vectors whose column falls in the tile (9-ary search on the ascending
+//   col_idx); the store pass (warp j: windows j, j+4, ...; lanes = consecutive vectors) gives
+//   each of them one 2V-byte shared load and one 2V-byte global store.  A window that is not
+//   strictly ascending is recomputed afterwards by the gather kernel (sddmm.cu).
 //
 // SpMM  C[i][n] = sum_p vals[p*V + i%V] * B[col_idx[p]][n]   (§5)  [opt-in build]
-//   Unit = (problem, 32-row block of A / C).  The unit's stored vectors (contiguous: the
-//   windows of the 32 rows) are decoded once into a dense [32 rows x K] fp16 tile in shared
-//   memory (K-major, 128-byte swizzle; K <= 2048), then for every 128-column panel of B:
-//   D[128 panel cols x 32 rows] (fp32, TMEM) = B[:, n0:n0+128]^T * A_tile^T with tcgen05.mma
-//   M = 128, N = 32, K = 16 (the operand switch of P:858-871: B columns on the MMA M side, B
-//   MN-major straight from TMA 2-D tiles), and the epilogue stores the tile into C (fp16 RN;
-//   to every destination of vs_spmm_scatter).  Absent vectors are exact zeros of the tile.
-//   A window whose col_idx is not strictly ascending (duplicates, any order) is not taken here:
-//   its rows are left to the gather kernel, which checks the same condition.
+//   Unit = (problem, 128-row block of A / C), K <= 512: the block's stored vectors are decoded
+//   into a dense K-major [128 x K] fp16 tile in shared memory (windows that are not strictly
+//   ascending are flagged and left to the gather kernel), then per panel of <= 256 columns
+//   tcgen05.mma M = 128 rows x N = panel with B MN-major from TMA, epilogue to every
+//   vs_spmm_scatter destination (details at spmm_dense_kernel).
+
 #include <cuda.h>
 #include <cudaTypedefs.h>
 
@@ -67,9 +65,15 @@ namespace dt {
 constexpr int kSdThreads = 128;              // 4 warps = the 4 TMEM lane quarters
 constexpr int kSdSlab = 128 * 128;           // bytes: 128 rows x 64 k fp16 (16 KB)
 constexpr int kSdStage = 2 * kSdSlab;        // Bt slab + A slab
-constexpr int kSdStages = 2;
+// 1 stage: 4 CTAs per SM (TMEM: 4 x 128 columns) hide the serial slab round trips better than
+// 2 stages at 3 CTAs per SM (65 KB of shared memory each): DLMC step 0.830 -> 0.824 ms
+// (profiles/r03_dense_sddmm.md)
+#ifndef VS_SD_STAGES
+#define VS_SD_STAGES 1
+#endif
+constexpr int kSdStages = VS_SD_STAGES;
 constexpr int kSdSmem = kSdStages * kSdStage + 1024;  // + 1024-byte alignment slack (SWIZZLE_128B)
-constexpr int kSdCtasPerSm = 3;
+constexpr int kSdCtasPerSm = kSdStages == 1 ? 4 : 3;
 constexpr uint32_t kIdescSd = tc::idesc_f16(128, 128, 0, 0);
 static_assert(128 * 256 <= kSdStages * kSdStage, "Tt tile reuses the stage ring");
 
@@ -245,11 +249,11 @@ __global__ void __launch_bounds__(kSdThreads, kSdCtasPerSm) sddmm_dense_kernel(c
   const int r0 = (int)(rb * 128), c0 = (int)(ct * 128);
 
   if (warp == 0) {
-    // ---- TMA producer: slab kb -> stage kb & 1 (Bt slab, then A slab)
+    // ---- TMA producer: slab kb -> stage kb % kSdStages (Bt slab, then A slab)
     if (lane == 0) {
       for (int kb = 0; kb < KB; ++kb) {
-        const int s = kb & 1;
-        if (kb >= 2) tc::mbar_wait(smem_u32(&empty_bar[s]), ((kb >> 1) - 1) & 1);
+        const int s = kb % kSdStages, use = kb / kSdStages;
+        if (use > 0) tc::mbar_wait(smem_u32(&empty_bar[s]), (use - 1) & 1);
         const uint32_t st = smem + s * kSdStage;
         tc::mbar_expect_tx(smem_u32(&full_bar[s]), kSdStage);
         tc::tma_load_2d(st, &d.tmBt, kb * 64, c0, smem_u32(&full_bar[s]));
@@ -261,8 +265,8 @@ __global__ void __launch_bounds__(kSdThreads, kSdCtasPerSm) sddmm_dense_kernel(c
     // ---- MMA issuer
     if (lane == 0) {
       for (int kb = 0; kb < KB; ++kb) {
-        const int s = kb & 1;
-        tc::mbar_wait(smem_u32(&full_bar[s]), (kb >> 1) & 1);
+        const int s = kb % kSdStages, use = kb / kSdStages;
+        tc::mbar_wait(smem_u32(&full_bar[s]), use & 1);
         tc::fence_after();
         const uint32_t st = smem + s * kSdStage;
 #pragma unroll
