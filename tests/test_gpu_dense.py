@@ -147,6 +147,34 @@ def test_sddmm_dense_unsorted_windows(vs, V, kind):
     assert_within(host(out), o64, s64, f"unsorted {kind} V{V}")
 
 
+def test_sddmm_dense_batched_equals_single(vs):
+    """vs_sddmm_batched == vs_sddmm bit for bit on problems whose row blocks take the dense-tile
+    kernel (inner K >= 256), mixed with gather-only problems in the same batch; every output
+    also within the oracle's tolerance."""
+    rng = gen.make_rng("gdense_batched")
+    cases = [(130, 300, 256, 2, 0.5), (300, 640, 320, 4, 0.4), (512, 384, 512, 8, 0.6),
+             (256, 200, 256, 1, 0.3), (200, 256, 64, 4, 0.5), (384, 512, 264, 2, 0.02)]
+    single, batch, ref = [], [], []
+    for (M, N, K, V, dens) in cases:
+        mask = gen.colvec_mask(rng, M, N, V, dens)
+        A = gen.dense_operand(rng, M, K)
+        Bt = gen.dense_operand(rng, N, K)
+        rp, ci, _ = oracle.encode(M, N, V, mask=mask)
+        nnz = int(rp[-1])
+        o1 = torch.full((max(nnz, 1) * V,), 7.0, dtype=torch.float16, device="cuda")
+        o2 = torch.full_like(o1, 3.0)
+        drp, dci, dA, dBt = dev(rp), dev(ci), dev(A), dev(Bt)
+        vs.vs_sddmm(M, N, K, V, drp, dci, dA, dBt, o1)
+        single.append((o1, nnz * V))
+        batch.append((M, N, K, V, drp, dci, dA, dBt, o2))
+        ref.append(oracle.sddmm(M, N, K, V, rp, ci, A, Bt))
+    vs.vs_sddmm_batched(batch)
+    torch.cuda.synchronize()
+    for (o1, n), b, (o64, s64), c in zip(single, batch, ref, cases):
+        assert torch.equal(o1[:n].view(torch.int16), b[8][:n].view(torch.int16)), c
+        assert_within(host(o1[:n]), o64, s64, f"batched dense {c}")
+
+
 def test_sddmm_dense_deterministic(vs):
     rng = gen.make_rng("gdense_det")
     M, N, K, V = 512, 512, 256, 4
