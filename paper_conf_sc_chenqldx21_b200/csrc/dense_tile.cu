@@ -125,12 +125,40 @@ __device__ __forceinline__ void sd_sample_store(uint32_t a, uint16_t* dst, bool 
 }
 
 // Smallest i in [lo, hi] with a[i] >= x, for two targets at once (a[lo, hi) ascending, a[hi]
-// taken as +inf): 9-ary search, 8 independent probes per target per round trip (a 1024-entry
-// window takes 3 rounds + one of <= 8 loads), so the latency of one thread's search is ~4 L2
-// round trips.  On a window that is not ascending the result is some index in [lo, hi].
+// taken as +inf): 9-ary search, 8 independent probes per target per round trip.  The first
+// round is placed around a guess of each answer (g1, g2: where x would sit if the window's
+// columns were spread evenly), 8 probes dd apart with dd ~ sqrt(n) / 4, so on a random mask it
+// brackets the answer to dd entries and one more round of <= 8 loads finishes: ~2 L2 round
+// trips instead of ~4 for a 1024-entry window.  Any placement of the probes keeps the search
+// exact (it counts the probes below x).  On a window that is not ascending the result is some
+// index in [lo, hi].
 __device__ __forceinline__ void kary_lower_bound2(const int32_t* __restrict__ a, int lo, int hi, int x1, int x2,
-                                                  int& r1, int& r2) {
+                                                  int g1, int g2, int& r1, int& r2) {
   int l1 = lo, h1 = hi, l2 = lo, h2 = hi;
+  const int n = hi - lo;
+  int dd = (int)(sqrtf((float)n) * 0.25f);
+  dd = dd < 1 ? 1 : dd;
+  if (8 * dd <= n && n > 16) {  // guided first round: probes base + dd * i, i = 1..8, inside [lo, hi)
+    auto place = [&](int g) {
+      int base = g - 4 * dd;
+      base = base < lo - 1 ? lo - 1 : base;
+      base = base > hi - 1 - 8 * dd ? hi - 1 - 8 * dd : base;
+      return base;
+    };
+    const int b1 = place(g1), b2 = place(g2);
+    int c1 = 0, c2 = 0;
+#pragma unroll
+    for (int i = 1; i <= 8; ++i) {
+      c1 += __ldg(a + b1 + dd * i) < x1 ? 1 : 0;
+      c2 += __ldg(a + b2 + dd * i) < x2 ? 1 : 0;
+    }
+    const int nh1 = c1 < 8 ? b1 + dd * (c1 + 1) : h1;
+    l1 = c1 > 0 ? b1 + dd * c1 + 1 : l1;
+    h1 = nh1;
+    const int nh2 = c2 < 8 ? b2 + dd * (c2 + 1) : h2;
+    l2 = c2 > 0 ? b2 + dd * c2 + 1 : l2;
+    h2 = nh2;
+  }
   while (h1 - l1 > 8 || h2 - l2 > 8) {
     const int s1 = (h1 - l1) / 9, s2 = (h2 - l2) / 9;
     int c1 = 0, c2 = 0;
@@ -185,21 +213,29 @@ __device__ __forceinline__ void sd_store(const SdDesc& d, uint32_t tt, const int
       lo[u] = wl < nwin ? lo_s[wl] : 0;
       hi[u] = wl < nwin ? hi_s[wl] : 0;
     }
+    // an ascending window has at most 128 vectors in the tile: four 32-vector chunks per window,
+    // all sixteen loads of the round in flight together
+    int cc[4][2];
 #pragma unroll
     for (int u = 0; u < 4; ++u) {
       ca[u] = lo[u] + lane < hi[u] ? __ldg(ci + lo[u] + lane) : -1;
       cb[u] = lo[u] + 32 + lane < hi[u] ? __ldg(ci + lo[u] + 32 + lane) : -1;
+#pragma unroll
+      for (int q = 0; q < 2; ++q)
+        cc[u][q] = lo[u] + 64 + 32 * q + lane < hi[u] ? __ldg(ci + lo[u] + 64 + 32 * q + lane) : -1;
     }
 #pragma unroll
     for (int u = 0; u < 4; ++u) {
       const uint32_t rofs = (uint32_t)((wb + 4 * u) * V);
       sd_store1<V>(d, tt, rofs, lo[u] + lane, ca[u], c0, vec);
       sd_store1<V>(d, tt, rofs, lo[u] + 32 + lane, cb[u], c0, vec);
+#pragma unroll
+      for (int q = 0; q < 2; ++q) sd_store1<V>(d, tt, rofs, lo[u] + 64 + 32 * q + lane, cc[u][q], c0, vec);
     }
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {  // windows with more than 64 vectors in the tile (dense ones)
+    for (int u = 0; u < 4; ++u) {  // past 128 vectors: only a window that is not ascending
       const uint32_t rofs = (uint32_t)((wb + 4 * u) * V);
-      for (int e0 = lo[u] + 64; e0 < hi[u]; e0 += 64) {
+      for (int e0 = lo[u] + 128; e0 < hi[u]; e0 += 64) {
         const int e1 = e0 + lane, e2 = e0 + 32 + lane;
         const int c1 = e1 < hi[u] ? __ldg(ci + e1) : -1;
         const int c2 = e2 < hi[u] ? __ldg(ci + e2) : -1;
@@ -210,24 +246,44 @@ __device__ __forceinline__ void sd_store(const SdDesc& d, uint32_t tt, const int
   }
 }
 
+// Phase timing of the dense SDDMM CTAs (tuning builds only, -DVS_SD_TIMING=1): clock64 at the
+// phase boundaries of the first kSdTimed CTAs of a launch, read back with vs_debug_sd_timing.
+#ifndef VS_SD_TIMING
+#define VS_SD_TIMING 0
+#endif
+#if VS_SD_TIMING
+constexpr int kSdTimed = 8192;
+__device__ unsigned long long g_sd_t[kSdTimed][8];
+#define SD_T(slot) do { if (blockIdx.x < kSdTimed) g_sd_t[blockIdx.x][slot] = clock64(); } while (0)
+#else
+#define SD_T(slot) do { } while (0)
+#endif
+
 __global__ void __launch_bounds__(kSdThreads, kSdCtasPerSm) sddmm_dense_kernel(const __grid_constant__ SdBatch b) {
   extern __shared__ uint8_t smem_raw[];
   __shared__ __align__(8) uint64_t full_bar[kSdStages], empty_bar[kSdStages], done_bar;
   __shared__ uint32_t tmem_base_sh;
   __shared__ int32_t lo_s[128], hi_s[128];  // per window: its vectors in the tile's column range
+  __shared__ int32_t wptr[129];              // row_ptr of the block's windows
   pdl_launch_dependents();  // the gather kernel that follows may start at once (sddmm.cu)
+  if (threadIdx.x == 0) SD_T(0);
   const int64_t u = blockIdx.x;
   const int p = first_problem(b.first_unit, b.count, u);
   const SdDesc& d = b.d[p];
   const int loc = (int)(u - b.first_unit[p]);  // < 2^31: units = ceil(M/128) * ceil(N/128), both < 2^24
   const int n_ct = (int)d.n_ct;
   const int rb = loc / n_ct, ct = loc - rb * n_ct;
-  if (!sddmm_rb_dense(d.row_ptr, d.W, d.V, rb, d.N)) return;  // CTA-uniform: the gather kernel's block
+  const int64_t w0 = rb * (128 / d.V);
+  const int nwin = (int)((w0 + 128 / d.V < d.W ? w0 + 128 / d.V : d.W) - w0);
+  // one round trip: the block's window pointers (the dense / gather decision and the searches)
+  for (int i = threadIdx.x; i <= nwin; i += kSdThreads) wptr[i] = __ldg(d.row_ptr + w0 + i);
+  __syncthreads();
+  // CTA-uniform: a row block of the gather kernel (the predicate of sddmm_rb_dense)
+  if ((int64_t)(wptr[nwin] - wptr[0]) * (int64_t)VS_SDDMM_DENSE_CF <= (int64_t)kDenseRows * (n_ct * 128)) return;
+  if (threadIdx.x == 0) SD_T(1);
 
   const uint32_t smem = (smem_u32(smem_raw) + 1023u) & ~1023u;
   const int warp = threadIdx.x >> 5, lane = lane_id();
-  const int64_t w0 = rb * (128 / d.V);
-  const int nwin = (int)((w0 + 128 / d.V < d.W ? w0 + 128 / d.V : d.W) - w0);
   if (threadIdx.x == 0) {
     for (int s = 0; s < kSdStages; ++s) {
       tc::mbar_init(smem_u32(&full_bar[s]), 1);
@@ -247,6 +303,7 @@ __global__ void __launch_bounds__(kSdThreads, kSdCtasPerSm) sddmm_dense_kernel(c
   const uint32_t tmem = tmem_base_sh;
   const int KB = (int)ceil_div64(d.K, 64);
   const int r0 = (int)(rb * 128), c0 = (int)(ct * 128);
+  if (threadIdx.x == 0) SD_T(2);
 
   if (warp == 0) {
     // ---- TMA producer: slab kb -> stage kb % kSdStages (Bt slab, then A slab)
@@ -282,17 +339,21 @@ __global__ void __launch_bounds__(kSdThreads, kSdCtasPerSm) sddmm_dense_kernel(c
     // ---- warps 2-3, while the TMA / MMA run: per window (thread = window), its vectors with a
     // column in [c0, c0 + 128) are the range [lo, hi) of its (ascending) col_idx
     for (int i = threadIdx.x - 64; i < nwin; i += kSdThreads - 64) {
-      const int pb = __ldg(d.row_ptr + w0 + i), pe = __ldg(d.row_ptr + w0 + i + 1);
+      const int pb = wptr[i], pe = wptr[i + 1];
+      const int64_t nn = pe - pb;
       int lo, hi;
-      kary_lower_bound2(d.col_idx, pb, pe, c0, c0 + 128, lo, hi);
+      kary_lower_bound2(d.col_idx, pb, pe, c0, c0 + 128, pb + (int)(nn * c0 / d.N),
+                        pb + (int)(nn * (c0 + 128) / d.N), lo, hi);
       lo_s[i] = lo;
       hi_s[i] = hi > lo ? hi : lo;
     }
+    if (threadIdx.x == 64) SD_T(3);
   }
 
   // ---- drain: thread = mask column c = TMEM lane 32 * warp + lane; Tt[c][r] fp16 over the ring
   tc::mbar_wait(smem_u32(&done_bar), 0);
   tc::fence_after();
+  if (threadIdx.x == 0) SD_T(4);
   const int c = 32 * warp + lane;
   const uint32_t trow = smem + (uint32_t)c * 256;
   const int64_t rows_valid = d.M - r0;  // rows >= M are stored as +0
@@ -317,6 +378,7 @@ __global__ void __launch_bounds__(kSdThreads, kSdCtasPerSm) sddmm_dense_kernel(c
   }
   tc::fence_before();
   __syncthreads();  // Tt complete, TMEM drained
+  if (threadIdx.x == 0) SD_T(5);
   if (warp == 0) {
     tc::fence_after();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 128;" ::"r"(tmem));
@@ -327,6 +389,10 @@ __global__ void __launch_bounds__(kSdThreads, kSdCtasPerSm) sddmm_dense_kernel(c
     case 4: sd_store<4>(d, smem, lo_s, hi_s, nwin, c0, warp, lane); break;
     default: sd_store<8>(d, smem, lo_s, hi_s, nwin, c0, warp, lane); break;
   }
+#if VS_SD_TIMING
+  __syncthreads();
+  if (threadIdx.x == 0) SD_T(6);
+#endif
 }
 
 static cudaError_t launch_sd(const SdBatch& b, cudaStream_t s) {
@@ -343,6 +409,14 @@ static cudaError_t launch_sd(const SdBatch& b, cudaStream_t s) {
 }
 
 }  // namespace dt
+
+#if VS_SD_TIMING
+// tuning builds only: copies the phase clocks of the last dense SDDMM launch (n CTAs x 8)
+extern "C" int vs_debug_sd_timing(void* host, int n) {
+  if (n > dt::kSdTimed) n = dt::kSdTimed;
+  return (int)cudaMemcpyFromSymbol(host, dt::g_sd_t, (size_t)n * 8 * sizeof(unsigned long long));
+}
+#endif
 
 // Problems the dense SDDMM path can take at all (the per-row-block choice is made on the
 // device): 0 < K with K % 8 == 0 (16-byte TMA row stride), 16-byte aligned A and Bt, row and
