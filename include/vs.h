@@ -210,9 +210,9 @@ vs_status_t vs_spmm_scatter(int64_t M, int64_t K, int64_t N, int V,
  *   N, so it is the same for vs_sddmm_batched and for any 128-row-aligned row-window shard
  *   (same bits).  A window whose col_idx is not strictly ascending inside a dense block is
  *   recomputed by the gather kernel after the dense kernel (any order and duplicates are
- *   supported; each stored vector gets its own output).  The call enqueues two kernels
- *   (the second overlapped with the first by programmatic dependent launch) and completes
- *   when both have.
+ *   supported; each stored vector gets its own output).  The call enqueues two kernels in
+ *   stream order (dense tiles, then the gather kernel, which may start early by programmatic
+ *   dependent launch when the dense grid is small); the call completes when both have.
  */
 vs_status_t vs_sddmm(int64_t M, int64_t N, int64_t K, int V,
                      const int32_t* row_ptr, const int32_t* col_idx,

@@ -65,17 +65,21 @@ namespace dt {
 constexpr int kSdThreads = 128;              // 4 warps = the 4 TMEM lane quarters
 constexpr int kSdSlab = 128 * 128;           // bytes: 128 rows x 64 k fp16 (16 KB)
 constexpr int kSdStage = 2 * kSdSlab;        // Bt slab + A slab
-// 1 stage: 4 CTAs per SM (TMEM: 4 x 128 columns) hide the serial slab round trips better than
-// 2 stages at 3 CTAs per SM (65 KB of shared memory each): DLMC step 0.830 -> 0.824 ms
-// (profiles/r03_dense_sddmm.md)
-#ifndef VS_SD_STAGES
-#define VS_SD_STAGES 1
-#endif
-constexpr int kSdStages = VS_SD_STAGES;
-constexpr int kSdSmem = kSdStages * kSdStage + 1024;  // + 1024-byte alignment slack (SWIZZLE_128B)
-constexpr int kSdCtasPerSm = kSdStages == 1 ? 4 : 3;
+// Ring depth, chosen per launch from the launch's largest K (two instantiations): problems with
+// K <= 256 (<= 4 slabs) one stage, 4 CTAs per SM (TMEM: 4 x 128 columns) -- they hide the serial
+// slab round trips better than 2 stages at 3 CTAs per SM (DLMC step 0.830 -> 0.824 ms); longer K
+// (e.g. the ResNet-50 layers' 3136) three stages at 2 CTAs per SM, so slabs stream instead of one
+// round trip each (profiles/r03_dense_sddmm.md).
+constexpr int kSdStagesShort = 1;
+constexpr int kSdStagesLong = 3;
+constexpr int kSdShortKB = 4;  // slabs a one-stage launch takes (K <= 256)
+template <int S>
+struct SdCfg {
+  static constexpr int kSmem = S * kSdStage + 1024;  // + 1024-byte alignment slack (SWIZZLE_128B)
+  static constexpr int kCtasPerSm = S == 1 ? 4 : (S == 2 ? 3 : 2);
+};
+static_assert(128 * 256 <= kSdStagesShort * kSdStage, "Tt tile reuses the stage ring");  // 32 KB
 constexpr uint32_t kIdescSd = tc::idesc_f16(128, 128, 0, 0);
-static_assert(128 * 256 <= kSdStages * kSdStage, "Tt tile reuses the stage ring");
 
 struct alignas(64) SdDesc {
   CUtensorMap tmA;   // A [M x K] fp16, box {64, 128}, SWIZZLE_128B
@@ -259,7 +263,9 @@ __device__ unsigned long long g_sd_t[kSdTimed][8];
 #define SD_T(slot) do { } while (0)
 #endif
 
-__global__ void __launch_bounds__(kSdThreads, kSdCtasPerSm) sddmm_dense_kernel(const __grid_constant__ SdBatch b) {
+template <int kSdStages>
+__global__ void __launch_bounds__(kSdThreads, SdCfg<kSdStages>::kCtasPerSm)
+    sddmm_dense_kernel(const __grid_constant__ SdBatch b) {
   extern __shared__ uint8_t smem_raw[];
   __shared__ __align__(8) uint64_t full_bar[kSdStages], empty_bar[kSdStages], done_bar;
   __shared__ uint32_t tmem_base_sh;
@@ -395,16 +401,25 @@ __global__ void __launch_bounds__(kSdThreads, kSdCtasPerSm) sddmm_dense_kernel(c
 #endif
 }
 
-static cudaError_t launch_sd(const SdBatch& b, cudaStream_t s) {
+template <int S>
+static void launch_sd_s(const SdBatch& b, int64_t units, cudaStream_t s) {
   static std::once_flag once[64];
   int dev = 0;
   cudaGetDevice(&dev);
   if (dev >= 0 && dev < 64)
     std::call_once(once[dev], [] {
-      cudaFuncSetAttribute(sddmm_dense_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kSdSmem);
+      cudaFuncSetAttribute(sddmm_dense_kernel<S>, cudaFuncAttributeMaxDynamicSharedMemorySize, SdCfg<S>::kSmem);
     });
+  sddmm_dense_kernel<S><<<(unsigned)units, kSdThreads, SdCfg<S>::kSmem, s>>>(b);
+}
+
+static cudaError_t launch_sd(const SdBatch& b, cudaStream_t s) {
   const int64_t units = b.first_unit[b.count];
-  if (units > 0) sddmm_dense_kernel<<<(unsigned)units, kSdThreads, kSdSmem, s>>>(b);
+  if (units <= 0) return cudaSuccess;
+  int64_t kb_max = 0;
+  for (int i = 0; i < b.count; ++i) kb_max = std::max<int64_t>(kb_max, ceil_div64(b.d[i].K, 64));
+  if (kb_max <= kSdShortKB) launch_sd_s<kSdStagesShort>(b, units, s);
+  else launch_sd_s<kSdStagesLong>(b, units, s);
   return cudaGetLastError();
 }
 

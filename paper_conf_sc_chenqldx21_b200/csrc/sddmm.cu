@@ -264,8 +264,9 @@ __device__ __forceinline__ void sddmm_window_any(int64_t M, int64_t K,
 // whose col_idx is not strictly ascending: the dense kernel finds a window's vectors of each
 // column tile by a search that assumes ascending order, so such a window (rare: the encoder
 // emits ascending windows) is computed here in full by the warp of its first item, after the
-// dense kernel has completed (this kernel follows it on the stream, overlapped by programmatic
-// dependent launch: the warp waits for it with griddepcontrol.wait), overwriting its writes.
+// dense kernel has completed (this kernel follows it on the stream; when the two overlap by
+// programmatic dependent launch the warp waits for it with griddepcontrol.wait), overwriting its
+// writes.
 // Returns the q to use for the item, 0 to skip it, or -1 for such a window.
 __device__ __forceinline__ int64_t sddmm_gather_q(bool dense_ok, int64_t N, int V, int64_t W,
                                                   const int32_t* __restrict__ row_ptr,
@@ -454,13 +455,23 @@ static int sddmm_batched_ctas_per_sm() {
   return n;
 }
 
-// Launch, overlapped with the dense-tile kernel just launched on the stream (pdl = true:
-// programmatic dependent launch; the gather kernel's blocks start while it runs and complete
-// after it, see sddmm_gather_q) or plainly.
+// Launch after the dense-tile kernel just launched on the stream: overlapped with it by
+// programmatic dependent launch (pdl: the gather kernel's blocks start while it runs and
+// complete after it, see sddmm_gather_q), or plainly (stream order).
+// VS_SDDMM_PDL (build time, default 1): the gather kernel follows a dense-tile launch of at most
+// kSddmmPdlMaxUnits units (CTAs) with programmatic dependent launch.  Measured (profiles/
+// r03_dense_sddmm.md): single calls ~5 % faster and the ResNet-50 layer step 0.954 -> ~0.90 ms,
+// but back-to-back C5 steps (a 65536-CTA dense grid ahead of the persistent gather grid)
+// 110 -> 171 ms, so launches with larger dense grids follow plainly (stream order).
+#ifndef VS_SDDMM_PDL
+#define VS_SDDMM_PDL 1
+#endif
+constexpr int64_t kSddmmPdlMaxUnits = 8192;
+static int64_t sddmm_dense_units(int64_t M, int64_t N) { return ceil_div64(M, 128) * ceil_div64(N, 128); }
 template <typename... KArgs, typename... Args>
 static void launch_maybe_pdl(bool pdl, void (*kern)(KArgs...), dim3 grid, dim3 block, cudaStream_t s,
                              Args... args) {
-  if (!pdl) {
+  if (!pdl || !VS_SDDMM_PDL) {
     kern<<<grid, block, 0, s>>>(args...);
     return;
   }
@@ -480,11 +491,11 @@ static void launch_maybe_pdl(bool pdl, void (*kern)(KArgs...), dim3 grid, dim3 b
 template <int V, bool VEC, int KC, bool ARES, bool FAST = false>
 static void launch_sddmm_one(int64_t M, int64_t K, const int32_t* row_ptr, const int32_t* col_idx,
                              const uint16_t* A, const uint16_t* Bt, uint16_t* out, int num_sms,
-                             cudaStream_t s, int64_t N, bool dense_ok) {
+                             cudaStream_t s, int64_t N, bool dense_ok, bool pdl) {
   const int64_t W = ceil_div64(M, V);
   const bool out4 = (reinterpret_cast<uintptr_t>(out) & 3) == 0;
   dim3 grid((unsigned)(num_sms * sddmm_ctas_per_sm<V, VEC, KC, ARES, FAST>()));
-  launch_maybe_pdl(dense_ok, sddmm_kernel<V, VEC, KC, ARES, FAST>, grid, dim3(kSddmmWarps * 32), s, M, K, W,
+  launch_maybe_pdl(pdl, sddmm_kernel<V, VEC, KC, ARES, FAST>, grid, dim3(kSddmmWarps * 32), s, M, K, W,
                    row_ptr, col_idx, A, Bt, out, out4, sddmm_pair_on(), N, dense_ok);
 }
 
@@ -509,6 +520,7 @@ static cudaError_t launch_sddmm_v(int64_t M, int64_t N, int64_t K, const int32_t
                                   uint16_t* out, bool vec, int num_sms, cudaStream_t s) {
   const int V_ = V;
   const bool dok = sddmm_dense_eligible(M, N, K, V, A, Bt);
+  const bool pdl = dok && sddmm_dense_units(M, N) <= kSddmmPdlMaxUnits;
   if (dok) {
     // dense row blocks first (short non-persistent CTAs); the persistent gather grid then
     // takes the remaining row blocks
@@ -519,13 +531,13 @@ static cudaError_t launch_sddmm_v(int64_t M, int64_t N, int64_t K, const int32_t
     if (de != cudaSuccess) return de;
   }
   switch ((vec ? 8 : 0) + sddmm_variant(K, vec)) {
-    case 8 + 2: launch_sddmm_one<V, true, 1, false>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok); break;
-    case 8 + 3: launch_sddmm_one<V, true, 1, true>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok); break;
-    case 8 + 4: launch_sddmm_one<V, true, 2, false>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok); break;
-    case 8 + 5: launch_sddmm_one<V, true, 2, true>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok); break;
-    case 8 + 6: launch_sddmm_one<V, true, 2, true, true>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok); break;
-    case 3: launch_sddmm_one<V, false, 1, true>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok); break;
-    default: launch_sddmm_one<V, false, 1, false>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok); break;
+    case 8 + 2: launch_sddmm_one<V, true, 1, false>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok, pdl); break;
+    case 8 + 3: launch_sddmm_one<V, true, 1, true>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok, pdl); break;
+    case 8 + 4: launch_sddmm_one<V, true, 2, false>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok, pdl); break;
+    case 8 + 5: launch_sddmm_one<V, true, 2, true>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok, pdl); break;
+    case 8 + 6: launch_sddmm_one<V, true, 2, true, true>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok, pdl); break;
+    case 3: launch_sddmm_one<V, false, 1, true>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok, pdl); break;
+    default: launch_sddmm_one<V, false, 1, false>(M, K, row_ptr, col_idx, A, Bt, out, num_sms, s, N, dok, pdl); break;
   }
   return cudaGetLastError();
 }
@@ -597,13 +609,18 @@ cudaError_t launch_sddmm_batched(int64_t count, const int64_t* M, const int64_t*
   if (!sddmm_tc_on()) {
     // the dense-tile kernel (taking the dense row blocks), then the gather kernels (skipping them)
     bool dense = false;
+    int64_t units = 0;
     for (int64_t i = 0; i < count && VS_SDDMM_DENSE_CF != 0; ++i)
-      dense = dense || sddmm_dense_eligible(M[i], N[i], K[i], V[i], A[i], Bt[i]);
+      if (sddmm_dense_eligible(M[i], N[i], K[i], V[i], A[i], Bt[i])) {
+        dense = true;
+        units += sddmm_dense_units(M[i], N[i]);
+      }
     if (dense) {
       const cudaError_t e = launch_sddmm_dense(count, M, N, K, V, row_ptr, col_idx, A, Bt, out, num_sms, s);
       if (e != cudaSuccess) return e;
     }
-    return launch_sddmm_mma_batched(count, M, N, K, V, row_ptr, col_idx, A, Bt, out, num_sms, s, dense);
+    return launch_sddmm_mma_batched(count, M, N, K, V, row_ptr, col_idx, A, Bt, out, num_sms, s,
+                                    dense && units <= kSddmmPdlMaxUnits);
   }
   std::vector<int64_t> sel[2];
   for (int64_t i = 0; i < count; ++i) sel[sddmm_tc_eligible(K[i], A[i], Bt[i], out[i]) ? 1 : 0].push_back(i);
