@@ -51,7 +51,7 @@ def parse_args(argv=None):
     ap.add_argument("--workload", default=None,
                     help="default: dlmc_layer at --gpus 1 (configs[1] x configs[2]); c5 at --gpus N > 1 "
                          "(configs[4], the case that shards)")
-    ap.add_argument("--priority", choices=["none", "first", "sddmm", "encode"], default="sddmm",
+    ap.add_argument("--priority", choices=["none", "first", "sddmm", "encode"], default="first",
                     help="high stream priority for part of the chain schedule (see step_chains)")
     ap.add_argument("--schedule", choices=["chains", "phases"], default="chains",
                     help="batched step as one chain per V group on concurrent branches, or as "
@@ -524,9 +524,10 @@ def run_ours(args):
             vs.make_spmm_batch([(b.p.M, b.p.K, b.p.N, b.p.V, b.row_ptr, b.col_idx, b.vals, b.X, b.Y) for b in gb]),
             vs.make_sddmm_batch([(b.p.M, b.p.K, b.p.N, b.p.V, b.row_ptr, b.col_idx, b.G, b.X, b.dW) for b in gb])))
     # --priority: which chain streams get the high stream priority (captured into the graph's
-    # kernel nodes): "first" = the V = 2 chain (its SDDMM is the longest), "sddmm" = every
-    # SDDMM branch (default: 0.916 -> 0.902 ms per step, profiles/r01g_priority.md), "encode" =
-    # every encode -> SpMM branch, "none" = all default.
+    # kernel nodes): "first" = the V = 2 chain (its SDDMM and SpMM are the longest; default since
+    # the dense-tile SDDMM: 0.829 -> 0.819 ms per step, profiles/r03_dense_sddmm.md), "sddmm" =
+    # every SDDMM branch (round 1's default: 0.916 -> 0.902 ms, profiles/r01g_priority.md),
+    # "encode" = every encode -> SpMM branch, "none" = all default.
     def _prio(i, side):
         hi = {"first": i == 0, "sddmm": side, "encode": not side}.get(args.priority, False)
         return torch.cuda.Stream(priority=-1) if hi else torch.cuda.Stream()
