@@ -175,6 +175,32 @@ def test_sddmm_dense_batched_equals_single(vs):
         assert_within(host(o1[:n]), o64, s64, f"batched dense {c}")
 
 
+def test_sddmm_dense_batched_many_problems(vs):
+    """More dense-eligible problems than one dense launch takes (32): several dense launches in one
+    batched call, then the gather launch; every output vs the oracle, batch == single bitwise."""
+    rng = gen.make_rng("gdense_many")
+    single, batch, ref = [], [], []
+    for i in range(40):
+        M, N, K, V = int(rng.integers(64, 300)), int(rng.integers(64, 400)), 256, int(rng.choice([2, 4, 8]))
+        mask = gen.colvec_mask(rng, M, N, V, 0.5)
+        A = gen.dense_operand(rng, M, K)
+        Bt = gen.dense_operand(rng, N, K)
+        rp, ci, _ = oracle.encode(M, N, V, mask=mask)
+        nnz = int(rp[-1])
+        o1 = torch.full((max(nnz, 1) * V,), 7.0, dtype=torch.float16, device="cuda")
+        o2 = torch.full_like(o1, 3.0)
+        drp, dci, dA, dBt = dev(rp), dev(ci), dev(A), dev(Bt)
+        vs.vs_sddmm(M, N, K, V, drp, dci, dA, dBt, o1)
+        single.append((o1, nnz * V))
+        batch.append((M, N, K, V, drp, dci, dA, dBt, o2))
+        ref.append(oracle.sddmm(M, N, K, V, rp, ci, A, Bt))
+    vs.vs_sddmm_batched(batch)
+    torch.cuda.synchronize()
+    for (o1, n), b, (o64, s64) in zip(single, batch, ref):
+        assert torch.equal(o1[:n].view(torch.int16), b[8][:n].view(torch.int16))
+        assert_within(host(b[8][:n]), o64, s64, "many")
+
+
 def test_sddmm_dense_deterministic(vs):
     rng = gen.make_rng("gdense_det")
     M, N, K, V = 512, 512, 256, 4
