@@ -1613,7 +1613,8 @@ def run_train(args):
                                    "a parallel branch",
                        "l2": "warm (per-step graph timing, min of steps)"},
             "dense_step_ms": t_dense, "speedup_vs_dense": t_dense / t_sparse,
-            "gpu_launches": len(layers) * 2 + 3 * 3, "clocks": clk, "e2e": None}
+            # + 1: the dense-tile SDDMM launch ahead of the dW gather launch (inner N = 256 >= 256)
+            "gpu_launches": len(layers) * 2 + 3 * 3 + 1, "clocks": clk, "e2e": None}
     print(json.dumps(line), flush=True)
     return 0
 
