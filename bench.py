@@ -1202,7 +1202,10 @@ def run_c5(args):
                             "frac": gb / (cls[dom] * 1e-3) / 1e9 / GATHER_PEAK_GBS, "kernel": dom,
                             "peak_source": "measured: tools/gather_bench.cu ldg_line (profiles/r01e_gather.md)"},
         "kernels": {k: {"ms": v} for k, v in cls.items()},
-        "gpu_launches": 8 * args.steps,
+        # per step: encode A (count, scan, compact), SpMM, encode the mask rows (count, scan, compact
+        # without values), the dense-tile SDDMM launch (inner K >= 256: its CTAs find no dense block
+        # at 10 % density / V = 8 and exit) and the gather SDDMM
+        "gpu_launches": 9 * args.steps,
         "clocks": clk,
         "parity_gate": gate,
         "replicated_output": rep_out,

@@ -466,7 +466,7 @@ static int sddmm_batched_ctas_per_sm() {
 #ifndef VS_SDDMM_PDL
 #define VS_SDDMM_PDL 1
 #endif
-constexpr int64_t kSddmmPdlMaxUnits = 8192;
+constexpr int64_t kSddmmPdlMaxUnits = 4096;  // DLMC V groups 1088, ResNet-50 layers 1532; C5 >= 8192 per rank
 static int64_t sddmm_dense_units(int64_t M, int64_t N) { return ceil_div64(M, 128) * ceil_div64(N, 128); }
 template <typename... KArgs, typename... Args>
 static void launch_maybe_pdl(bool pdl, void (*kern)(KArgs...), dim3 grid, dim3 block, cudaStream_t s,
